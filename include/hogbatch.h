@@ -1,0 +1,209 @@
+/*
+ * hogbatch.h — C ABI of libhogbatch.so, the B200 (sm_100a) hot path of
+ * Adaptive Hogbatch (Ma, Rusu, Wu, Sim, IPDPSW/MARWS 2021; /root/reference/PAPER.md).
+ *
+ * Every entry point returns an int status: HB_OK (0) or a negative HB_E* code;
+ * hb_last_error() returns a thread-local human-readable message for the last
+ * failure on the calling thread.  No C++ exception crosses this boundary.
+ * No torch types appear here: device memory is passed as raw pointers (the
+ * Python binding allocates it with torch), streams as cudaStream_t cast to void*.
+ *
+ * Notation (§III): an MLP with L weight layers and widths
+ * n_0 = d_in, n_1..n_{L-1} hidden, n_L = C classes.  Layer l (1-based) holds
+ * W_l in R^{n_l x n_{l-1}} (the paper's W^l in R^{d_{l+1} x d_l}, row-major
+ * [out, in]) and a bias b_l in R^{n_l}.  Hidden activation: sigmoid; output:
+ * softmax with cross-entropy loss (L258).  The batch loss is the mean over
+ * the batch (R10).
+ */
+#ifndef HOGBATCH_H
+#define HOGBATCH_H
+
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+#define HB_ABI_VERSION 1
+
+/* status codes */
+enum {
+  HB_OK = 0,
+  HB_EINVAL = -1,       /* bad argument (size, pointer, dtype, state)          */
+  HB_ENOMEM = -2,       /* device or host allocation failed                    */
+  HB_ECUDA = -3,        /* a CUDA runtime/driver call failed (message captured) */
+  HB_ENCCL = -4,        /* an NCCL call failed                                 */
+  HB_ESTATE = -5,       /* call not valid in the object's current state        */
+  HB_EUNSUPPORTED = -6  /* valid request this build does not implement         */
+};
+
+/* hidden activation F_l (sigmoid) */
+enum { HB_SIGMOID = 0 };
+
+/* arithmetic of a model (fixed at creation) */
+enum {
+  HB_PREC_BF16 = 0,      /* tcgen05 tensor cores: bf16 operands, fp32 accumulate, fp32 master */
+  HB_PREC_FP32_CHECK = 1 /* fp32 CUDA-core check mode (SIMT GEMMs, fp32 activations)          */
+};
+
+/* dtype of the input matrix X */
+enum { HB_BF16 = 0, HB_F32 = 1 };
+
+/* scheduling policies (§VI) */
+enum {
+  HB_MINIBATCH = 0, /* one worker, fixed b: mini-batch SGD (L55–L56, L262)            */
+  HB_HOGBATCH = 1,  /* Algorithm 1: every worker gets the same b (L147–L170)          */
+  HB_STATIC = 2,    /* CPU+GPU Hogbatch: fixed per-worker b (L172–L179)               */
+  HB_ADAPTIVE = 3   /* Algorithm 2: adaptive per-worker b (L181–L238)                 */
+};
+
+/* Algorithm 2 readings (R3, R21) */
+enum { HB_RESET_FASTEST = 0, HB_RESET_NONE = 1 };          /* u^E <- min_u in the "fastest" branch, or never */
+enum { HB_CREDIT_DISPATCH = 0, HB_CREDIT_COMPLETION = 1 }; /* when u^E += incr is counted                    */
+
+/* trace actions */
+enum { HB_ACT_NONE = 0, HB_ACT_HALVE = 1, HB_ACT_DOUBLE = 2, HB_ACT_CLAMP_LO = 3, HB_ACT_CLAMP_HI = 4 };
+
+typedef struct hb_model hb_model;
+typedef struct hb_worker hb_worker;
+typedef struct hb_comm hb_comm;
+
+/* Per-worker policy (Algorithm 2 inputs min_b^E, max_b^E [L194]; initial size [L236]). */
+typedef struct hb_worker_policy {
+  int32_t min_b;  /* lower threshold (never crossed, L236)                                */
+  int32_t max_b;  /* upper threshold                                                        */
+  int32_t init_b; /* initial batch size                                                     */
+  float incr;     /* updates credited per served batch: 1 (Alg. 1 worker) or t*beta (L234)  */
+  double c0, c1;  /* deterministic mode: virtual cost T(b) = c0 + c1*b                      */
+} hb_worker_policy;
+
+typedef struct hb_policy {
+  int32_t kind;          /* HB_MINIBATCH .. HB_ADAPTIVE                                      */
+  int32_t alpha;         /* batch scale factor, default 2 (L236)                              */
+  double eta0;           /* learning rate at batch b0; lr = eta0 * b / b0 (L179)              */
+  int32_t b0;
+  int32_t reset;         /* HB_RESET_*                                                        */
+  int32_t credit;        /* HB_CREDIT_*                                                       */
+  int32_t deterministic; /* 1: virtual clock + SERIAL execution in trace order (L125–L128)   */
+  int32_t eval_loss;     /* 1: full-data loss at every epoch end (excluded from timing, L258) */
+  int64_t max_steps;     /* stop after this many served batches in total (0 = no limit)      */
+  int32_t merges_per_epoch; /* multi-GPU: replica merges per epoch (needs comm; 0 = none)     */
+  float merge_gamma;     /* W <- W_base + gamma * sum(W_E - W_base); 1 = delta sum (R18)     */
+  hb_comm* comm;         /* nullable; NCCL communicator for the merge                         */
+  int32_t n_workers;     /* entries in workers[]                                              */
+  const hb_worker_policy* workers;
+} hb_policy;
+
+/* Training data resident in device memory (borrowed; caller-owned). */
+typedef struct hb_dataset {
+  const void* X;  /* [n x ldx] row-major, dtype x_dtype; ldx*elemsize must be a multiple of 16 */
+  int64_t ldx;    /* row stride in elements (>= n_0)                                           */
+  int32_t x_dtype;/* HB_BF16 (required for HB_PREC_BF16) or HB_F32                             */
+  const int32_t* y; /* [n] labels in [0, C)                                                    */
+  int64_t n;      /* number of examples N                                                      */
+} hb_dataset;
+
+/* One record per ScheduleWork message (O5). */
+typedef struct hb_trace_rec {
+  int64_t seq;
+  int32_t epoch, worker;
+  double vtime, u_before;
+  int32_t b_before, action, b_after, served;
+  double u_after;
+  int64_t offset; /* first row of the served batch, -1 if not served */
+  double lr;      /* 0 if not served                                 */
+} hb_trace_rec;
+
+/* Output statistics of hogbatch_run.  All pointers are caller-owned and nullable. */
+typedef struct hb_stats {
+  int32_t max_epochs;     /* capacity of the per-epoch arrays                                 */
+  int32_t epochs_done;
+  double* epoch_loss;     /* [max_epochs] full-data loss at epoch end (NaN if not evaluated) */
+  double* epoch_train_s;  /* [max_epochs] training seconds of the epoch (loss eval excluded) */
+  int64_t* updates;       /* [max_epochs * n_workers] served batches per worker per epoch    */
+  int64_t* samples;       /* [max_epochs * n_workers] examples per worker per epoch          */
+  hb_trace_rec* trace;    /* [trace_cap] schedule trace (all modes)                          */
+  int64_t trace_cap, trace_len;
+  float* step_loss;       /* [step_loss_cap] per-step batch loss, deterministic mode only    */
+  int64_t step_loss_cap, n_steps;
+  double total_train_s;   /* training seconds, loss evaluation excluded                     */
+  int64_t total_samples;
+  int32_t n_merges;
+} hb_stats;
+
+/* ---- library ---------------------------------------------------------------- */
+const char* hb_last_error(void);
+int hb_abi_version(void);
+/* 1 if a CUDA device of compute capability 10.x is visible, else 0 */
+int hb_device_ok(int32_t device);
+
+/* ---- model (§V.B: "The global model is allocated and initialized") ----
+ * dims[0..n_dims-1] = n_0 .. n_L; n_dims >= 2, all > 0, n_L >= 2 -> else HB_EINVAL.
+ * activation must be HB_SIGMOID.  precision HB_PREC_*.  Weights are initialised
+ * W ~ N(0, 1/fan_in), b = 0 from `seed` (R11).  The model owns its device
+ * memory: fp32 master weights+biases, bf16 shadow weights (bf16 mode). */
+int mlp_create(const int32_t* dims, int32_t n_dims, int32_t activation, int32_t precision,
+               uint64_t seed, int32_t device, hb_model** out);
+int mlp_destroy(hb_model* m);
+/* number of parameters P + sum n_l (weights + biases) */
+int mlp_num_params(const hb_model* m, int64_t* n_out);
+/* host flat fp32 layout: [W_1 (n_1 x n_0 row-major, unpadded), b_1, W_2, b_2, ...]; n must equal
+ * mlp_num_params.  Blocking.  set also refreshes the bf16 shadow. */
+int mlp_get_params(const hb_model* m, float* host_dst, int64_t n);
+int mlp_set_params(hb_model* m, const float* host_src, int64_t n);
+
+/* ---- worker (§V.A: GPU worker, exclusive device interface) ----------
+ * max_batch >= 1 sizes the worker's activation scratch.  replica must be 0 (a reference
+ * replica: the worker updates the shared model in place, Hogbatch L170).  cuda_stream may
+ * be NULL (the worker creates its own non-blocking stream) or a borrowed cudaStream_t. */
+int mlp_worker_create(hb_model* m, int32_t max_batch, int32_t replica, void* cuda_stream,
+                      hb_worker** out);
+int mlp_worker_destroy(hb_worker* w);
+/* cudaStream_t of the worker (borrowed) */
+void* mlp_worker_stream(hb_worker* w);
+
+/* ---- one SGD step (Alg. 1 ExecuteWork lines 2–3, Eq. (1)–(3)) ----------------------
+ * X: device pointer to the first row of the batch, [batch x ldx] of x_dtype (bf16 mode needs
+ * HB_BF16 and (ldx*2) % 16 == 0 and X 16-byte aligned); y: device int32 [batch] labels in
+ * [0, C) (out-of-range labels are undefined behaviour).  1 <= batch <= max_batch.
+ * Enqueued asynchronously on the worker's stream; if loss_out != NULL the call blocks and
+ * writes the batch-mean loss of the forward pass (before the update). */
+int mlp_step(hb_worker* w, const void* X, int64_t ldx, int32_t x_dtype, const int32_t* y,
+             int32_t batch, float lr, float* loss_out);
+/* test-only: same forward/backward as mlp_step but no update; copies the gradients to
+ * host_grads in the mlp_get_params flat layout (blocking). */
+int mlp_step_grads(hb_worker* w, const void* X, int64_t ldx, int32_t x_dtype, const int32_t* y,
+                   int32_t batch, float* host_grads, int64_t n, float* loss_out);
+
+/* ---- epoch-end loss (L273: "The loss computation is always performed on the GPU") ---
+ * mean cross-entropy over n examples, reduced deterministically in fp64.  Blocking. */
+int mlp_loss(hb_model* m, const void* X, int64_t ldx, int32_t x_dtype, const int32_t* y,
+             int64_t n, double* loss_out);
+
+/* ---- coordinator (Algorithms 1 and 2) ------------------------------------------------
+ * Runs the policy's coordinator on the deterministic virtual clock (hb_worker_policy c0/c1)
+ * over N examples for `epochs` epochs, without touching any GPU; writes up to cap records. */
+int hb_schedule_trace(const hb_policy* p, int64_t N, int32_t epochs, hb_trace_rec* out,
+                      int64_t cap, int64_t* n_out);
+/* Trains with n_workers workers (one host thread each, concurrent Hogbatch updates of the
+ * shared model, L170) under policy p for `epochs` epochs over data.  Blocking.
+ * p->deterministic = 1 executes the virtual-clock trace serially (SERIAL policy, L125). */
+int hogbatch_run(hb_worker** workers, int32_t n_workers, const hb_policy* p,
+                 const hb_dataset* data, int32_t epochs, hb_stats* stats_out);
+
+/* ---- multi-GPU replica merge over NCCL (future work L277) -------- */
+int hb_nccl_unique_id(uint8_t out[128]);
+int hb_comm_create(const uint8_t id[128], int32_t nranks, int32_t rank, int32_t device,
+                   hb_comm** out);
+int hb_comm_destroy(hb_comm* c);
+/* snapshot the current model as the merge base W_base (call when all ranks agree) */
+int hb_merge_begin(hb_model* m);
+/* W <- W_base + gamma * allreduce_sum(W - W_base); W_base <- W; bf16 shadow refreshed.
+ * Collective: every rank must call it.  stream may be NULL (model's internal stream).
+ * Blocking. */
+int hb_merge(hb_model* m, hb_comm* c, float gamma, void* cuda_stream);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* HOGBATCH_H */

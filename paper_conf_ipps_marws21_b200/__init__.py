@@ -1,0 +1,254 @@
+"""B200-native hot path of Adaptive Hogbatch (Ma, Rusu, Wu, Sim — IPDPSW/MARWS 2021).
+
+Thin Python binding over the C-ABI library ``libhogbatch.so`` (``include/hogbatch.h``):
+argument marshalling only — every step of the path runs in the library's CUDA kernels.
+PyTorch tensors are accepted wherever device memory is needed (only ``data_ptr()``,
+``stride()``, ``dtype`` and ``shape`` are read); PyTorch is plumbing, not the product.
+
+Names follow the paper: ``mlp_create`` / ``mlp_step`` / ``mlp_loss`` / ``hogbatch_run``.
+"""
+from __future__ import annotations
+
+import ctypes as C
+from dataclasses import dataclass, field
+
+import numpy as np
+
+from . import _lib
+from ._lib import (ACTIONS, HB_ADAPTIVE, HB_BF16, HB_CREDIT_COMPLETION, HB_CREDIT_DISPATCH, HB_F32,  # noqa: F401
+                   HB_HOGBATCH, HB_MINIBATCH, HB_PREC_BF16, HB_PREC_FP32_CHECK, HB_RESET_FASTEST,
+                   HB_RESET_NONE, HB_STATIC, HogbatchError)
+
+lib = _lib.load()
+
+
+def _check(rc: int):
+    if rc != 0:
+        raise HogbatchError(rc, lib.hb_last_error().decode(errors="replace"))
+
+
+def device_ok(device: int = 0) -> bool:
+    return bool(lib.hb_device_ok(device))
+
+
+def _xdtype(t) -> int:
+    s = str(t.dtype)
+    if "bfloat16" in s:
+        return HB_BF16
+    if "float32" in s:
+        return HB_F32
+    raise TypeError(f"X must be bfloat16 or float32, got {s}")
+
+
+def _stream_ptr(stream):
+    if stream is None:
+        return None
+    return C.c_void_p(int(getattr(stream, "cuda_stream", stream)))
+
+
+class MLP:
+    """``mlp_create(dims, activation)``: the global model (fp32 master + bf16 shadow on device)."""
+
+    def __init__(self, dims, precision: str = "bf16", seed: int = 0, device: int = 0):
+        self.dims = [int(d) for d in dims]
+        self.precision = precision
+        self.device = device
+        arr = (C.c_int32 * len(self.dims))(*self.dims)
+        h = C.c_void_p()
+        prec = HB_PREC_BF16 if precision == "bf16" else HB_PREC_FP32_CHECK
+        _check(lib.mlp_create(arr, len(self.dims), 0, prec, seed, device, C.byref(h)))
+        self.h = h
+
+    @property
+    def num_params(self) -> int:
+        n = C.c_int64()
+        _check(lib.mlp_num_params(self.h, C.byref(n)))
+        return n.value
+
+    def get_params(self) -> np.ndarray:
+        out = np.empty(self.num_params, dtype=np.float32)
+        _check(lib.mlp_get_params(self.h, out.ctypes.data_as(C.POINTER(C.c_float)), out.size))
+        return out
+
+    def set_params(self, flat) -> None:
+        flat = np.ascontiguousarray(flat, dtype=np.float32)
+        _check(lib.mlp_set_params(self.h, flat.ctypes.data_as(C.POINTER(C.c_float)), flat.size))
+
+    def loss(self, X, y, n: int | None = None) -> float:
+        """``mlp_loss``: mean cross-entropy over the first n rows of (X, y) (device tensors)."""
+        n = X.shape[0] if n is None else n
+        out = C.c_double()
+        _check(lib.mlp_loss(self.h, C.c_void_p(X.data_ptr()), X.stride(0), _xdtype(X),
+                            C.c_void_p(y.data_ptr()), n, C.byref(out)))
+        return out.value
+
+    def merge_begin(self):
+        _check(lib.hb_merge_begin(self.h))
+
+    def merge(self, comm: "Comm", gamma: float = 1.0, stream=None):
+        _check(lib.hb_merge(self.h, comm.h, gamma, _stream_ptr(stream)))
+
+    def close(self):
+        if getattr(self, "h", None):
+            lib.mlp_destroy(self.h)
+            self.h = None
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
+
+
+class Worker:
+    """A GPU worker (§V.A): activation scratch for max_batch rows and a stream."""
+
+    def __init__(self, model: MLP, max_batch: int, stream=None):
+        self.model = model
+        self.max_batch = max_batch
+        h = C.c_void_p()
+        _check(lib.mlp_worker_create(model.h, max_batch, 0, _stream_ptr(stream), C.byref(h)))
+        self.h = h
+
+    @property
+    def stream_handle(self) -> int:
+        return lib.mlp_worker_stream(self.h) or 0
+
+    def step(self, X, y, batch: int | None = None, lr: float = 0.1, want_loss: bool = False):
+        """``mlp_step(worker, X, y, batch, lr)`` on the rows starting at X[0] / y[0]."""
+        batch = X.shape[0] if batch is None else batch
+        out = C.c_float()
+        _check(lib.mlp_step(self.h, C.c_void_p(X.data_ptr()), X.stride(0), _xdtype(X),
+                            C.c_void_p(y.data_ptr()), batch, lr, C.byref(out) if want_loss else None))
+        return out.value if want_loss else None
+
+    def step_grads(self, X, y, batch: int | None = None):
+        """Test-only: gradients of the batch (flat mlp_get_params layout) and the batch loss."""
+        batch = X.shape[0] if batch is None else batch
+        g = np.empty(self.model.num_params, dtype=np.float32)
+        out = C.c_float()
+        _check(lib.mlp_step_grads(self.h, C.c_void_p(X.data_ptr()), X.stride(0), _xdtype(X),
+                                  C.c_void_p(y.data_ptr()), batch,
+                                  g.ctypes.data_as(C.POINTER(C.c_float)), g.size, C.byref(out)))
+        return g, out.value
+
+    def close(self):
+        if getattr(self, "h", None):
+            lib.mlp_worker_destroy(self.h)
+            self.h = None
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
+
+
+@dataclass
+class WorkerSpec:
+    min_b: int
+    max_b: int
+    init_b: int
+    incr: float = 1.0
+    c0: float = 0.0
+    c1: float = 1.0
+
+
+@dataclass
+class Policy:
+    """hb_policy: scheduling policy and hyperparameters held by the coordinator (L123)."""
+    kind: int = HB_ADAPTIVE
+    workers: list = field(default_factory=list)
+    alpha: int = 2
+    eta0: float = 0.1
+    b0: int = 32
+    reset: int = HB_RESET_FASTEST
+    credit: int = HB_CREDIT_DISPATCH
+    deterministic: bool = False
+    eval_loss: bool = False
+    max_steps: int = 0
+    merges_per_epoch: int = 0
+    merge_gamma: float = 1.0
+    comm: "Comm | None" = None
+
+    def to_c(self):
+        ws = (_lib.WorkerPolicy * len(self.workers))(*[
+            _lib.WorkerPolicy(w.min_b, w.max_b, w.init_b, w.incr, w.c0, w.c1) for w in self.workers])
+        p = _lib.Policy(self.kind, self.alpha, self.eta0, self.b0, self.reset, self.credit,
+                        int(self.deterministic), int(self.eval_loss), self.max_steps,
+                        self.merges_per_epoch, self.merge_gamma,
+                        self.comm.h if self.comm is not None else None, len(self.workers), ws)
+        return p, ws
+
+
+def _rec_tuple(r):
+    return (r.seq, r.epoch, r.worker, r.vtime, r.u_before, r.b_before, ACTIONS[r.action], r.b_after,
+            r.u_after, r.served, r.offset, r.lr)
+
+
+def schedule_trace(policy: Policy, N: int, epochs: int, cap: int = 1 << 20):
+    """``hb_schedule_trace``: the coordinator on the virtual clock (no GPU needed)."""
+    p, _keep = policy.to_c()
+    buf = (_lib.TraceRec * cap)()
+    n = C.c_int64()
+    _check(lib.hb_schedule_trace(C.byref(p), N, epochs, buf, cap, C.byref(n)))
+    return [_rec_tuple(buf[i]) for i in range(min(n.value, cap))]
+
+
+def hogbatch_run(workers, policy: Policy, X, y, epochs: int = 1, n: int | None = None,
+                 trace_cap: int = 0, step_loss_cap: int = 0, max_epochs: int | None = None):
+    """``hogbatch_run(workers, policy, epochs)`` over device data (X [N x ldx], y [N])."""
+    n = X.shape[0] if n is None else n
+    p, _keep = policy.to_c()
+    W = len(workers)
+    me = max_epochs or epochs
+    el = (C.c_double * me)()
+    et = (C.c_double * me)()
+    up = (C.c_int64 * (me * W))()
+    sm = (C.c_int64 * (me * W))()
+    tr = (_lib.TraceRec * max(trace_cap, 1))()
+    sl = (C.c_float * max(step_loss_cap, 1))()
+    st = _lib.Stats(me, 0, el, et, up, sm, tr, trace_cap, 0, sl, step_loss_cap, 0, 0.0, 0, 0)
+    ds = _lib.Dataset(X.data_ptr(), X.stride(0), _xdtype(X), y.data_ptr(), n)
+    hs = (C.c_void_p * W)(*[w.h.value for w in workers])
+    _check(lib.hogbatch_run(hs, W, C.byref(p), C.byref(ds), epochs, C.byref(st)))
+    ed = st.epochs_done
+    return dict(
+        epochs_done=ed,
+        epoch_loss=[el[i] for i in range(min(ed, me))],
+        epoch_train_s=[et[i] for i in range(min(ed, me))],
+        updates=np.array([up[i] for i in range(me * W)]).reshape(me, W)[:max(ed, 1)],
+        samples=np.array([sm[i] for i in range(me * W)]).reshape(me, W)[:max(ed, 1)],
+        trace=[_rec_tuple(tr[i]) for i in range(min(st.trace_len, trace_cap))],
+        trace_len=st.trace_len,
+        step_loss=[sl[i] for i in range(min(st.n_steps, step_loss_cap))],
+        n_steps=st.n_steps,
+        total_train_s=st.total_train_s,
+        total_samples=st.total_samples,
+        n_merges=st.n_merges,
+    )
+
+
+class Comm:
+    """NCCL communicator for the replica merge (one rank per GPU)."""
+
+    @staticmethod
+    def unique_id() -> bytes:
+        buf = (C.c_uint8 * 128)()
+        _check(lib.hb_nccl_unique_id(buf))
+        return bytes(buf)
+
+    def __init__(self, uid: bytes, nranks: int, rank: int, device: int):
+        buf = (C.c_uint8 * 128)(*uid)
+        h = C.c_void_p()
+        _check(lib.hb_comm_create(buf, nranks, rank, device, C.byref(h)))
+        self.h = h
+
+    def close(self):
+        if getattr(self, "h", None):
+            lib.hb_comm_destroy(self.h)
+            self.h = None
+
+
+def pad_to(n: int, m: int = 8) -> int:
+    return (n + m - 1) // m * m

@@ -1,0 +1,141 @@
+// epilogue.cuh — the fused per-element epilogues of the MLP-SGD GEMMs.
+//
+//   EPI_FWD_SIG    Eq. (1) hidden layer [PAPER.md L43, L258]: z = acc + b_n; H = sigma(z);
+//                  S = sigma'(z) = sigma(z)(1 - sigma(z)) stashed for the backward pass.
+//   EPI_FWD_LOGITS Eq. (1) output layer: logits = acc + b_n (fp32), softmax follows.
+//   EPI_DGRAD_SIG  Eq. (2) [L49]: dZ_{l-1} = (dZ_l W_l) * sigma'(Z_{l-1})  (acc * S).
+//   EPI_WGRAD_SGD  Eq. (3) [L53] fused into the dW GEMM: W -= lr * dW in place on the
+//                  shared fp32 master, bf16 shadow rewritten (Hogbatch update, L170).
+//   EPI_WGRAD_STORE test-only: dW written out (mlp_step_grads).
+#pragma once
+
+#include "common.cuh"
+
+namespace hb {
+
+enum { EPI_FWD_SIG = 0, EPI_FWD_LOGITS = 1, EPI_DGRAD_SIG = 2, EPI_WGRAD_SGD = 3, EPI_WGRAD_STORE = 4 };
+
+struct EpiArgs {
+  int M, N;             // valid output extent (rows, cols of the GEMM result)
+  const float* bias;    // FWD: [N]
+  void* out0;           // FWD_SIG: H; LOGITS: fp32 logits; DGRAD: dZ; WGRAD_STORE: fp32 grad
+  int64_t ld0;
+  void* out1;           // FWD_SIG: S = sigma'(z) (nullable: forward-only / loss evaluation)
+  int64_t ld1;
+  const void* aux;      // DGRAD: S of the layer below
+  int64_t ldaux;
+  float* master;        // WGRAD_SGD: fp32 master weights
+  __nv_bfloat16* shadow;// WGRAD_SGD: bf16 shadow (nullable in fp32 check mode)
+  int64_t ldw;
+  float lr;
+  int transposed;       // WGRAD: result element (m, n) belongs to W[n][m]
+};
+
+template <typename T>
+__device__ __forceinline__ T to_act(float v);
+template <>
+__device__ __forceinline__ float to_act<float>(float v) { return v; }
+template <>
+__device__ __forceinline__ __nv_bfloat16 to_act<__nv_bfloat16>(float v) { return __float2bfloat16_rn(v); }
+
+__device__ __forceinline__ float act_to_f(float v) { return v; }
+__device__ __forceinline__ float act_to_f(__nv_bfloat16 v) { return __bfloat162float(v); }
+
+// Scalar epilogue for one output element (r, n) with accumulator value v.
+// TAct = activation storage type (bf16 in the tensor-core path, fp32 in check mode).
+// PRECISE selects expf (check mode) instead of __expf.
+template <int EPI, typename TAct, bool PRECISE>
+__device__ __forceinline__ void epi_elem(const EpiArgs& ep, int r, int n, float v) {
+  if (EPI == EPI_FWD_SIG) {
+    float z = v + ep.bias[n];
+    float h = PRECISE ? 1.0f / (1.0f + expf(-z)) : sigmoidf_(z);
+    static_cast<TAct*>(ep.out0)[(int64_t)r * ep.ld0 + n] = to_act<TAct>(h);
+    if (ep.out1) static_cast<TAct*>(ep.out1)[(int64_t)r * ep.ld1 + n] = to_act<TAct>(h * (1.0f - h));
+  } else if (EPI == EPI_FWD_LOGITS) {
+    static_cast<float*>(ep.out0)[(int64_t)r * ep.ld0 + n] = v + ep.bias[n];
+  } else if (EPI == EPI_DGRAD_SIG) {
+    float s = act_to_f(static_cast<const TAct*>(ep.aux)[(int64_t)r * ep.ldaux + n]);
+    static_cast<TAct*>(ep.out0)[(int64_t)r * ep.ld0 + n] = to_act<TAct>(v * s);
+  } else if (EPI == EPI_WGRAD_SGD) {
+    int64_t idx = ep.transposed ? (int64_t)n * ep.ldw + r : (int64_t)r * ep.ldw + n;
+    float w = ep.master[idx] - ep.lr * v;
+    ep.master[idx] = w;
+    if (ep.shadow) ep.shadow[idx] = __float2bfloat16_rn(w);
+  } else {  // EPI_WGRAD_STORE
+    int64_t idx = ep.transposed ? (int64_t)n * ep.ldw + r : (int64_t)r * ep.ldw + n;
+    static_cast<float*>(ep.out0)[idx] = v;
+  }
+}
+
+__device__ __forceinline__ uint32_t pack_bf16x2(float a, float b) {
+  __nv_bfloat162 t = __floats2bfloat162_rn(a, b);
+  return *reinterpret_cast<uint32_t*>(&t);
+}
+
+// Vectorised epilogue for 16 consecutive columns n0..n0+15 of row r (all valid, 16-byte
+// aligned rows).  Used by the tensor-core kernel for full column chunks.
+template <int EPI>
+__device__ __forceinline__ void epi_row16_bf16(const EpiArgs& ep, int r, int n0, const float* v) {
+  if (EPI == EPI_FWD_SIG) {
+    uint32_t hp[8], sp[8];
+    const float4* b4 = reinterpret_cast<const float4*>(ep.bias + n0);
+#pragma unroll
+    for (int q = 0; q < 4; ++q) {
+      float4 bb = __ldg(b4 + q);
+      float z0 = v[4 * q] + bb.x, z1 = v[4 * q + 1] + bb.y, z2 = v[4 * q + 2] + bb.z,
+            z3 = v[4 * q + 3] + bb.w;
+      float h0 = sigmoidf_(z0), h1 = sigmoidf_(z1), h2 = sigmoidf_(z2), h3 = sigmoidf_(z3);
+      hp[2 * q] = pack_bf16x2(h0, h1);
+      hp[2 * q + 1] = pack_bf16x2(h2, h3);
+      sp[2 * q] = pack_bf16x2(h0 * (1.f - h0), h1 * (1.f - h1));
+      sp[2 * q + 1] = pack_bf16x2(h2 * (1.f - h2), h3 * (1.f - h3));
+    }
+    uint4* H = reinterpret_cast<uint4*>(static_cast<__nv_bfloat16*>(ep.out0) + (int64_t)r * ep.ld0 + n0);
+    H[0] = make_uint4(hp[0], hp[1], hp[2], hp[3]);
+    H[1] = make_uint4(hp[4], hp[5], hp[6], hp[7]);
+    if (ep.out1) {
+      uint4* S = reinterpret_cast<uint4*>(static_cast<__nv_bfloat16*>(ep.out1) + (int64_t)r * ep.ld1 + n0);
+      S[0] = make_uint4(sp[0], sp[1], sp[2], sp[3]);
+      S[1] = make_uint4(sp[4], sp[5], sp[6], sp[7]);
+    }
+  } else if (EPI == EPI_DGRAD_SIG) {
+    const uint4* S = reinterpret_cast<const uint4*>(static_cast<const __nv_bfloat16*>(ep.aux) +
+                                                    (int64_t)r * ep.ldaux + n0);
+    uint4 s0 = S[0], s1 = S[1];
+    const __nv_bfloat162* sv0 = reinterpret_cast<const __nv_bfloat162*>(&s0);
+    const __nv_bfloat162* sv1 = reinterpret_cast<const __nv_bfloat162*>(&s1);
+    uint32_t o[8];
+#pragma unroll
+    for (int q = 0; q < 4; ++q) {
+      float2 a = __bfloat1622float2(sv0[q]);
+      o[q] = pack_bf16x2(v[2 * q] * a.x, v[2 * q + 1] * a.y);
+      float2 c = __bfloat1622float2(sv1[q]);
+      o[4 + q] = pack_bf16x2(v[8 + 2 * q] * c.x, v[8 + 2 * q + 1] * c.y);
+    }
+    uint4* D = reinterpret_cast<uint4*>(static_cast<__nv_bfloat16*>(ep.out0) + (int64_t)r * ep.ld0 + n0);
+    D[0] = make_uint4(o[0], o[1], o[2], o[3]);
+    D[1] = make_uint4(o[4], o[5], o[6], o[7]);
+  } else if (EPI == EPI_WGRAD_SGD && 1) {
+    float4* W = reinterpret_cast<float4*>(ep.master + (int64_t)r * ep.ldw + n0);
+    uint32_t sp[8];
+#pragma unroll
+    for (int q = 0; q < 4; ++q) {
+      float4 w = W[q];
+      w.x -= ep.lr * v[4 * q];
+      w.y -= ep.lr * v[4 * q + 1];
+      w.z -= ep.lr * v[4 * q + 2];
+      w.w -= ep.lr * v[4 * q + 3];
+      W[q] = w;
+      sp[2 * q] = pack_bf16x2(w.x, w.y);
+      sp[2 * q + 1] = pack_bf16x2(w.z, w.w);
+    }
+    uint4* Sh = reinterpret_cast<uint4*>(ep.shadow + (int64_t)r * ep.ldw + n0);
+    Sh[0] = make_uint4(sp[0], sp[1], sp[2], sp[3]);
+    Sh[1] = make_uint4(sp[4], sp[5], sp[6], sp[7]);
+  } else {
+#pragma unroll
+    for (int j = 0; j < 16; ++j) epi_elem<EPI, __nv_bfloat16, false>(ep, r, n0 + j, v[j]);
+  }
+}
+
+}  // namespace hb

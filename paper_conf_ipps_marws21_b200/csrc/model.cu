@@ -1,0 +1,686 @@
+// model.cu — C ABI of the MLP-SGD hot path: model and worker objects, one SGD step
+// (forward GEMM chain, softmax-xent head, dX/dW GEMMs, fused in-place SGD), epilogue-free loss
+// evaluation, parameter I/O and the NCCL replica merge.
+//
+// Paper: Ma, Rusu, Wu, Sim (IPDPSW/MARWS 2021), §III (Eq. (1)–(3),
+// L41–L56), §V.A (workers, L132–L134), §VI (Hogbatch, L147–L170), §VII.A (sigmoid hidden layers,
+// softmax cross-entropy, L258).
+#include <cudaTypedefs.h>
+
+#include <atomic>
+#include <cmath>
+#include <cstring>
+#include <mutex>
+#include <random>
+#include <set>
+#include <string>
+#include <vector>
+
+#include "kernels.cuh"
+#include "model.h"
+#include "tc_gemm.cuh"
+
+namespace hb {
+
+// ----------------------------------------------------------------------------------------
+// errors
+// ----------------------------------------------------------------------------------------
+static thread_local std::string g_err;
+void set_error(const std::string& msg) { g_err = msg; }
+int fail(int code, const std::string& msg) {
+  g_err = msg;
+  return code;
+}
+
+// ----------------------------------------------------------------------------------------
+// TMA tensor maps (driver entry point; no link-time dependency on libcuda)
+// ----------------------------------------------------------------------------------------
+static PFN_cuTensorMapEncodeTiled_v12000 g_encode = nullptr;
+
+static int ensure_encode() {
+  static std::once_flag once;
+  static cudaError_t err = cudaSuccess;
+  std::call_once(once, [] {
+    void* fn = nullptr;
+    cudaDriverEntryPointQueryResult q;
+    err = cudaGetDriverEntryPoint("cuTensorMapEncodeTiled", &fn, cudaEnableDefault, &q);
+    if (err == cudaSuccess && q == cudaDriverEntryPointSuccess)
+      g_encode = reinterpret_cast<PFN_cuTensorMapEncodeTiled_v12000>(fn);
+  });
+  if (!g_encode) return fail(HB_ECUDA, std::string("cuTensorMapEncodeTiled unavailable: ") + cudaGetErrorString(err));
+  return HB_OK;
+}
+
+// bf16 2-D map: dims {inner, outer}, row stride in bytes, box {box_inner, box_outer}, 128B swizzle,
+// out-of-bounds elements read as zero (this is how ragged M/N/K tails are handled).
+static int make_map(CUtensorMap* out, const void* base, uint64_t inner, uint64_t outer,
+                    uint64_t stride_bytes, uint32_t box_inner, uint32_t box_outer) {
+  int rc = ensure_encode();
+  if (rc) return rc;
+  cuuint64_t dims[2] = {inner, outer};
+  cuuint64_t strides[1] = {stride_bytes};
+  cuuint32_t box[2] = {box_inner, box_outer};
+  cuuint32_t es[2] = {1, 1};
+  CUresult r = g_encode(out, CU_TENSOR_MAP_DATA_TYPE_BFLOAT16, 2, const_cast<void*>(base), dims, strides,
+                        box, es, CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_128B,
+                        CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+  if (r != CUDA_SUCCESS)
+    return fail(HB_ECUDA, "cuTensorMapEncodeTiled failed (" + std::to_string((int)r) + ") inner=" +
+                              std::to_string(inner) + " outer=" + std::to_string(outer) +
+                              " stride=" + std::to_string(stride_bytes));
+  return HB_OK;
+}
+
+// ----------------------------------------------------------------------------------------
+// GEMM dispatch
+// ----------------------------------------------------------------------------------------
+static std::mutex g_attr_mu;
+static std::set<std::pair<const void*, int>> g_attr_done;
+
+template <int BN, bool A_MN, bool B_MN, int EPI>
+static int launch_tc(const CUtensorMap& ma, const CUtensorMap& mb, int M, int N, int K, const EpiArgs& ep,
+                     cudaStream_t s) {
+  using Cfg = TcCfg<BN, B_MN>;
+  auto kern = tc_gemm_kernel<BN, A_MN, B_MN, EPI>;
+  int dev = 0;
+  cudaGetDevice(&dev);
+  {
+    std::lock_guard<std::mutex> g(g_attr_mu);
+    auto key = std::make_pair((const void*)kern, dev);
+    if (!g_attr_done.count(key)) {
+      HB_CUDA_TRY(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, Cfg::SMEM_BYTES));
+      g_attr_done.insert(key);
+    }
+  }
+  dim3 grid((N + BN - 1) / BN, (M + TC_BM - 1) / TC_BM);
+  kern<<<grid, TC_THREADS, Cfg::SMEM_BYTES, s>>>(ma, mb, K, ep);
+  HB_CUDA_TRY(cudaGetLastError());
+  return HB_OK;
+}
+
+template <bool A_MN, bool B_MN, int EPI>
+static int launch_tc_bn(int bn, const CUtensorMap& ma, const CUtensorMap& mb, int M, int N, int K,
+                        const EpiArgs& ep, cudaStream_t s) {
+  switch (bn) {
+    case 16: return launch_tc<16, A_MN, B_MN, EPI>(ma, mb, M, N, K, ep, s);
+    case 32: return launch_tc<32, A_MN, B_MN, EPI>(ma, mb, M, N, K, ep, s);
+    case 64: return launch_tc<64, A_MN, B_MN, EPI>(ma, mb, M, N, K, ep, s);
+    case 128: return launch_tc<128, A_MN, B_MN, EPI>(ma, mb, M, N, K, ep, s);
+    default: return launch_tc<256, A_MN, B_MN, EPI>(ma, mb, M, N, K, ep, s);
+  }
+}
+
+int choose_bn(int M, int N) {
+  if (N <= 16) return 16;
+  if (N <= 32) return 32;
+  if (N <= 64) return 64;
+  if (N <= 128) return 128;
+  const long mt = (M + TC_BM - 1) / TC_BM;
+  if (mt * ((N + 255) / 256) >= 148) return 256;
+  return 128;
+}
+
+// tensor-core GEMM on bf16 operands.  A is [M x K] (K-major, row stride lda) or stored [K x M]
+// (MN-major); B is [N x K] (K-major) or stored [K x N] (MN-major).
+static int gemm_tc(int epi, bool a_mn, bool b_mn, int M, int N, int K, const void* A, int64_t lda,
+                   const void* B, int64_t ldb, const EpiArgs& ep, cudaStream_t s) {
+  const int bn = choose_bn(M, N);
+  CUtensorMap ma, mb;
+  int rc = a_mn ? make_map(&ma, A, M, K, lda * 2, 64, 64) : make_map(&ma, A, K, M, lda * 2, 64, TC_BM);
+  if (rc) return rc;
+  rc = b_mn ? make_map(&mb, B, N, K, ldb * 2, 64, 64) : make_map(&mb, B, K, N, ldb * 2, 64, bn);
+  if (rc) return rc;
+  if (!a_mn && !b_mn) {
+    if (epi == EPI_FWD_SIG) return launch_tc_bn<false, false, EPI_FWD_SIG>(bn, ma, mb, M, N, K, ep, s);
+    if (epi == EPI_FWD_LOGITS) return launch_tc_bn<false, false, EPI_FWD_LOGITS>(bn, ma, mb, M, N, K, ep, s);
+  } else if (!a_mn && b_mn) {
+    if (epi == EPI_DGRAD_SIG) return launch_tc_bn<false, true, EPI_DGRAD_SIG>(bn, ma, mb, M, N, K, ep, s);
+  } else if (a_mn && b_mn) {
+    if (epi == EPI_WGRAD_SGD) return launch_tc_bn<true, true, EPI_WGRAD_SGD>(bn, ma, mb, M, N, K, ep, s);
+    if (epi == EPI_WGRAD_STORE) return launch_tc_bn<true, true, EPI_WGRAD_STORE>(bn, ma, mb, M, N, K, ep, s);
+  }
+  return fail(HB_EUNSUPPORTED, "gemm_tc: unsupported epilogue/major combination");
+}
+
+template <int EPI, typename TA, typename TB>
+static int launch_simt_t(const void* A, int64_t sam, int64_t sak, const void* B, int64_t sbn, int64_t sbk,
+                         int M, int N, int K, const EpiArgs& ep, cudaStream_t s) {
+  dim3 grid((N + 63) / 64, (M + 63) / 64);
+  simt_gemm_kernel<EPI, TA, TB><<<grid, 256, 0, s>>>(static_cast<const TA*>(A), sam, sak,
+                                                     static_cast<const TB*>(B), sbn, sbk, M, N, K, ep);
+  HB_CUDA_TRY(cudaGetLastError());
+  return HB_OK;
+}
+
+template <int EPI>
+static int launch_simt(const void* A, int adt, int64_t sam, int64_t sak, const void* B, int bdt, int64_t sbn,
+                       int64_t sbk, int M, int N, int K, const EpiArgs& ep, cudaStream_t s) {
+  if (adt == HB_F32 && bdt == HB_F32) return launch_simt_t<EPI, float, float>(A, sam, sak, B, sbn, sbk, M, N, K, ep, s);
+  if (adt == HB_BF16 && bdt == HB_F32)
+    return launch_simt_t<EPI, __nv_bfloat16, float>(A, sam, sak, B, sbn, sbk, M, N, K, ep, s);
+  if (adt == HB_F32 && bdt == HB_BF16)
+    return launch_simt_t<EPI, float, __nv_bfloat16>(A, sam, sak, B, sbn, sbk, M, N, K, ep, s);
+  return launch_simt_t<EPI, __nv_bfloat16, __nv_bfloat16>(A, sam, sak, B, sbn, sbk, M, N, K, ep, s);
+}
+
+// fp32 check-mode GEMM with the same operand conventions as gemm_tc
+static int gemm_simt(int epi, bool a_mn, bool b_mn, int M, int N, int K, const void* A, int64_t lda, int adt,
+                     const void* B, int64_t ldb, int bdt, const EpiArgs& ep, cudaStream_t s) {
+  const int64_t sam = a_mn ? 1 : lda, sak = a_mn ? lda : 1;
+  const int64_t sbn = b_mn ? 1 : ldb, sbk = b_mn ? ldb : 1;
+  switch (epi) {
+    case EPI_FWD_SIG: return launch_simt<EPI_FWD_SIG>(A, adt, sam, sak, B, bdt, sbn, sbk, M, N, K, ep, s);
+    case EPI_FWD_LOGITS: return launch_simt<EPI_FWD_LOGITS>(A, adt, sam, sak, B, bdt, sbn, sbk, M, N, K, ep, s);
+    case EPI_DGRAD_SIG: return launch_simt<EPI_DGRAD_SIG>(A, adt, sam, sak, B, bdt, sbn, sbk, M, N, K, ep, s);
+    case EPI_WGRAD_SGD: return launch_simt<EPI_WGRAD_SGD>(A, adt, sam, sak, B, bdt, sbn, sbk, M, N, K, ep, s);
+    default: return launch_simt<EPI_WGRAD_STORE>(A, adt, sam, sak, B, bdt, sbn, sbk, M, N, K, ep, s);
+  }
+}
+
+static int gemm(const hb_model* m, int epi, bool a_mn, bool b_mn, int M, int N, int K, const void* A, int64_t lda,
+                int adt, const void* B, int64_t ldb, int bdt, const EpiArgs& ep, cudaStream_t s) {
+  if (M <= 0 || N <= 0 || K <= 0) return HB_OK;
+  if (m->prec == HB_PREC_BF16) {
+    if (adt != HB_BF16 || bdt != HB_BF16) return fail(HB_EINVAL, "bf16 mode needs bf16 operands (X must be HB_BF16)");
+    return gemm_tc(epi, a_mn, b_mn, M, N, K, A, lda, B, ldb, ep, s);
+  }
+  return gemm_simt(epi, a_mn, b_mn, M, N, K, A, lda, adt, B, ldb, bdt, ep, s);
+}
+
+// ----------------------------------------------------------------------------------------
+// model / worker
+// ----------------------------------------------------------------------------------------
+static int act_dt(const hb_model* m) { return m->prec == HB_PREC_BF16 ? HB_BF16 : HB_F32; }
+static size_t act_size(const hb_model* m) { return m->prec == HB_PREC_BF16 ? 2 : 4; }
+
+static void free_worker_buffers(hb_worker* w) {
+  for (void* p : w->H) cudaFree(p);
+  for (void* p : w->S) cudaFree(p);
+  for (void* p : w->dZ) cudaFree(p);
+  w->H.clear();
+  w->S.clear();
+  w->dZ.clear();
+  cudaFree(w->logits);
+  cudaFree(w->row_loss);
+  cudaFree(w->partial);
+  cudaFree(w->dsum);
+  cudaFree(w->grads);
+  if (w->h_dsum) cudaFreeHost(w->h_dsum);
+  w->logits = w->row_loss = w->partial = w->grads = nullptr;
+  w->dsum = nullptr;
+  w->h_dsum = nullptr;
+}
+
+static int alloc_worker(hb_model* m, int max_b, cudaStream_t stream, bool own, hb_worker** out) {
+  hb_worker* w = new hb_worker();
+  w->m = m;
+  w->max_b = max_b;
+  w->stream = stream;
+  w->own_stream = own;
+  const int L = (int)m->layers.size();
+  const size_t es = act_size(m);
+  auto fail_free = [&](int rc) {
+    free_worker_buffers(w);
+    if (w->own_stream && w->stream) cudaStreamDestroy(w->stream);
+    delete w;
+    return rc;
+  };
+  int max_w = 1;
+  for (int l = 0; l < L; ++l) {
+    const Layer& Ly = m->layers[l];
+    max_w = std::max(max_w, Ly.n_out);
+    void* p = nullptr;
+    if (l < L - 1) {
+      if (cudaMalloc(&p, (size_t)max_b * Ly.ldo * es) != cudaSuccess) return fail_free(fail(HB_ENOMEM, "H alloc"));
+      w->H.push_back(p);
+      if (cudaMalloc(&p, (size_t)max_b * Ly.ldo * es) != cudaSuccess) return fail_free(fail(HB_ENOMEM, "S alloc"));
+      w->S.push_back(p);
+    }
+    if (cudaMalloc(&p, (size_t)max_b * Ly.ldo * es) != cudaSuccess) return fail_free(fail(HB_ENOMEM, "dZ alloc"));
+    cudaMemset(p, 0, (size_t)max_b * Ly.ldo * es);
+    w->dZ.push_back(p);
+  }
+  const int C = m->layers.back().n_out;
+  w->ldc = (int)round_up(C, 4);
+  w->splits_max = (max_b + 127) / 128;
+  if (cudaMalloc(&w->logits, (size_t)max_b * w->ldc * 4) != cudaSuccess ||
+      cudaMalloc(&w->row_loss, (size_t)max_b * 4) != cudaSuccess ||
+      cudaMalloc(&w->partial, (size_t)w->splits_max * max_w * 4) != cudaSuccess ||
+      cudaMalloc(&w->dsum, 64 * sizeof(double)) != cudaSuccess ||
+      cudaMallocHost(&w->h_dsum, 64 * sizeof(double)) != cudaSuccess)
+    return fail_free(fail(HB_ENOMEM, "worker scratch alloc"));
+  *out = w;
+  return HB_OK;
+}
+
+}  // namespace hb
+
+using namespace hb;
+
+// ----------------------------------------------------------------------------------------
+// one SGD step: Eq. (1) forward, softmax-xent head, Eq. (2) backward, Eq. (3) in-place update
+// ----------------------------------------------------------------------------------------
+namespace hb {
+
+int run_step(hb_worker* w, const void* X, int64_t ldx, int32_t xdt, const int32_t* y, int b, float lr,
+             bool grads_only, cudaStream_t s) {
+  hb_model* m = w->m;
+  const int L = (int)m->layers.size();
+  const int adt = act_dt(m);
+  const bool bf = m->prec == HB_PREC_BF16;
+  int rc;
+  // ---- forward, Eq. (1) ----
+  const void* Ain = X;
+  int64_t lda = ldx;
+  int ain_dt = xdt;
+  for (int l = 0; l < L; ++l) {
+    const Layer& Ly = m->layers[l];
+    EpiArgs ep{};
+    ep.M = b;
+    ep.N = Ly.n_out;
+    ep.bias = m->master + Ly.b_off;
+    int epi;
+    if (l < L - 1) {
+      epi = EPI_FWD_SIG;
+      ep.out0 = w->H[l];
+      ep.ld0 = Ly.ldo;
+      ep.out1 = w->S[l];
+      ep.ld1 = Ly.ldo;
+    } else {
+      epi = EPI_FWD_LOGITS;
+      ep.out0 = w->logits;
+      ep.ld0 = w->ldc;
+    }
+    const void* Wp = bf ? (const void*)(m->shadow + Ly.w_off) : (const void*)(m->master + Ly.w_off);
+    rc = gemm(m, epi, false, false, b, Ly.n_out, Ly.n_in, Ain, lda, ain_dt, Wp, Ly.ldw, bf ? HB_BF16 : HB_F32, ep, s);
+    if (rc) return rc;
+    if (l < L - 1) {
+      Ain = w->H[l];
+      lda = Ly.ldo;
+      ain_dt = adt;
+    }
+  }
+  // ---- softmax cross-entropy head: loss rows + dZ_L = (softmax - onehot)/b ----
+  {
+    const Layer& Ly = m->layers[L - 1];
+    const int threads = 256;
+    const int blocks = (b * 32 + threads - 1) / threads;
+    if (bf)
+      softmax_xent_kernel<__nv_bfloat16><<<blocks, threads, 0, s>>>(
+          w->logits, w->ldc, y, b, Ly.n_out, static_cast<__nv_bfloat16*>(w->dZ[L - 1]), Ly.ldo, w->row_loss,
+          1.0f / (float)b);
+    else
+      softmax_xent_kernel<float><<<blocks, threads, 0, s>>>(w->logits, w->ldc, y, b, Ly.n_out,
+                                                           static_cast<float*>(w->dZ[L - 1]), Ly.ldo,
+                                                           w->row_loss, 1.0f / (float)b);
+    HB_CUDA_TRY(cudaGetLastError());
+  }
+  // ---- backward, Eq. (2), with the update of Eq. (3) fused into the dW GEMM ----
+  for (int l = L - 1; l >= 0; --l) {
+    const Layer& Ly = m->layers[l];
+    const void* dZl = w->dZ[l];
+    const void* Al = l == 0 ? X : w->H[l - 1];
+    const int64_t ldal = l == 0 ? ldx : m->layers[l - 1].ldo;
+    const int al_dt = l == 0 ? xdt : adt;
+    const void* Wp = bf ? (const void*)(m->shadow + Ly.w_off) : (const void*)(m->master + Ly.w_off);
+    if (l > 0) {  // dZ_{l-1} = (dZ_l W_l) * sigma'(Z_{l-1}); reads W_l before it is updated below
+      const Layer& Lp = m->layers[l - 1];
+      EpiArgs ep{};
+      ep.M = b;
+      ep.N = Ly.n_in;
+      ep.out0 = w->dZ[l - 1];
+      ep.ld0 = Lp.ldo;
+      ep.aux = w->S[l - 1];
+      ep.ldaux = Lp.ldo;
+      rc = gemm(m, EPI_DGRAD_SIG, false, true, b, Ly.n_in, Ly.n_out, dZl, Ly.ldo, adt, Wp, Ly.ldw,
+                bf ? HB_BF16 : HB_F32, ep, s);
+      if (rc) return rc;
+    }
+    {  // W_l -= lr * dZ_l^T A_{l-1}
+      EpiArgs ep{};
+      const int epi = grads_only ? EPI_WGRAD_STORE : EPI_WGRAD_SGD;
+      ep.master = m->master + Ly.w_off;
+      ep.shadow = bf ? m->shadow + Ly.w_off : nullptr;
+      ep.ldw = Ly.ldw;
+      ep.lr = lr;
+      if (grads_only) ep.out0 = w->grads + Ly.w_off;
+      const bool tr = Ly.n_out < 128 && Ly.n_out < Ly.n_in;  // small head: M = n_in instead of n_out
+      ep.transposed = tr ? 1 : 0;
+      if (!tr) {
+        ep.M = Ly.n_out;
+        ep.N = Ly.n_in;
+        rc = gemm(m, epi, true, true, Ly.n_out, Ly.n_in, b, dZl, Ly.ldo, adt, Al, ldal, al_dt, ep, s);
+      } else {
+        ep.M = Ly.n_in;
+        ep.N = Ly.n_out;
+        rc = gemm(m, epi, true, true, Ly.n_in, Ly.n_out, b, Al, ldal, al_dt, dZl, Ly.ldo, adt, ep, s);
+      }
+      if (rc) return rc;
+    }
+    {  // b_l -= lr * 1^T dZ_l (deterministic two-pass column sum)
+      const int splits = (b + 127) / 128;
+      dim3 g1((Ly.n_out + 63) / 64, splits), b1(64, 4);
+      if (bf)
+        colsum_partial_kernel<__nv_bfloat16><<<g1, b1, 0, s>>>(static_cast<const __nv_bfloat16*>(dZl), Ly.ldo, b,
+                                                              Ly.n_out, 128, w->partial);
+      else
+        colsum_partial_kernel<float><<<g1, b1, 0, s>>>(static_cast<const float*>(dZl), Ly.ldo, b, Ly.n_out, 128,
+                                                       w->partial);
+      bias_apply_kernel<<<(Ly.n_out + 255) / 256, 256, 0, s>>>(w->partial, splits, Ly.n_out, lr,
+                                                               m->master + Ly.b_off,
+                                                               grads_only ? w->grads + Ly.b_off : nullptr);
+      HB_CUDA_TRY(cudaGetLastError());
+    }
+  }
+  return HB_OK;
+}
+
+static int check_step_args(hb_worker* w, const void* X, int64_t ldx, int32_t xdt, const int32_t* y, int32_t batch) {
+  if (!w) return fail(HB_EINVAL, "null worker");
+  hb_model* m = w->m;
+  HB_CHECK_ARG(X && y, "null X or y");
+  HB_CHECK_ARG(batch >= 1 && batch <= w->max_b, "batch must be in [1, max_batch]");
+  HB_CHECK_ARG(xdt == HB_BF16 || xdt == HB_F32, "x_dtype must be HB_BF16 or HB_F32");
+  HB_CHECK_ARG(ldx >= m->dims[0], "ldx < n_0");
+  if (m->prec == HB_PREC_BF16) {
+    HB_CHECK_ARG(xdt == HB_BF16, "bf16 model needs HB_BF16 input");
+    HB_CHECK_ARG((ldx * 2) % 16 == 0, "ldx*2 must be a multiple of 16 bytes (pad n_0 to a multiple of 8)");
+    HB_CHECK_ARG((reinterpret_cast<uintptr_t>(X) & 15) == 0, "X must be 16-byte aligned");
+  }
+  return HB_OK;
+}
+
+void sum_rows_into(hb_worker* w, int b, double* dst, cudaStream_t s) {
+  sum_rows_kernel<<<1, 1024, 0, s>>>(w->row_loss, b, dst, 0);
+}
+
+int finish_loss(hb_worker* w, int b, float* loss_out, cudaStream_t s) {
+  sum_rows_kernel<<<1, 1024, 0, s>>>(w->row_loss, b, w->dsum, 0);
+  HB_CUDA_TRY(cudaGetLastError());
+  HB_CUDA_TRY(cudaMemcpyAsync(w->h_dsum, w->dsum, sizeof(double), cudaMemcpyDeviceToHost, s));
+  HB_CUDA_TRY(cudaStreamSynchronize(s));
+  *loss_out = (float)(w->h_dsum[0] / (double)b);
+  return HB_OK;
+}
+
+}  // namespace hb
+
+extern "C" {
+
+const char* hb_last_error(void) { return hb::g_err.c_str(); }
+int hb_abi_version(void) { return HB_ABI_VERSION; }
+
+int hb_device_ok(int32_t device) {
+  int n = 0;
+  if (cudaGetDeviceCount(&n) != cudaSuccess || device < 0 || device >= n) return 0;
+  cudaDeviceProp p;
+  if (cudaGetDeviceProperties(&p, device) != cudaSuccess) return 0;
+  return p.major == 10 ? 1 : 0;
+}
+
+int mlp_create(const int32_t* dims, int32_t n_dims, int32_t activation, int32_t precision, uint64_t seed,
+               int32_t device, hb_model** out) {
+  HB_CHECK_ARG(out, "null out");
+  *out = nullptr;
+  HB_CHECK_ARG(dims && n_dims >= 2, "need n_dims >= 2");
+  for (int i = 0; i < n_dims; ++i) HB_CHECK_ARG(dims[i] > 0, "all dims must be > 0");
+  HB_CHECK_ARG(dims[n_dims - 1] >= 2, "need at least 2 classes");
+  if (activation != HB_SIGMOID) return fail(HB_EUNSUPPORTED, "only HB_SIGMOID hidden activation (PAPER.md L258)");
+  HB_CHECK_ARG(precision == HB_PREC_BF16 || precision == HB_PREC_FP32_CHECK, "bad precision");
+  HB_CUDA_TRY(cudaSetDevice(device));
+  if (precision == HB_PREC_BF16 && !hb_device_ok(device))
+    return fail(HB_EUNSUPPORTED, "bf16 tensor-core path needs an sm_100 (B200) device");
+  hb_model* m = new hb_model();
+  m->device = device;
+  m->prec = precision;
+  m->dims.assign(dims, dims + n_dims);
+  size_t off = 0;
+  for (int l = 1; l < n_dims; ++l) {
+    Layer Ly;
+    Ly.n_in = dims[l - 1];
+    Ly.n_out = dims[l];
+    Ly.ldw = (int)round_up(Ly.n_in, 8);
+    Ly.ldo = (int)round_up(Ly.n_out, 8);
+    Ly.w_off = round_up(off, 16);
+    Ly.b_off = round_up(Ly.w_off + (size_t)Ly.n_out * Ly.ldw, 16);
+    off = Ly.b_off + Ly.n_out;
+    m->layers.push_back(Ly);
+  }
+  m->total = round_up(off, 16);
+  if (cudaMalloc(&m->master, m->total * 4) != cudaSuccess ||
+      (precision == HB_PREC_BF16 && cudaMalloc(&m->shadow, m->total * 2) != cudaSuccess)) {
+    cudaFree(m->master);
+    delete m;
+    return fail(HB_ENOMEM, "model alloc");
+  }
+  if (cudaStreamCreateWithFlags(&m->stream, cudaStreamNonBlocking) != cudaSuccess) {
+    cudaFree(m->master);
+    cudaFree(m->shadow);
+    delete m;
+    return fail(HB_ECUDA, "stream create");
+  }
+  // W ~ N(0, 1/fan_in), b = 0 (R11)
+  std::vector<float> h(m->total, 0.f);
+  std::mt19937_64 gen(seed);
+  std::normal_distribution<double> nd(0.0, 1.0);
+  for (const Layer& Ly : m->layers) {
+    const double sd = 1.0 / std::sqrt((double)Ly.n_in);
+    for (int i = 0; i < Ly.n_out; ++i)
+      for (int j = 0; j < Ly.n_in; ++j) h[Ly.w_off + (size_t)i * Ly.ldw + j] = (float)(nd(gen) * sd);
+  }
+  int rc = [&]() -> int {
+    HB_CUDA_TRY(cudaMemcpy(m->master, h.data(), m->total * 4, cudaMemcpyHostToDevice));
+    if (m->shadow) {
+      refresh_shadow_kernel<<<256, 256, 0, m->stream>>>(m->master, m->shadow, (int64_t)m->total);
+      HB_CUDA_TRY(cudaGetLastError());
+      HB_CUDA_TRY(cudaStreamSynchronize(m->stream));
+    }
+    return HB_OK;
+  }();
+  if (rc) {
+    mlp_destroy(m);
+    return rc;
+  }
+  *out = m;
+  return HB_OK;
+}
+
+int mlp_destroy(hb_model* m) {
+  if (!m) return HB_OK;
+  cudaSetDevice(m->device);
+  if (m->eval) mlp_worker_destroy(m->eval);
+  cudaFree(m->master);
+  cudaFree(m->shadow);
+  cudaFree(m->base);
+  cudaFree(m->delta);
+  cudaFree(m->chunk_sums);
+  if (m->stream) cudaStreamDestroy(m->stream);
+  delete m;
+  return HB_OK;
+}
+
+int mlp_num_params(const hb_model* m, int64_t* n_out) {
+  HB_CHECK_ARG(m && n_out, "null arg");
+  int64_t n = 0;
+  for (const Layer& Ly : m->layers) n += (int64_t)Ly.n_out * Ly.n_in + Ly.n_out;
+  *n_out = n;
+  return HB_OK;
+}
+
+int mlp_get_params(const hb_model* m, float* host_dst, int64_t n) {
+  int64_t need;
+  int rc = mlp_num_params(m, &need);
+  if (rc) return rc;
+  HB_CHECK_ARG(host_dst && n == need, "n must equal mlp_num_params");
+  HB_CUDA_TRY(cudaSetDevice(m->device));
+  std::vector<float> h(m->total);
+  HB_CUDA_TRY(cudaMemcpy(h.data(), m->master, m->total * 4, cudaMemcpyDeviceToHost));
+  int64_t o = 0;
+  for (const Layer& Ly : m->layers) {
+    for (int i = 0; i < Ly.n_out; ++i)
+      for (int j = 0; j < Ly.n_in; ++j) host_dst[o++] = h[Ly.w_off + (size_t)i * Ly.ldw + j];
+    for (int i = 0; i < Ly.n_out; ++i) host_dst[o++] = h[Ly.b_off + i];
+  }
+  return HB_OK;
+}
+
+int mlp_set_params(hb_model* m, const float* host_src, int64_t n) {
+  int64_t need;
+  int rc = mlp_num_params(m, &need);
+  if (rc) return rc;
+  HB_CHECK_ARG(host_src && n == need, "n must equal mlp_num_params");
+  HB_CUDA_TRY(cudaSetDevice(m->device));
+  std::vector<float> h(m->total, 0.f);
+  int64_t o = 0;
+  for (const Layer& Ly : m->layers) {
+    for (int i = 0; i < Ly.n_out; ++i)
+      for (int j = 0; j < Ly.n_in; ++j) h[Ly.w_off + (size_t)i * Ly.ldw + j] = host_src[o++];
+    for (int i = 0; i < Ly.n_out; ++i) h[Ly.b_off + i] = host_src[o++];
+  }
+  HB_CUDA_TRY(cudaDeviceSynchronize());
+  HB_CUDA_TRY(cudaMemcpy(m->master, h.data(), m->total * 4, cudaMemcpyHostToDevice));
+  if (m->shadow) {
+    refresh_shadow_kernel<<<256, 256, 0, m->stream>>>(m->master, m->shadow, (int64_t)m->total);
+    HB_CUDA_TRY(cudaGetLastError());
+  }
+  HB_CUDA_TRY(cudaStreamSynchronize(m->stream));
+  return HB_OK;
+}
+
+int mlp_worker_create(hb_model* m, int32_t max_batch, int32_t replica, void* cuda_stream, hb_worker** out) {
+  HB_CHECK_ARG(m && out, "null arg");
+  *out = nullptr;
+  HB_CHECK_ARG(max_batch >= 1, "max_batch must be >= 1");
+  if (replica != 0) return fail(HB_EUNSUPPORTED, "only reference replicas (in-place Hogbatch updates) are implemented");
+  HB_CUDA_TRY(cudaSetDevice(m->device));
+  cudaStream_t s = static_cast<cudaStream_t>(cuda_stream);
+  bool own = false;
+  if (!s) {
+    HB_CUDA_TRY(cudaStreamCreateWithFlags(&s, cudaStreamNonBlocking));
+    own = true;
+  }
+  return alloc_worker(m, max_batch, s, own, out);
+}
+
+int mlp_worker_destroy(hb_worker* w) {
+  if (!w) return HB_OK;
+  cudaSetDevice(w->m->device);
+  cudaStreamSynchronize(w->stream);
+  free_worker_buffers(w);
+  if (w->own_stream) cudaStreamDestroy(w->stream);
+  delete w;
+  return HB_OK;
+}
+
+void* mlp_worker_stream(hb_worker* w) { return w ? (void*)w->stream : nullptr; }
+
+int mlp_step(hb_worker* w, const void* X, int64_t ldx, int32_t x_dtype, const int32_t* y, int32_t batch, float lr,
+             float* loss_out) {
+  int rc = check_step_args(w, X, ldx, x_dtype, y, batch);
+  if (rc) return rc;
+  HB_CUDA_TRY(cudaSetDevice(w->m->device));
+  rc = run_step(w, X, ldx, x_dtype, y, batch, lr, false, w->stream);
+  if (rc) return rc;
+  if (loss_out) return finish_loss(w, batch, loss_out, w->stream);
+  return HB_OK;
+}
+
+int mlp_step_grads(hb_worker* w, const void* X, int64_t ldx, int32_t x_dtype, const int32_t* y, int32_t batch,
+                   float* host_grads, int64_t n, float* loss_out) {
+  int rc = check_step_args(w, X, ldx, x_dtype, y, batch);
+  if (rc) return rc;
+  hb_model* m = w->m;
+  int64_t need;
+  mlp_num_params(m, &need);
+  HB_CHECK_ARG(host_grads && n == need, "n must equal mlp_num_params");
+  HB_CUDA_TRY(cudaSetDevice(m->device));
+  if (!w->grads) HB_CUDA_TRY(cudaMalloc(&w->grads, m->total * 4));
+  HB_CUDA_TRY(cudaMemsetAsync(w->grads, 0, m->total * 4, w->stream));
+  rc = run_step(w, X, ldx, x_dtype, y, batch, 0.f, true, w->stream);
+  if (rc) return rc;
+  std::vector<float> h(m->total);
+  HB_CUDA_TRY(cudaMemcpyAsync(h.data(), w->grads, m->total * 4, cudaMemcpyDeviceToHost, w->stream));
+  HB_CUDA_TRY(cudaStreamSynchronize(w->stream));
+  int64_t o = 0;
+  for (const Layer& Ly : m->layers) {
+    for (int i = 0; i < Ly.n_out; ++i)
+      for (int j = 0; j < Ly.n_in; ++j) host_grads[o++] = h[Ly.w_off + (size_t)i * Ly.ldw + j];
+    for (int i = 0; i < Ly.n_out; ++i) host_grads[o++] = h[Ly.b_off + i];
+  }
+  if (loss_out) return finish_loss(w, batch, loss_out, w->stream);
+  return HB_OK;
+}
+
+int mlp_loss(hb_model* m, const void* X, int64_t ldx, int32_t x_dtype, const int32_t* y, int64_t n,
+             double* loss_out) {
+  HB_CHECK_ARG(m && loss_out, "null arg");
+  HB_CHECK_ARG(n >= 1, "n must be >= 1");
+  HB_CUDA_TRY(cudaSetDevice(m->device));
+  HB_CUDA_TRY(cudaDeviceSynchronize());  // see every update enqueued before this call
+  const int chunk = 8192;
+  std::lock_guard<std::mutex> g(m->eval_mu);
+  if (!m->eval) {
+    int rc = alloc_worker(m, chunk, m->stream, false, &m->eval);
+    if (rc) return rc;
+  }
+  hb_worker* w = m->eval;
+  int rc = check_step_args(w, X, ldx, x_dtype, y, (int)std::min<int64_t>(n, chunk));
+  if (rc) return rc;
+  const int64_t nchunks = (n + chunk - 1) / chunk;
+  if (m->chunk_cap < nchunks) {
+    cudaFree(m->chunk_sums);
+    m->chunk_sums = nullptr;
+    HB_CUDA_TRY(cudaMalloc(&m->chunk_sums, nchunks * sizeof(double)));
+    m->chunk_cap = nchunks;
+  }
+  const int L = (int)m->layers.size();
+  const bool bf = m->prec == HB_PREC_BF16;
+  const size_t xes = x_dtype == HB_BF16 ? 2 : 4;
+  cudaStream_t s = w->stream;
+  for (int64_t c = 0; c < nchunks; ++c) {
+    const int64_t r0 = c * chunk;
+    const int b = (int)std::min<int64_t>(chunk, n - r0);
+    const void* Ain = static_cast<const char*>(X) + r0 * ldx * xes;
+    int64_t lda = ldx;
+    int adt = x_dtype;
+    for (int l = 0; l < L; ++l) {
+      const Layer& Ly = m->layers[l];
+      EpiArgs ep{};
+      ep.M = b;
+      ep.N = Ly.n_out;
+      ep.bias = m->master + Ly.b_off;
+      int epi;
+      if (l < L - 1) {
+        epi = EPI_FWD_SIG;
+        ep.out0 = w->H[l];
+        ep.ld0 = Ly.ldo;
+      } else {
+        epi = EPI_FWD_LOGITS;
+        ep.out0 = w->logits;
+        ep.ld0 = w->ldc;
+      }
+      const void* Wp = bf ? (const void*)(m->shadow + Ly.w_off) : (const void*)(m->master + Ly.w_off);
+      rc = gemm(m, epi, false, false, b, Ly.n_out, Ly.n_in, Ain, lda, adt, Wp, Ly.ldw, bf ? HB_BF16 : HB_F32, ep, s);
+      if (rc) return rc;
+      if (l < L - 1) {
+        Ain = w->H[l];
+        lda = Ly.ldo;
+        adt = act_dt(m);
+      }
+    }
+    const int blocks = (b * 32 + 255) / 256;
+    softmax_xent_kernel<float><<<blocks, 256, 0, s>>>(w->logits, w->ldc, y + r0, b, m->layers.back().n_out,
+                                                     (float*)nullptr, 0, w->row_loss, 1.0f);
+    sum_rows_kernel<<<1, 1024, 0, s>>>(w->row_loss, b, m->chunk_sums, (int)c);
+    HB_CUDA_TRY(cudaGetLastError());
+  }
+  std::vector<double> h(nchunks);
+  HB_CUDA_TRY(cudaMemcpyAsync(h.data(), m->chunk_sums, nchunks * sizeof(double), cudaMemcpyDeviceToHost, s));
+  HB_CUDA_TRY(cudaStreamSynchronize(s));
+  double tot = 0.0;
+  for (double v : h) tot += v;
+  *loss_out = tot / (double)n;
+  return HB_OK;
+}
+
+}  // extern "C"

@@ -1,0 +1,67 @@
+// model.h — internal definitions of hb_model / hb_worker (not part of the ABI).
+#pragma once
+
+#include <cuda_bf16.h>
+#include <cuda_runtime.h>
+
+#include <mutex>
+#include <vector>
+
+#include "../../include/hogbatch.h"
+
+namespace hb {
+
+// One fully-connected layer W_l [n_out x n_in] (row stride ldw, padded to 8 elements so every
+// bf16 row is 16-byte aligned for TMA) and bias b_l [n_out]; offsets index the flat parameter
+// buffers (fp32 master, bf16 shadow share the indexing).
+struct Layer {
+  int n_in = 0, n_out = 0;
+  int ldw = 0;  // row stride of W (elements)
+  int ldo = 0;  // row stride of this layer's activations / gradients (elements)
+  size_t w_off = 0, b_off = 0;
+};
+
+int choose_bn(int M, int N);
+
+}  // namespace hb
+
+struct hb_model {
+  int device = 0;
+  int prec = HB_PREC_BF16;
+  std::vector<int> dims;
+  std::vector<hb::Layer> layers;
+  size_t total = 0;                 // floats in the flat parameter buffer (incl. padding)
+  float* master = nullptr;          // fp32 master weights + biases (the shared global model)
+  __nv_bfloat16* shadow = nullptr;  // bf16 copy read by the tensor cores
+  float* base = nullptr;            // merge base W_base (hb_merge_begin)
+  float* delta = nullptr;           // merge send/recv buffer
+  cudaStream_t stream = nullptr;    // internal stream (loss evaluation, merges)
+  hb_worker* eval = nullptr;        // scratch for mlp_loss
+  std::mutex eval_mu;
+  double* chunk_sums = nullptr;
+  int64_t chunk_cap = 0;
+};
+
+struct hb_worker {
+  hb_model* m = nullptr;
+  int max_b = 0;
+  cudaStream_t stream = nullptr;
+  bool own_stream = false;
+  std::vector<void*> H, S, dZ;  // per-layer activations, sigma' stash, output gradients
+  float* logits = nullptr;      // [max_b x ldc] fp32
+  int ldc = 0;
+  float* row_loss = nullptr;    // [max_b]
+  float* partial = nullptr;     // [splits x max width] bias-gradient partial sums
+  int splits_max = 0;
+  double* dsum = nullptr;
+  double* h_dsum = nullptr;     // pinned
+  float* grads = nullptr;       // mlp_step_grads output (flat padded layout)
+};
+
+namespace hb {
+int run_step(hb_worker* w, const void* X, int64_t ldx, int32_t xdt, const int32_t* y, int b, float lr,
+             bool grads_only, cudaStream_t s);
+int finish_loss(hb_worker* w, int b, float* loss_out, cudaStream_t s);
+// enqueue sum of the last step's per-row losses into *dst (device double)
+void sum_rows_into(hb_worker* w, int b, double* dst, cudaStream_t s);
+}  // namespace hb

@@ -1,0 +1,119 @@
+"""GPU parity: the CUDA path (through the C ABI) against the fp64 oracle.
+
+Tolerances (BASELINE.json north_star): normwise relative error per tensor
+<= 1e-2 for the bf16 tensor-core path, <= 1e-5 for the fp32 CUDA-core check mode.
+The oracle sees exactly the GPU's inputs: bf16-exact X and fp32-exact parameters, in fp64.
+"""
+import numpy as np
+import pytest
+
+torch = pytest.importorskip("torch")
+pytestmark = pytest.mark.gpu
+
+import paper_conf_ipps_marws21_b200 as hb  # noqa: E402
+from oracle import mlp64  # noqa: E402
+from tests.helpers import dataset, init_params, params_to_flat, rel_err, split_flat, to_device  # noqa: E402
+
+TOL = {"bf16": 1e-2, "fp32": 1e-5}
+
+
+def _need_gpu():
+    if not torch.cuda.is_available() or not hb.device_ok(0):
+        pytest.fail("no sm_100 GPU visible: the -m gpu tests must run on a B200")
+
+
+def make(dims, prec, max_batch, seed=2, scale=1.0):
+    _need_gpu()
+    m = hb.MLP(dims, precision=prec, seed=0)
+    params = init_params(dims, seed=seed, scale=scale)
+    m.set_params(params_to_flat(params))
+    w = hb.Worker(m, max_batch)
+    return m, w, params
+
+
+def grads_case(dims, kind, b, prec, scale=1.0, d=None):
+    X, y = dataset(kind, b, d=d or dims[0], seed=7)
+    y = (y % dims[-1]).astype(np.int32)
+    m, w, params = make(dims, prec, b, scale=scale)
+    tX, ty = to_device(X, y, "bf16" if prec == "bf16" else "f32")
+    g, loss = w.step_grads(tX, ty, b)
+    dW, db, l_ref = mlp64.grads(params, X.astype(np.float64), y)
+    got = split_flat(g, dims)
+    errs = []
+    for l in range(len(dims) - 1):
+        errs.append(rel_err(got[l][0], dW[l]))
+        errs.append(rel_err(got[l][1], db[l]))
+    return max(errs), abs(loss - l_ref) / l_ref, errs
+
+
+CASES = [
+    # (dims, dataset kind, batch) — tiny C1, ragged batches/widths, paper-shaped heads
+    ([54, 64, 64, 7], "covtype", 32),
+    ([54, 64, 64, 7], "covtype", 1),
+    ([54, 512, 512, 7], "covtype", 300),
+    ([54, 200, 136, 7], "covtype", 129),
+    ([300, 1024, 1024, 2], "w8a", 1000),
+    ([2000, 256, 2], "realsim", 200),
+    ([24, 40, 3], "gauss", 77),
+]
+
+
+@pytest.mark.parametrize("dims,kind,b", CASES)
+def test_gradients_bf16_tensor_cores(dims, kind, b):
+    e, le, errs = grads_case(dims, kind, b, "bf16")
+    assert e <= TOL["bf16"], errs
+    assert le <= TOL["bf16"]
+
+
+@pytest.mark.parametrize("dims,kind,b", CASES)
+def test_gradients_fp32_check_mode(dims, kind, b):
+    e, le, errs = grads_case(dims, kind, b, "fp32")
+    assert e <= TOL["fp32"], errs
+    assert le <= 1e-6
+
+
+def test_gradients_saturated_init_bf16():
+    # hard part: sigma' near saturation; S = sigma'(z) is stashed from fp32, not from bf16 H
+    e, _, errs = grads_case([54, 512, 512, 512, 512, 7], "covtype", 256, "bf16", scale=4.0)
+    assert e <= TOL["bf16"], errs
+
+
+@pytest.mark.parametrize("prec", ["bf16", "fp32"])
+def test_one_sgd_step_updates_model_in_place(prec):
+    dims = [54, 128, 64, 7]
+    X, y = dataset("covtype", 256, seed=3)
+    m, w, params = make(dims, prec, 256)
+    tX, ty = to_device(X, y, "bf16" if prec == "bf16" else "f32")
+    lr = 0.5
+    loss = w.step(tX, ty, 256, lr, want_loss=True)
+    new, l_ref = mlp64.sgd_step(params, X.astype(np.float64), y, lr)
+    got = split_flat(m.get_params(), dims)
+    for l in range(3):
+        # compare the UPDATE (W_new - W_old) normwise; the params themselves agree far tighter
+        assert rel_err(got[l][0] - params[l][0], new[l][0] - params[l][0]) <= TOL[prec]
+        assert rel_err(got[l][1] - params[l][1], new[l][1] - params[l][1]) <= TOL[prec]
+    assert abs(loss - l_ref) / l_ref <= TOL[prec]
+
+
+@pytest.mark.parametrize("prec", ["bf16", "fp32"])
+def test_mlp_loss_full_data(prec):
+    dims = [54, 96, 7]
+    X, y = dataset("covtype", 20000, seed=1)
+    m, w, params = make(dims, prec, 64)
+    tX, ty = to_device(X, y, "bf16" if prec == "bf16" else "f32")
+    got = m.loss(tX, ty)
+    ref = mlp64.full_loss(params, X.astype(np.float64), y)
+    assert abs(got - ref) / ref <= (1e-3 if prec == "bf16" else 1e-6)
+
+
+def test_step_argument_errors():
+    dims = [54, 64, 7]
+    X, y = dataset("covtype", 64, seed=1)
+    m, w, _ = make(dims, "bf16", 32)
+    tX, ty = to_device(X, y)
+    with pytest.raises(hb.HogbatchError):
+        w.step(tX, ty, 33, 0.1)          # batch > max_batch
+    with pytest.raises(hb.HogbatchError):
+        w.step(tX, ty, 0, 0.1)           # empty batch
+    with pytest.raises(hb.HogbatchError):
+        w.step(tX.float(), ty, 8, 0.1)   # bf16 model needs bf16 X
