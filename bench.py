@@ -1,0 +1,403 @@
+#!/usr/bin/env python
+"""bench.py — MLP-SGD throughput of the Adaptive Hogbatch hot path on B200.
+
+    python bench.py [--gpus N] [--steps K] [--warmup W] [--impl ours|reference] [--config covtype]
+
+One STEP = one Adaptive Hogbatch epoch (hogbatch_run, Alg. 2) over the rank's
+synthetic dataset, i.e. one pass of every hot-path row: batch selection, forward GEMM chain,
+softmax-xent head, dX/dW GEMMs with the fused in-place SGD, the adaptive batch-size rule.
+Loss evaluation is excluded.  Default workload = BASELINE.json configs[1]:
+covtype-shaped 581,012 x 54, 7 classes, MLP 54-512x4-7, Adaptive Hogbatch with a large-batch
+and a small-batch worker on one B200.  N > 1 ranks (torchrun): each rank trains its own
+dataset shard of the same size (weak scaling) and the replicas are merged over NCCL
+ `--merges` times per epoch.
+
+Timing: W warm-up steps, then K steps each bracketed by CUDA events on the legacy default
+stream (the library's worker streams are blocking streams, so the events bracket all their
+work); the L2 is flushed (256 MiB write) between timed steps; max over ranks.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import statistics
+import subprocess
+import sys
+import threading
+import time
+
+import numpy as np
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+CONFIGS = {
+    # name: dataset, dims, N, large-worker max b, small worker range
+    "covtype": dict(data="covtype", dims=[54, 512, 512, 512, 512, 7], N=581012,
+                    workload="covtype-shaped 581012x54, 7 classes, MLP 54-512x4-7 sigmoid/softmax-CE"),
+    "w8a": dict(data="w8a", dims=[300, 1024, 1024, 1024, 2], N=64700,
+                workload="w8a-shaped 64700x300, 2 classes, MLP 300-1024x3-2"),
+    "realsim": dict(data="realsim", dims=[20958, 4096, 4096, 4096, 4096, 2], N=72309,
+                    workload="real-sim-shaped 72309x20958 (dense), 2 classes, MLP 20958-4096x4-2"),
+    "tiny": dict(data="covtype", dims=[54, 64, 64, 7], N=10000,
+                 workload="tiny covtype-shaped 10000x54, MLP 54-64-64-7, batch 32"),
+}
+
+
+def flops_per_sample(dims):
+    P = sum(dims[i] * dims[i - 1] for i in range(1, len(dims)))
+    return 6 * P - 2 * dims[0] * dims[1]
+
+
+def load_peaks():
+    try:
+        with open(os.path.join(ROOT, "MEASURED_PEAKS.json")) as f:
+            p = json.load(f)
+        return dict(hbm=p["hbm_gbs"], bf16=p["bf16_tflops"], bf16_sus=p.get("bf16_tflops_sustained", p["bf16_tflops"]),
+                    src="measured")
+    except Exception:
+        return dict(hbm=6650.0, bf16=1590.0, bf16_sus=1400.0, src="fallback")
+
+
+class ClockSampler:
+    """nvidia-smi clocks/throttle reasons sampled during the timed region (B200_PROFILING.md)."""
+    Q = ("index,clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.active,"
+         "clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown,"
+         "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, index):
+        self.index, self.lines, self.proc = index, [], None
+
+    def start(self):
+        try:
+            self.proc = subprocess.Popen(["nvidia-smi", "-i", str(self.index), "--query-gpu=" + self.Q,
+                                          "--format=csv,noheader,nounits", "-lms", "200"],
+                                         stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
+            self.t = threading.Thread(target=self._read, daemon=True)
+            self.t.start()
+        except Exception:
+            self.proc = None
+
+    def _read(self):
+        for line in self.proc.stdout:
+            self.lines.append(line.strip())
+
+    def stop(self):
+        if not self.proc:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["nvidia-smi unavailable"]}
+        self.proc.terminate()
+        try:
+            self.proc.wait(timeout=2)
+        except Exception:
+            self.proc.kill()
+        sm, mx, reasons = [], None, set()
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        for ln in self.lines:
+            f = [x.strip() for x in ln.split(",")]
+            if len(f) < 9:
+                continue
+            try:
+                sm.append(float(f[1]))
+                mx = float(f[2])
+            except ValueError:
+                continue
+            for n, v in zip(names, f[5:9]):
+                if v.lower() == "active":
+                    reasons.add(n)
+        return {"sm_mhz": statistics.median(sm) if sm else None, "sm_max_mhz": mx,
+                "reasons": sorted(reasons), "samples": len(sm)}
+
+
+def make_data(cfg, rank, N):
+    from synth import covtype_like, pad_cols
+    from synth.data import csr_to_dense, sparse_like
+    d = cfg["dims"][0]
+    if cfg["data"] == "covtype":
+        X, y = covtype_like(N, seed=rank)
+        return pad_cols(X, (d + 7) // 8 * 8), y
+    if cfg["data"] == "w8a":
+        csr, y = sparse_like(N, 300, 11.6, 0.03, True, seed=rank)
+    else:
+        csr, y = sparse_like(N, 20958, 51.5, 0.31, False, seed=rank)
+    return csr_to_dense(csr, d, (d + 7) // 8 * 8), y
+
+
+# --------------------------------------------------------------------------------------------
+# reference arm: the fp64 oracle on the host cores (bounded sample of the same workload)
+# --------------------------------------------------------------------------------------------
+def oracle_arm(cfg, args, rows_per_step, budget_note):
+    from threadpoolctl import threadpool_info
+    from oracle import mlp64
+    from synth import init_params
+    dims = cfg["dims"]
+    b = min(8192, rows_per_step)
+    Xp, y = make_data(cfg, 0, rows_per_step)
+    X = Xp[:, :dims[0]].astype(np.float64)
+    params = init_params(dims, seed=2)
+    lr = args.eta0 * b / args.b0
+
+    def step(P):
+        for s in range(0, rows_per_step - b + 1, b):
+            P, _ = mlp64.sgd_step(P, X[s:s + b], y[s:s + b], lr)
+        return P
+
+    for _ in range(args.warmup):
+        params = step(params)
+    times = []
+    for _ in range(args.steps):
+        t0 = time.perf_counter()
+        params = step(params)
+        times.append(time.perf_counter() - t0)
+    cores = sum(i.get("num_threads", 0) for i in threadpool_info() if i.get("internal_api") in ("openblas", "mkl")) or 1
+    per = (rows_per_step // b) * b
+    return per / statistics.mean(times), cores, statistics.mean(times), budget_note
+
+
+def cpu_baseline(cfg, args):
+    # ~10-20 s of CPU work: 3 warm-up-free steps of 65,536 rows (8 batches of 8192)
+    class A:
+        pass
+    a = A()
+    a.warmup, a.steps, a.eta0, a.b0 = 0, 1, args.eta0, args.b0
+    rows = 65536 if cfg["dims"][1] <= 1024 else 1024
+    v, cores, t, _ = oracle_arm(cfg, a, rows, "")
+    return {"value": v, "unit": "samples/s", "cores": cores, "kind": "oracle",
+            "sample": f"fp64 NumPy oracle SGD steps (batch {min(8192, rows)}) over the first {rows} rows of the "
+                      f"same synthetic dataset, {t:.1f} s"}
+
+
+# --------------------------------------------------------------------------------------------
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=10)
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
+    ap.add_argument("--config", default="covtype", choices=list(CONFIGS))
+    ap.add_argument("--policy", default="adaptive", choices=["adaptive", "minibatch"])
+    ap.add_argument("--eta0", type=float, default=0.05)
+    ap.add_argument("--b0", type=int, default=32)
+    ap.add_argument("--merges", type=int, default=4, help="replica merges per epoch (N > 1)")
+    ap.add_argument("--n", type=int, default=0, help="rows per rank (default: the config's N)")
+    ap.add_argument("--e2e-steps", type=int, default=3)
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--no-prof", action="store_true")
+    args = ap.parse_args()
+    cfg = CONFIGS[args.config]
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    N = args.n or cfg["N"]
+    dims = cfg["dims"]
+    F = flops_per_sample(dims)
+
+    if args.impl == "reference":
+        if rank != 0:
+            return
+        rows = 65536 if dims[1] <= 1024 else 1024
+        v, cores, t, _ = oracle_arm(cfg, args, rows, "")
+        line = {"impl": "reference", "metric": f"MLP SGD samples/sec ({args.config})", "value": v,
+                "unit": "samples/s", "n_gpus": 0, "steps": args.steps, "warmup": args.warmup,
+                "ms_per_step": t * 1e3, "higher_is_better": True, "scaling": "weak", "vs_baseline": None,
+                "dtype": "f64", "data": "synthetic",
+                "config": {"workload": cfg["workload"], "sample_rows_per_step": rows},
+                "cpu_baseline": {"value": v, "unit": "samples/s", "cores": cores, "kind": "oracle",
+                                 "sample": f"fp64 NumPy oracle, {rows} rows per step (batch {min(8192, rows)})"},
+                "e2e": {"value": v, "unit": "samples/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
+        print(json.dumps(line), flush=True)
+        return
+
+    import torch
+    import torch.distributed as dist
+    torch.cuda.set_device(local)
+    if world > 1:
+        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+    import paper_conf_ipps_marws21_b200 as hb
+    from synth import init_params, params_to_flat
+
+    # ---- data + model (resident in HBM before timing) ----
+    Xp, y = make_data(cfg, rank, N)
+    ld = Xp.shape[1]
+    X_host = torch.from_numpy(Xp).to(torch.bfloat16).pin_memory()
+    y_host = torch.from_numpy(y.astype(np.int32)).pin_memory()
+    Xd = X_host.to(f"cuda:{local}")
+    yd = y_host.to(f"cuda:{local}")
+    model = hb.MLP(dims, precision="bf16", seed=0, device=local)
+    model.set_params(params_to_flat(init_params(dims, seed=2)))
+    big_max = 8192
+    wl = hb.Worker(model, big_max)
+    torch.cuda.synchronize()
+
+    # ---- lower threshold of the large worker: smallest power of 2 with >= 50% of the
+    #      samples/s at the upper threshold ("GPU utilization for the lower
+    #      threshold is about 50%") — calibrated on this GPU, outside the timed region ----
+    def step_rate(b, reps=6):
+        for _ in range(2):
+            wl.step(Xd, yd, b, 0.0)
+        s0, s1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        torch.cuda.synchronize()
+        s0.record()
+        for i in range(reps):
+            wl.step(Xd[i * b:], yd[i * b:], b, 0.0)
+        s1.record()
+        torch.cuda.synchronize()
+        return b * reps / (s0.elapsed_time(s1) * 1e-3)
+    params0 = params_to_flat(init_params(dims, seed=2))
+    if args.policy == "adaptive" and args.config != "tiny":
+        r_max = step_rate(big_max)
+        big_min = big_max
+        b = big_max // 2
+        while b >= 64 and step_rate(b) >= 0.5 * r_max:
+            big_min = b
+            b //= 2
+        model.set_params(params0)
+        ws = hb.Worker(model, 2048)
+        workers = [wl, ws]
+        specs = [hb.WorkerSpec(big_min, big_max, big_max), hb.WorkerSpec(32, 2048, 32)]
+        pol = hb.Policy(kind=hb.HB_ADAPTIVE, workers=specs, eta0=args.eta0, b0=args.b0)
+    else:
+        bsz = 32 if args.config == "tiny" else big_max
+        big_min = bsz
+        workers = [wl]
+        specs = [hb.WorkerSpec(bsz, bsz, bsz)]
+        pol = hb.Policy(kind=hb.HB_MINIBATCH, workers=specs, eta0=args.eta0, b0=args.b0)
+    comm = None
+    if world > 1:
+        uid = [hb.Comm.unique_id() if rank == 0 else None]
+        dist.broadcast_object_list(uid, src=0)
+        comm = hb.Comm(uid[0], world, rank, local)
+        model.merge_begin()
+        pol.comm = comm
+        pol.merges_per_epoch = args.merges
+
+    flush = torch.empty(256 << 20, dtype=torch.uint8, device=f"cuda:{local}")
+
+    def run_epoch():
+        return hb.hogbatch_run(workers, pol, Xd, yd, epochs=1)
+
+    for _ in range(args.warmup):
+        run_epoch()
+    torch.cuda.synchronize()
+    if world > 1:
+        dist.barrier()
+    if not args.no_prof:
+        hb.prof_read(reset=True)
+        hb.prof_enable(True)
+    clocks = ClockSampler(local)
+    clocks.start()
+    l0 = hb.kernel_launches()
+    ms, samples, share = [], 0, np.zeros(len(workers))
+    bsz_hist = {}
+    for _ in range(args.steps):
+        flush.zero_()
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        if world > 1:
+            dist.barrier()
+        torch.cuda.synchronize()
+        e0.record()
+        st = run_epoch()
+        e1.record()
+        torch.cuda.synchronize()
+        ms.append(e0.elapsed_time(e1))
+        samples += st["total_samples"]
+        share += st["updates"][0]
+    launches = hb.kernel_launches() - l0
+    clk = clocks.stop()
+    prof = hb.prof_read(reset=True) if not args.no_prof else None
+    hb.prof_enable(False)
+    tot_ms = sum(ms)
+    t = torch.tensor([tot_ms], device=f"cuda:{local}")
+    s = torch.tensor([float(samples)], device=f"cuda:{local}")
+    if world > 1:
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        dist.all_reduce(s, op=dist.ReduceOp.SUM)
+    value = s.item() / (t.item() * 1e-3)
+
+    # ---- e2e: host (pinned) -> device copy of the step's inputs + the step + D2H of the
+    #      trained parameters, through the public API, every step ----
+    e2e_ms, e2e_samples = [], 0
+    h2d = X_host.numel() * 2 + y_host.numel() * 4
+    d2h = model.num_params * 4
+    for _ in range(args.e2e_steps):
+        flush.zero_()
+        if world > 1:
+            dist.barrier()
+        torch.cuda.synchronize()
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        e0.record()
+        Xd.copy_(X_host, non_blocking=True)
+        yd.copy_(y_host, non_blocking=True)
+        st = run_epoch()
+        _ = model.get_params()
+        e1.record()
+        torch.cuda.synchronize()
+        e2e_ms.append(e0.elapsed_time(e1))
+        e2e_samples += st["total_samples"]
+    te = torch.tensor([sum(e2e_ms)], device=f"cuda:{local}")
+    se = torch.tensor([float(e2e_samples)], device=f"cuda:{local}")
+    if world > 1:
+        dist.all_reduce(te, op=dist.ReduceOp.MAX)
+        dist.all_reduce(se, op=dist.ReduceOp.SUM)
+    e2e_value = se.item() / (te.item() * 1e-3) if args.e2e_steps else None
+
+    if rank == 0:
+        peaks = load_peaks()
+        roof = None
+        if prof:
+            gem = {k: v for k, v in prof.items() if v["launches"] and v["ms"] > 0}
+            dom = max(gem, key=lambda k: gem[k]["ms"])
+            d = gem[dom]
+            ai = d["flops"] / d["bytes"] if d["bytes"] else 0.0
+            ridge = peaks["bf16_sus"] * 1e12 / (peaks["hbm"] * 1e9)
+            if d["flops"] > 0 and ai >= ridge:
+                ach, peak, unit, bound = d["flops"] / (d["ms"] * 1e-3) / 1e12, peaks["bf16_sus"], "TFLOP/s", "tensor"
+            else:
+                ach, peak, unit, bound = d["bytes"] / (d["ms"] * 1e-3) / 1e9, peaks["hbm"], "GB/s", "hbm"
+            traffic = None
+            try:
+                with open(os.path.join(ROOT, "profiles", "ncu_traffic.json")) as f:
+                    traffic = json.load(f).get(args.config, {}).get(dom)
+            except Exception:
+                pass
+            roof = {"bound": bound, "achieved": ach, "peak": peak, "unit": unit, "frac": ach / peak,
+                    "traffic": traffic, "kernel": dom, "launches": d["launches"],
+                    "ms_per_launch": d["ms"] / d["launches"],
+                    "flops_per_launch": d["flops"] / d["launches"], "bytes_per_launch": d["bytes"] / d["launches"],
+                    "peak_source": f"{peaks['src']} ({'bf16_tflops_sustained' if bound == 'tensor' else 'hbm_gbs'})",
+                    "classes": {k: {"ms": round(v["ms"], 3), "launches": v["launches"],
+                                    "TFLOP/s": round(v["flops"] / (v["ms"] * 1e-3) / 1e12, 1) if v["ms"] else None,
+                                    "GB/s": round(v["bytes"] / (v["ms"] * 1e-3) / 1e9, 1) if v["ms"] else None}
+                                for k, v in gem.items()}}
+        cpu = None
+        if not args.no_cpu_baseline and world == 1:
+            cpu = cpu_baseline(cfg, args)
+        line = {
+            "metric": f"MLP SGD samples/sec ({'Adaptive Hogbatch' if args.policy == 'adaptive' else 'mini-batch'}, {args.config})",
+            "value": value, "unit": "samples/s", "n_gpus": world, "steps": args.steps, "warmup": args.warmup,
+            "ms_per_step": t.item() / args.steps, "higher_is_better": True, "scaling": "weak", "vs_baseline": None,
+            "dtype": "bf16", "data": "synthetic",
+            "config": {"workload": cfg["workload"] + (", Adaptive Hogbatch: large worker [%d, %d] init %d + small "
+                                                      "worker [32, 2048] init 32, shared model (Hogwild)"
+                                                      % (big_min, big_max, big_max) if args.policy == "adaptive" else ""),
+                       "rows_per_rank": N, "step": "one hogbatch_run epoch per rank",
+                       "eta0_at_b0": [args.eta0, args.b0], "merges_per_epoch": args.merges if world > 1 else 0,
+                       "l2": "flushed between timed steps (256 MiB write)"},
+            "tc_peak_frac": value * F / (world * peaks["bf16_sus"] * 1e12),
+            "flops_per_sample": F,
+            "update_share": (share / share.sum()).round(4).tolist() if share.sum() else None,
+            "roofline": roof,
+            "cpu_baseline": cpu,
+            "e2e": {"value": e2e_value, "unit": "samples/s", "h2d_bytes_per_step": h2d, "d2h_bytes_per_step": d2h},
+            "gpu_launches": launches,
+            "clocks": clk,
+        }
+        print(json.dumps(line), flush=True)
+    if comm is not None:
+        comm.close()
+    if world > 1:
+        dist.destroy_process_group()
+
+
+if __name__ == "__main__":
+    main()

@@ -191,6 +191,30 @@ int hb_schedule_trace(const hb_policy* p, int64_t N, int32_t epochs, hb_trace_re
 int hogbatch_run(hb_worker** workers, int32_t n_workers, const hb_policy* p,
                  const hb_dataset* data, int32_t epochs, hb_stats* stats_out);
 
+/* ---- instrumentation ----------------------------------------------------------------
+ * hb_kernel_launches: number of CUDA kernels this library launched in this process.
+ * hb_prof_enable(1): every kernel launch of the hot path is bracketed by CUDA events on its
+ * own stream; hb_prof_read (blocking: synchronises the device) accumulates per class the
+ * launch count, device milliseconds and the ALGORITHMIC flops / bytes of those launches
+ * (DESIGN.md §Roofline), writes n <= HB_PROF_N entries and optionally resets. */
+enum {
+  HB_PROF_FWD_GEMM = 0,   /* hidden-layer forward GEMM + bias + sigmoid/sigma' epilogue */
+  HB_PROF_HEAD_GEMM = 1,  /* output-layer forward GEMM (logits)                         */
+  HB_PROF_SOFTMAX = 2,    /* softmax cross-entropy + dZ_L                               */
+  HB_PROF_DGRAD_GEMM = 3, /* dX GEMM + sigma' epilogue                                  */
+  HB_PROF_WGRAD_GEMM = 4, /* dW GEMM + fused in-place SGD epilogue                      */
+  HB_PROF_BIAS = 5,       /* bias gradient + bias SGD                                   */
+  HB_PROF_OTHER = 6,      /* loss reduction, shadow refresh, merge kernels              */
+  HB_PROF_N = 7
+};
+typedef struct hb_prof_entry {
+  int64_t launches;
+  double ms, flops, bytes;
+} hb_prof_entry;
+int64_t hb_kernel_launches(void);
+int hb_prof_enable(int32_t on);
+int hb_prof_read(hb_prof_entry* out, int32_t n, int32_t reset);
+
 /* ---- multi-GPU replica merge over NCCL (future work L277) -------- */
 int hb_nccl_unique_id(uint8_t out[128]);
 int hb_comm_create(const uint8_t id[128], int32_t nranks, int32_t rank, int32_t device,

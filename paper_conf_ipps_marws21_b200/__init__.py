@@ -250,5 +250,23 @@ class Comm:
             self.h = None
 
 
+def kernel_launches() -> int:
+    """Kernels this library has launched in this process."""
+    return int(lib.hb_kernel_launches())
+
+
+def prof_enable(on: bool = True):
+    _check(lib.hb_prof_enable(int(on)))
+
+
+def prof_read(reset: bool = False) -> dict:
+    """Per kernel class: launches, device ms, algorithmic flops and bytes (blocking)."""
+    n = len(_lib.PROF_CLASSES)
+    buf = (_lib.ProfEntry * n)()
+    _check(lib.hb_prof_read(buf, n, int(reset)))
+    return {name: dict(launches=buf[i].launches, ms=buf[i].ms, flops=buf[i].flops, bytes=buf[i].bytes)
+            for i, name in enumerate(_lib.PROF_CLASSES)}
+
+
 def pad_to(n: int, m: int = 8) -> int:
     return (n + m - 1) // m * m

@@ -25,7 +25,9 @@ EXPORTS = ("hb_last_error", "hb_abi_version", "hb_device_ok", "mlp_create", "mlp
            "mlp_num_params", "mlp_get_params", "mlp_set_params", "mlp_worker_create",
            "mlp_worker_destroy", "mlp_worker_stream", "mlp_step", "mlp_step_grads", "mlp_loss",
            "hb_schedule_trace", "hogbatch_run", "hb_nccl_unique_id", "hb_comm_create",
-           "hb_comm_destroy", "hb_merge_begin", "hb_merge")
+           "hb_comm_destroy", "hb_merge_begin", "hb_merge", "hb_kernel_launches", "hb_prof_enable",
+           "hb_prof_read")
+PROF_CLASSES = ("fwd_gemm", "head_gemm", "softmax_xent", "dgrad_gemm", "wgrad_sgd_gemm", "bias_sgd", "other")
 
 
 class WorkerPolicy(C.Structure):
@@ -64,9 +66,13 @@ class Stats(C.Structure):
                 ("total_samples", C.c_int64), ("n_merges", C.c_int32)]
 
 
+class ProfEntry(C.Structure):
+    _fields_ = [("launches", C.c_int64), ("ms", C.c_double), ("flops", C.c_double), ("bytes", C.c_double)]
+
+
 def load():
     if not os.path.exists(LIB_PATH):
-        raise ImportError(f"{LIB_PATH} is missing: run `python -m paper_conf_ipps_marws21_b200.build` "
+        raise ImportError(f"{LIB_PATH} is missing: run `python paper_conf_ipps_marws21_b200/build.py` "
                           "(there is no CPU fallback)")
     lib = C.CDLL(LIB_PATH)
     P, I32, I64, F, D, VP = C.POINTER, C.c_int32, C.c_int64, C.c_float, C.c_double, C.c_void_p
@@ -92,6 +98,9 @@ def load():
         "hb_comm_destroy": ([VP], C.c_int),
         "hb_merge_begin": ([VP], C.c_int),
         "hb_merge": ([VP, VP, F, VP], C.c_int),
+        "hb_kernel_launches": ([], I64),
+        "hb_prof_enable": ([I32], C.c_int),
+        "hb_prof_read": ([P(ProfEntry), I32, I32], C.c_int),
     }
     for name, (args, res) in sig.items():
         fn = getattr(lib, name)

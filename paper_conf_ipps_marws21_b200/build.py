@@ -1,6 +1,6 @@
 """Build libhogbatch.so (sm_100a only) in-tree with nvcc.
 
-    python -m paper_conf_ipps_marws21_b200.build        # or __graft_entry__.build()
+    python paper_conf_ipps_marws21_b200/build.py        # or __graft_entry__.build()
 """
 from __future__ import annotations
 

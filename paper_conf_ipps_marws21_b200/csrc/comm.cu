@@ -77,12 +77,14 @@ int hb_merge(hb_model* m, hb_comm* c, float gamma, void* cuda_stream) {
   cudaStream_t s = cuda_stream ? static_cast<cudaStream_t>(cuda_stream) : m->stream;
   HB_CUDA_TRY(cudaDeviceSynchronize());  // every worker's in-place updates are visible
   const int64_t n = (int64_t)m->total;
+  Prof pr(HB_PROF_OTHER, s);
   merge_delta_kernel<<<592, 256, 0, s>>>(m->master, m->base, m->delta, n);
   HB_CUDA_TRY(cudaGetLastError());
   ncclResult_t r = ncclAllReduce(m->delta, m->delta, (size_t)n, ncclFloat, ncclSum, c->comm, s);
   if (r != ncclSuccess) return fail(HB_ENCCL, std::string("ncclAllReduce: ") + ncclGetErrorString(r));
   merge_apply_kernel<<<592, 256, 0, s>>>(m->master, m->base, m->delta, gamma, m->shadow, n);
   HB_CUDA_TRY(cudaGetLastError());
+  pr.done(2, 0.0, 4.0 * 7.0 * n);
   HB_CUDA_TRY(cudaStreamSynchronize(s));
   return HB_OK;
 }

@@ -33,6 +33,53 @@ int fail(int code, const std::string& msg) {
 }
 
 // ----------------------------------------------------------------------------------------
+// instrumentation: launch counter + optional per-launch CUDA-event timing per kernel class
+// ----------------------------------------------------------------------------------------
+std::atomic<int64_t> g_launches{0};
+static std::atomic<bool> g_prof_on{false};
+struct PendRec {
+  cudaEvent_t e0, e1;
+  int cls;
+  double flops, bytes;
+  int nl;
+};
+static std::mutex g_prof_mu;
+static std::vector<PendRec> g_pend;
+static std::vector<cudaEvent_t> g_evpool;
+static hb_prof_entry g_agg[HB_PROF_N];
+
+static cudaEvent_t ev_get() {
+  {
+    std::lock_guard<std::mutex> g(g_prof_mu);
+    if (!g_evpool.empty()) {
+      cudaEvent_t e = g_evpool.back();
+      g_evpool.pop_back();
+      return e;
+    }
+  }
+  cudaEvent_t e = nullptr;
+  cudaEventCreate(&e);
+  return e;
+}
+
+Prof::Prof(int cls_, cudaStream_t s_) : cls(cls_), s(s_) {
+  if (g_prof_on.load(std::memory_order_relaxed)) {
+    e0 = ev_get();
+    cudaEventRecord(e0, s);
+  }
+}
+
+void Prof::done(int nlaunch, double flops, double bytes) {
+  g_launches.fetch_add(nlaunch, std::memory_order_relaxed);
+  if (!e0) return;
+  cudaEvent_t e1 = ev_get();
+  cudaEventRecord(e1, s);
+  std::lock_guard<std::mutex> g(g_prof_mu);
+  g_pend.push_back({e0, e1, cls, flops, bytes, nlaunch});
+  e0 = nullptr;
+}
+
+// ----------------------------------------------------------------------------------------
 // TMA tensor maps (driver entry point; no link-time dependency on libcuda)
 // ----------------------------------------------------------------------------------------
 static PFN_cuTensorMapEncodeTiled_v12000 g_encode = nullptr;
@@ -177,14 +224,36 @@ static int gemm_simt(int epi, bool a_mn, bool b_mn, int M, int N, int K, const v
   }
 }
 
+// algorithmic bytes of one GEMM launch (operands once, epilogue reads/writes once)
+static double gemm_bytes(int epi, int M, int N, int K, double es, bool shadow) {
+  const double mn = (double)M * N, io = ((double)M * K + (double)N * K) * es;
+  switch (epi) {
+    case EPI_FWD_SIG: return io + 2.0 * mn * es + 4.0 * N;
+    case EPI_FWD_LOGITS: return io + 4.0 * mn + 4.0 * N;
+    case EPI_DGRAD_SIG: return io + 2.0 * mn * es;
+    case EPI_WGRAD_SGD: return io + 8.0 * mn + (shadow ? 2.0 * mn : 0.0);
+    default: return io + 4.0 * mn;
+  }
+}
+
 static int gemm(const hb_model* m, int epi, bool a_mn, bool b_mn, int M, int N, int K, const void* A, int64_t lda,
                 int adt, const void* B, int64_t ldb, int bdt, const EpiArgs& ep, cudaStream_t s) {
   if (M <= 0 || N <= 0 || K <= 0) return HB_OK;
+  const int cls = epi == EPI_FWD_SIG ? HB_PROF_FWD_GEMM
+                  : epi == EPI_FWD_LOGITS ? HB_PROF_HEAD_GEMM
+                  : epi == EPI_DGRAD_SIG ? HB_PROF_DGRAD_GEMM
+                                         : HB_PROF_WGRAD_GEMM;
+  Prof pr(cls, s);
+  int rc;
   if (m->prec == HB_PREC_BF16) {
     if (adt != HB_BF16 || bdt != HB_BF16) return fail(HB_EINVAL, "bf16 mode needs bf16 operands (X must be HB_BF16)");
-    return gemm_tc(epi, a_mn, b_mn, M, N, K, A, lda, B, ldb, ep, s);
+    rc = gemm_tc(epi, a_mn, b_mn, M, N, K, A, lda, B, ldb, ep, s);
+  } else {
+    rc = gemm_simt(epi, a_mn, b_mn, M, N, K, A, lda, adt, B, ldb, bdt, ep, s);
   }
-  return gemm_simt(epi, a_mn, b_mn, M, N, K, A, lda, adt, B, ldb, bdt, ep, s);
+  const double es = m->prec == HB_PREC_BF16 ? 2.0 : 4.0;
+  if (!rc) pr.done(1, 2.0 * M * N * (double)K, gemm_bytes(epi, M, N, K, es, ep.shadow != nullptr || ep.out1 != nullptr));
+  return rc;
 }
 
 // ----------------------------------------------------------------------------------------
@@ -305,6 +374,7 @@ int run_step(hb_worker* w, const void* X, int64_t ldx, int32_t xdt, const int32_
     const Layer& Ly = m->layers[L - 1];
     const int threads = 256;
     const int blocks = (b * 32 + threads - 1) / threads;
+    Prof pr(HB_PROF_SOFTMAX, s);
     if (bf)
       softmax_xent_kernel<__nv_bfloat16><<<blocks, threads, 0, s>>>(
           w->logits, w->ldc, y, b, Ly.n_out, static_cast<__nv_bfloat16*>(w->dZ[L - 1]), Ly.ldo, w->row_loss,
@@ -314,6 +384,8 @@ int run_step(hb_worker* w, const void* X, int64_t ldx, int32_t xdt, const int32_
                                                            static_cast<float*>(w->dZ[L - 1]), Ly.ldo,
                                                            w->row_loss, 1.0f / (float)b);
     HB_CUDA_TRY(cudaGetLastError());
+    const double es = bf ? 2.0 : 4.0;
+    pr.done(1, 0.0, (double)b * Ly.n_out * (4.0 + es) + 8.0 * b);
   }
   // ---- backward, Eq. (2), with the update of Eq. (3) fused into the dW GEMM ----
   for (int l = L - 1; l >= 0; --l) {
@@ -359,6 +431,7 @@ int run_step(hb_worker* w, const void* X, int64_t ldx, int32_t xdt, const int32_
     }
     {  // b_l -= lr * 1^T dZ_l (deterministic two-pass column sum)
       const int splits = (b + 127) / 128;
+      Prof pr(HB_PROF_BIAS, s);
       dim3 g1((Ly.n_out + 63) / 64, splits), b1(64, 4);
       if (bf)
         colsum_partial_kernel<__nv_bfloat16><<<g1, b1, 0, s>>>(static_cast<const __nv_bfloat16*>(dZl), Ly.ldo, b,
@@ -370,6 +443,7 @@ int run_step(hb_worker* w, const void* X, int64_t ldx, int32_t xdt, const int32_
                                                                m->master + Ly.b_off,
                                                                grads_only ? w->grads + Ly.b_off : nullptr);
       HB_CUDA_TRY(cudaGetLastError());
+      pr.done(2, (double)b * Ly.n_out, (double)b * Ly.n_out * (bf ? 2.0 : 4.0) + 8.0 * Ly.n_out);
     }
   }
   return HB_OK;
@@ -391,10 +465,13 @@ static int check_step_args(hb_worker* w, const void* X, int64_t ldx, int32_t xdt
 }
 
 void sum_rows_into(hb_worker* w, int b, double* dst, cudaStream_t s) {
+  Prof pr(HB_PROF_OTHER, s);
   sum_rows_kernel<<<1, 1024, 0, s>>>(w->row_loss, b, dst, 0);
+  pr.done(1, 0.0, 4.0 * b);
 }
 
 int finish_loss(hb_worker* w, int b, float* loss_out, cudaStream_t s) {
+  g_launches.fetch_add(1, std::memory_order_relaxed);
   sum_rows_kernel<<<1, 1024, 0, s>>>(w->row_loss, b, w->dsum, 0);
   HB_CUDA_TRY(cudaGetLastError());
   HB_CUDA_TRY(cudaMemcpyAsync(w->h_dsum, w->dsum, sizeof(double), cudaMemcpyDeviceToHost, s));
@@ -408,6 +485,36 @@ int finish_loss(hb_worker* w, int b, float* loss_out, cudaStream_t s) {
 extern "C" {
 
 const char* hb_last_error(void) { return hb::g_err.c_str(); }
+
+int64_t hb_kernel_launches(void) { return hb::g_launches.load(); }
+
+int hb_prof_enable(int32_t on) {
+  hb::g_prof_on.store(on != 0);
+  return HB_OK;
+}
+
+int hb_prof_read(hb_prof_entry* out, int32_t n, int32_t reset) {
+  HB_CHECK_ARG(out || n == 0, "null out");
+  HB_CUDA_TRY(cudaDeviceSynchronize());
+  std::lock_guard<std::mutex> g(hb::g_prof_mu);
+  for (auto& r : hb::g_pend) {
+    float ms = 0.f;
+    if (cudaEventElapsedTime(&ms, r.e0, r.e1) == cudaSuccess) {
+      hb_prof_entry& a = hb::g_agg[r.cls];
+      a.launches += r.nl;
+      a.ms += ms;
+      a.flops += r.flops;
+      a.bytes += r.bytes;
+    }
+    hb::g_evpool.push_back(r.e0);
+    hb::g_evpool.push_back(r.e1);
+  }
+  hb::g_pend.clear();
+  for (int i = 0; i < n && i < HB_PROF_N; ++i) out[i] = hb::g_agg[i];
+  if (reset)
+    for (auto& a : hb::g_agg) a = hb_prof_entry{};
+  return HB_OK;
+}
 int hb_abi_version(void) { return HB_ABI_VERSION; }
 
 int hb_device_ok(int32_t device) {
@@ -556,7 +663,9 @@ int mlp_worker_create(hb_model* m, int32_t max_batch, int32_t replica, void* cud
   cudaStream_t s = static_cast<cudaStream_t>(cuda_stream);
   bool own = false;
   if (!s) {
-    HB_CUDA_TRY(cudaStreamCreateWithFlags(&s, cudaStreamNonBlocking));
+    // a blocking stream: ordered after work on the legacy default stream (e.g. the caller's
+    // torch copies of X/y), concurrent with the other workers' streams (Hogbatch, L170)
+    HB_CUDA_TRY(cudaStreamCreate(&s));
     own = true;
   }
   return alloc_worker(m, max_batch, s, own, out);

@@ -23,6 +23,16 @@ struct Layer {
 
 int choose_bn(int M, int N);
 
+// Brackets the kernel launches of one hot-path operation: counts launches and, when profiling
+// is enabled (hb_prof_enable), records CUDA events on the launch stream.
+struct Prof {
+  int cls;
+  cudaStream_t s;
+  cudaEvent_t e0 = nullptr;
+  Prof(int cls, cudaStream_t s);
+  void done(int nlaunch, double flops, double bytes);
+};
+
 }  // namespace hb
 
 struct hb_model {

@@ -52,6 +52,7 @@ def to_device(X, y, dtype="bf16", device="cuda:0"):
     tX = torch.from_numpy(Xp).to(device)
     tX = tX.to(torch.bfloat16) if dtype == "bf16" else tX
     ty = torch.from_numpy(np.asarray(y, np.int32)).to(device)
+    torch.cuda.synchronize()  # the library's streams do not order after torch's stream
     return tX, ty
 
 

@@ -89,9 +89,12 @@ def test_one_sgd_step_updates_model_in_place(prec):
     new, l_ref = mlp64.sgd_step(params, X.astype(np.float64), y, lr)
     got = split_flat(m.get_params(), dims)
     for l in range(3):
-        # compare the UPDATE (W_new - W_old) normwise; the params themselves agree far tighter
-        assert rel_err(got[l][0] - params[l][0], new[l][0] - params[l][0]) <= TOL[prec]
-        assert rel_err(got[l][1] - params[l][1], new[l][1] - params[l][1]) <= TOL[prec]
+        for j in (0, 1):
+            # the update lr*dW must match to the path's tolerance; the fp32 master adds at most
+            # one rounding of W_new (<= 2^-24 |W_new| per element)
+            err = np.linalg.norm(got[l][j] - new[l][j])
+            allowed = TOL[prec] * np.linalg.norm(new[l][j] - params[l][j]) + 2.0 ** -23 * np.linalg.norm(new[l][j])
+            assert err <= allowed, (l, j, err, allowed)
     assert abs(loss - l_ref) / l_ref <= TOL[prec]
 
 
