@@ -13,7 +13,8 @@
 
 namespace hb {
 
-enum { EPI_FWD_SIG = 0, EPI_FWD_LOGITS = 1, EPI_DGRAD_SIG = 2, EPI_WGRAD_SGD = 3, EPI_WGRAD_STORE = 4 };
+enum { EPI_FWD_SIG = 0, EPI_FWD_LOGITS = 1, EPI_DGRAD_SIG = 2, EPI_WGRAD_SGD = 3, EPI_WGRAD_STORE = 4,
+       EPI_HEAD_XENT = 5 };
 
 struct EpiArgs {
   int M, N;             // valid output extent (rows, cols of the GEMM result)
@@ -29,6 +30,18 @@ struct EpiArgs {
   int64_t ldw;
   float lr;
   int transposed;       // WGRAD: result element (m, n) belongs to W[n][m]
+  // bias gradient fused into the GEMMs (tensor-core path):
+  float* bpart_out;     // DGRAD / HEAD_XENT: column sums of the produced dZ per 128-row M tile
+  const float* bpart_in;// WGRAD: those partials for dZ_l; reduced in fixed order to db_l
+  int64_t ldp;          // row stride of the partial arrays (= n_out of the layer)
+  int n_mtiles;         // WGRAD: number of partial rows (ceil(b / 128))
+  float* bias_upd;      // WGRAD_SGD: b_l -= lr * db_l in place
+  float* bias_grad;     // WGRAD_STORE: db_l written out
+  // softmax cross-entropy head fused into the output-layer GEMM (C <= 16):
+  const int32_t* y;     // labels (dataset base when yoff != nullptr)
+  const int* yoff;      // device row offset of the batch (graph replay), nullable
+  float* row_loss;      // per-row cross-entropy
+  float inv_b;          // 1 / b (gradient of the batch MEAN loss)
 };
 
 template <typename T>

@@ -18,7 +18,7 @@ namespace hb {
 // ---------------------------------------------------------------------------------------
 template <typename TDZ>
 __global__ void softmax_xent_kernel(const float* __restrict__ logits, int64_t ldl,
-                                    const int32_t* __restrict__ y, int b, int C, TDZ* dZ,
+                                    const int32_t* __restrict__ y, const int* __restrict__ yoff, int b, int C, TDZ* dZ,
                                     int64_t ldz, float* __restrict__ row_loss, float inv_b) {
   const int warp = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
   const int lane = threadIdx.x & 31;
@@ -33,7 +33,7 @@ __global__ void softmax_xent_kernel(const float* __restrict__ logits, int64_t ld
 #pragma unroll
   for (int o = 16; o > 0; o >>= 1) s += __shfl_xor_sync(0xffffffffu, s, o);
   const float lse = m + logf(s);
-  const int yi = y[warp];
+  const int yi = y[(yoff ? *yoff : 0) + warp];
   if (lane == 0) row_loss[warp] = lse - z[yi];
   if (dZ) {
     TDZ* d = dZ + (int64_t)warp * ldz;

@@ -62,6 +62,8 @@ static cudaEvent_t ev_get() {
   return e;
 }
 
+bool prof_enabled() { return g_prof_on.load(); }
+
 Prof::Prof(int cls_, cudaStream_t s_) : cls(cls_), s(s_) {
   if (g_prof_on.load(std::memory_order_relaxed)) {
     e0 = ev_get();
@@ -125,8 +127,8 @@ static std::mutex g_attr_mu;
 static std::set<std::pair<const void*, int>> g_attr_done;
 
 template <int BN, bool A_MN, bool B_MN, int EPI>
-static int launch_tc(const CUtensorMap& ma, const CUtensorMap& mb, int M, int N, int K, const EpiArgs& ep,
-                     cudaStream_t s) {
+static int launch_tc(const CUtensorMap& ma, const CUtensorMap& mb, int M, int N, int K, const int* offA,
+                     const int* offB, const EpiArgs& ep, cudaStream_t s) {
   using Cfg = TcCfg<BN, B_MN>;
   auto kern = tc_gemm_kernel<BN, A_MN, B_MN, EPI>;
   int dev = 0;
@@ -140,20 +142,20 @@ static int launch_tc(const CUtensorMap& ma, const CUtensorMap& mb, int M, int N,
     }
   }
   dim3 grid((N + BN - 1) / BN, (M + TC_BM - 1) / TC_BM);
-  kern<<<grid, TC_THREADS, Cfg::SMEM_BYTES, s>>>(ma, mb, K, ep);
+  kern<<<grid, TC_THREADS, Cfg::SMEM_BYTES, s>>>(ma, mb, K, offA, offB, ep);
   HB_CUDA_TRY(cudaGetLastError());
   return HB_OK;
 }
 
 template <bool A_MN, bool B_MN, int EPI>
 static int launch_tc_bn(int bn, const CUtensorMap& ma, const CUtensorMap& mb, int M, int N, int K,
-                        const EpiArgs& ep, cudaStream_t s) {
+                        const int* offA, const int* offB, const EpiArgs& ep, cudaStream_t s) {
   switch (bn) {
-    case 16: return launch_tc<16, A_MN, B_MN, EPI>(ma, mb, M, N, K, ep, s);
-    case 32: return launch_tc<32, A_MN, B_MN, EPI>(ma, mb, M, N, K, ep, s);
-    case 64: return launch_tc<64, A_MN, B_MN, EPI>(ma, mb, M, N, K, ep, s);
-    case 128: return launch_tc<128, A_MN, B_MN, EPI>(ma, mb, M, N, K, ep, s);
-    default: return launch_tc<256, A_MN, B_MN, EPI>(ma, mb, M, N, K, ep, s);
+    case 16: return launch_tc<16, A_MN, B_MN, EPI>(ma, mb, M, N, K, offA, offB, ep, s);
+    case 32: return launch_tc<32, A_MN, B_MN, EPI>(ma, mb, M, N, K, offA, offB, ep, s);
+    case 64: return launch_tc<64, A_MN, B_MN, EPI>(ma, mb, M, N, K, offA, offB, ep, s);
+    case 128: return launch_tc<128, A_MN, B_MN, EPI>(ma, mb, M, N, K, offA, offB, ep, s);
+    default: return launch_tc<256, A_MN, B_MN, EPI>(ma, mb, M, N, K, offA, offB, ep, s);
   }
 }
 
@@ -167,24 +169,37 @@ int choose_bn(int M, int N) {
   return 128;
 }
 
-// tensor-core GEMM on bf16 operands.  A is [M x K] (K-major, row stride lda) or stored [K x M]
-// (MN-major); B is [N x K] (K-major) or stored [K x N] (MN-major).
-static int gemm_tc(int epi, bool a_mn, bool b_mn, int M, int N, int K, const void* A, int64_t lda,
-                   const void* B, int64_t ldb, const EpiArgs& ep, cudaStream_t s) {
-  const int bn = choose_bn(M, N);
+// One tcgen05 GEMM launch.  A is [M x K] (K-major) or stored [K x M] (MN-major); B is [N x K]
+// (K-major) or stored [K x N] (MN-major).  a_rows / b_rows = number of stored rows covered by
+// the tensor map (0: exactly the GEMM extent); offA / offB = device row offsets (nullable).
+struct TcOp {
+  const void* p;
+  int64_t ld;
+  int64_t rows;
+  const int* off;
+};
+
+static int gemm_tc(int epi, bool a_mn, bool b_mn, int M, int N, int K, TcOp A, TcOp B, const EpiArgs& ep,
+                   cudaStream_t s) {
+  const int bn = epi == EPI_HEAD_XENT ? 16 : choose_bn(M, N);
   CUtensorMap ma, mb;
-  int rc = a_mn ? make_map(&ma, A, M, K, lda * 2, 64, 64) : make_map(&ma, A, K, M, lda * 2, 64, TC_BM);
+  const int64_t ar = A.rows ? A.rows : (a_mn ? K : M);
+  const int64_t br = B.rows ? B.rows : (b_mn ? K : N);
+  int rc = a_mn ? make_map(&ma, A.p, M, ar, A.ld * 2, 64, 64) : make_map(&ma, A.p, K, ar, A.ld * 2, 64, TC_BM);
   if (rc) return rc;
-  rc = b_mn ? make_map(&mb, B, N, K, ldb * 2, 64, 64) : make_map(&mb, B, K, N, ldb * 2, 64, bn);
+  rc = b_mn ? make_map(&mb, B.p, N, br, B.ld * 2, 64, 64) : make_map(&mb, B.p, K, br, B.ld * 2, 64, bn);
   if (rc) return rc;
   if (!a_mn && !b_mn) {
-    if (epi == EPI_FWD_SIG) return launch_tc_bn<false, false, EPI_FWD_SIG>(bn, ma, mb, M, N, K, ep, s);
-    if (epi == EPI_FWD_LOGITS) return launch_tc_bn<false, false, EPI_FWD_LOGITS>(bn, ma, mb, M, N, K, ep, s);
+    if (epi == EPI_FWD_SIG) return launch_tc_bn<false, false, EPI_FWD_SIG>(bn, ma, mb, M, N, K, A.off, B.off, ep, s);
+    if (epi == EPI_FWD_LOGITS)
+      return launch_tc_bn<false, false, EPI_FWD_LOGITS>(bn, ma, mb, M, N, K, A.off, B.off, ep, s);
+    if (epi == EPI_HEAD_XENT) return launch_tc<16, false, false, EPI_HEAD_XENT>(ma, mb, M, N, K, A.off, B.off, ep, s);
   } else if (!a_mn && b_mn) {
-    if (epi == EPI_DGRAD_SIG) return launch_tc_bn<false, true, EPI_DGRAD_SIG>(bn, ma, mb, M, N, K, ep, s);
+    if (epi == EPI_DGRAD_SIG) return launch_tc_bn<false, true, EPI_DGRAD_SIG>(bn, ma, mb, M, N, K, A.off, B.off, ep, s);
   } else if (a_mn && b_mn) {
-    if (epi == EPI_WGRAD_SGD) return launch_tc_bn<true, true, EPI_WGRAD_SGD>(bn, ma, mb, M, N, K, ep, s);
-    if (epi == EPI_WGRAD_STORE) return launch_tc_bn<true, true, EPI_WGRAD_STORE>(bn, ma, mb, M, N, K, ep, s);
+    if (epi == EPI_WGRAD_SGD) return launch_tc_bn<true, true, EPI_WGRAD_SGD>(bn, ma, mb, M, N, K, A.off, B.off, ep, s);
+    if (epi == EPI_WGRAD_STORE)
+      return launch_tc_bn<true, true, EPI_WGRAD_STORE>(bn, ma, mb, M, N, K, A.off, B.off, ep, s);
   }
   return fail(HB_EUNSUPPORTED, "gemm_tc: unsupported epilogue/major combination");
 }
@@ -230,29 +245,35 @@ static double gemm_bytes(int epi, int M, int N, int K, double es, bool shadow) {
   switch (epi) {
     case EPI_FWD_SIG: return io + 2.0 * mn * es + 4.0 * N;
     case EPI_FWD_LOGITS: return io + 4.0 * mn + 4.0 * N;
+    case EPI_HEAD_XENT: return io + mn * es + 8.0 * M + 4.0 * N;
     case EPI_DGRAD_SIG: return io + 2.0 * mn * es;
     case EPI_WGRAD_SGD: return io + 8.0 * mn + (shadow ? 2.0 * mn : 0.0);
     default: return io + 4.0 * mn;
   }
 }
 
-static int gemm(const hb_model* m, int epi, bool a_mn, bool b_mn, int M, int N, int K, const void* A, int64_t lda,
-                int adt, const void* B, int64_t ldb, int bdt, const EpiArgs& ep, cudaStream_t s) {
+static int prof_class(int epi) {
+  return epi == EPI_FWD_SIG ? HB_PROF_FWD_GEMM
+         : (epi == EPI_FWD_LOGITS || epi == EPI_HEAD_XENT) ? HB_PROF_HEAD_GEMM
+         : epi == EPI_DGRAD_SIG ? HB_PROF_DGRAD_GEMM
+                                : HB_PROF_WGRAD_GEMM;
+}
+
+static int gemm_tc_p(int epi, bool a_mn, bool b_mn, int M, int N, int K, TcOp A, TcOp B, const EpiArgs& ep,
+                     cudaStream_t s) {
   if (M <= 0 || N <= 0 || K <= 0) return HB_OK;
-  const int cls = epi == EPI_FWD_SIG ? HB_PROF_FWD_GEMM
-                  : epi == EPI_FWD_LOGITS ? HB_PROF_HEAD_GEMM
-                  : epi == EPI_DGRAD_SIG ? HB_PROF_DGRAD_GEMM
-                                         : HB_PROF_WGRAD_GEMM;
-  Prof pr(cls, s);
-  int rc;
-  if (m->prec == HB_PREC_BF16) {
-    if (adt != HB_BF16 || bdt != HB_BF16) return fail(HB_EINVAL, "bf16 mode needs bf16 operands (X must be HB_BF16)");
-    rc = gemm_tc(epi, a_mn, b_mn, M, N, K, A, lda, B, ldb, ep, s);
-  } else {
-    rc = gemm_simt(epi, a_mn, b_mn, M, N, K, A, lda, adt, B, ldb, bdt, ep, s);
-  }
-  const double es = m->prec == HB_PREC_BF16 ? 2.0 : 4.0;
-  if (!rc) pr.done(1, 2.0 * M * N * (double)K, gemm_bytes(epi, M, N, K, es, ep.shadow != nullptr || ep.out1 != nullptr));
+  Prof pr(prof_class(epi), s);
+  int rc = gemm_tc(epi, a_mn, b_mn, M, N, K, A, B, ep, s);
+  if (!rc) pr.done(1, 2.0 * M * N * (double)K, gemm_bytes(epi, M, N, K, 2.0, true));
+  return rc;
+}
+
+static int gemm_simt_p(int epi, bool a_mn, bool b_mn, int M, int N, int K, const void* A, int64_t lda, int adt,
+                       const void* B, int64_t ldb, int bdt, const EpiArgs& ep, cudaStream_t s) {
+  if (M <= 0 || N <= 0 || K <= 0) return HB_OK;
+  Prof pr(prof_class(epi), s);
+  int rc = gemm_simt(epi, a_mn, b_mn, M, N, K, A, lda, adt, B, ldb, bdt, ep, s);
+  if (!rc) pr.done(1, 2.0 * M * N * (double)K, gemm_bytes(epi, M, N, K, 4.0, false));
   return rc;
 }
 
@@ -269,13 +290,19 @@ static void free_worker_buffers(hb_worker* w) {
   w->H.clear();
   w->S.clear();
   w->dZ.clear();
+  clear_graphs(w);
+  for (float* p : w->bpart) cudaFree(p);
+  w->bpart.clear();
+  cudaFree(w->d_off);
+  if (w->h_off) cudaFreeHost(w->h_off);
+  w->d_off = nullptr;
+  w->h_off = nullptr;
   cudaFree(w->logits);
   cudaFree(w->row_loss);
-  cudaFree(w->partial);
   cudaFree(w->dsum);
   cudaFree(w->grads);
   if (w->h_dsum) cudaFreeHost(w->h_dsum);
-  w->logits = w->row_loss = w->partial = w->grads = nullptr;
+  w->logits = w->row_loss = w->grads = nullptr;
   w->dsum = nullptr;
   w->h_dsum = nullptr;
 }
@@ -311,10 +338,16 @@ static int alloc_worker(hb_model* m, int max_b, cudaStream_t stream, bool own, h
   }
   const int C = m->layers.back().n_out;
   w->ldc = (int)round_up(C, 4);
-  w->splits_max = (max_b + 127) / 128;
+  const int mt = (max_b + 127) / 128;
+  for (int l = 0; l < L; ++l) {
+    float* p = nullptr;
+    if (cudaMalloc(&p, (size_t)mt * m->layers[l].n_out * 4) != cudaSuccess)
+      return fail_free(fail(HB_ENOMEM, "bias partial alloc"));
+    w->bpart.push_back(p);
+  }
   if (cudaMalloc(&w->logits, (size_t)max_b * w->ldc * 4) != cudaSuccess ||
       cudaMalloc(&w->row_loss, (size_t)max_b * 4) != cudaSuccess ||
-      cudaMalloc(&w->partial, (size_t)w->splits_max * max_w * 4) != cudaSuccess ||
+      cudaMalloc(&w->d_off, sizeof(int)) != cudaSuccess || cudaMallocHost(&w->h_off, sizeof(int)) != cudaSuccess ||
       cudaMalloc(&w->dsum, 64 * sizeof(double)) != cudaSuccess ||
       cudaMallocHost(&w->h_dsum, 64 * sizeof(double)) != cudaSuccess)
     return fail_free(fail(HB_ENOMEM, "worker scratch alloc"));
@@ -331,14 +364,12 @@ using namespace hb;
 // ----------------------------------------------------------------------------------------
 namespace hb {
 
-int run_step(hb_worker* w, const void* X, int64_t ldx, int32_t xdt, const int32_t* y, int b, float lr,
-             bool grads_only, cudaStream_t s) {
+// fp32 check mode: SIMT GEMMs, fp32 activations, standalone softmax / bias kernels.
+static int run_step_simt(hb_worker* w, const void* X, int64_t ldx, int32_t xdt, const int32_t* y, int b, float lr,
+                         bool grads_only, cudaStream_t s) {
   hb_model* m = w->m;
   const int L = (int)m->layers.size();
-  const int adt = act_dt(m);
-  const bool bf = m->prec == HB_PREC_BF16;
   int rc;
-  // ---- forward, Eq. (1) ----
   const void* Ain = X;
   int64_t lda = ldx;
   int ain_dt = xdt;
@@ -360,42 +391,29 @@ int run_step(hb_worker* w, const void* X, int64_t ldx, int32_t xdt, const int32_
       ep.out0 = w->logits;
       ep.ld0 = w->ldc;
     }
-    const void* Wp = bf ? (const void*)(m->shadow + Ly.w_off) : (const void*)(m->master + Ly.w_off);
-    rc = gemm(m, epi, false, false, b, Ly.n_out, Ly.n_in, Ain, lda, ain_dt, Wp, Ly.ldw, bf ? HB_BF16 : HB_F32, ep, s);
+    rc = gemm_simt_p(epi, false, false, b, Ly.n_out, Ly.n_in, Ain, lda, ain_dt, m->master + Ly.w_off, Ly.ldw, HB_F32,
+                     ep, s);
     if (rc) return rc;
-    if (l < L - 1) {
-      Ain = w->H[l];
-      lda = Ly.ldo;
-      ain_dt = adt;
-    }
+    Ain = w->H[l];
+    lda = Ly.ldo;
+    ain_dt = HB_F32;
   }
-  // ---- softmax cross-entropy head: loss rows + dZ_L = (softmax - onehot)/b ----
   {
     const Layer& Ly = m->layers[L - 1];
-    const int threads = 256;
-    const int blocks = (b * 32 + threads - 1) / threads;
     Prof pr(HB_PROF_SOFTMAX, s);
-    if (bf)
-      softmax_xent_kernel<__nv_bfloat16><<<blocks, threads, 0, s>>>(
-          w->logits, w->ldc, y, b, Ly.n_out, static_cast<__nv_bfloat16*>(w->dZ[L - 1]), Ly.ldo, w->row_loss,
-          1.0f / (float)b);
-    else
-      softmax_xent_kernel<float><<<blocks, threads, 0, s>>>(w->logits, w->ldc, y, b, Ly.n_out,
-                                                           static_cast<float*>(w->dZ[L - 1]), Ly.ldo,
-                                                           w->row_loss, 1.0f / (float)b);
+    softmax_xent_kernel<float><<<(b * 32 + 255) / 256, 256, 0, s>>>(
+        w->logits, w->ldc, y, nullptr, b, Ly.n_out, static_cast<float*>(w->dZ[L - 1]), Ly.ldo, w->row_loss,
+        1.0f / (float)b);
     HB_CUDA_TRY(cudaGetLastError());
-    const double es = bf ? 2.0 : 4.0;
-    pr.done(1, 0.0, (double)b * Ly.n_out * (4.0 + es) + 8.0 * b);
+    pr.done(1, 0.0, (double)b * Ly.n_out * 8.0 + 8.0 * b);
   }
-  // ---- backward, Eq. (2), with the update of Eq. (3) fused into the dW GEMM ----
   for (int l = L - 1; l >= 0; --l) {
     const Layer& Ly = m->layers[l];
     const void* dZl = w->dZ[l];
     const void* Al = l == 0 ? X : w->H[l - 1];
     const int64_t ldal = l == 0 ? ldx : m->layers[l - 1].ldo;
-    const int al_dt = l == 0 ? xdt : adt;
-    const void* Wp = bf ? (const void*)(m->shadow + Ly.w_off) : (const void*)(m->master + Ly.w_off);
-    if (l > 0) {  // dZ_{l-1} = (dZ_l W_l) * sigma'(Z_{l-1}); reads W_l before it is updated below
+    const int al_dt = l == 0 ? xdt : HB_F32;
+    if (l > 0) {
       const Layer& Lp = m->layers[l - 1];
       EpiArgs ep{};
       ep.M = b;
@@ -404,48 +422,213 @@ int run_step(hb_worker* w, const void* X, int64_t ldx, int32_t xdt, const int32_
       ep.ld0 = Lp.ldo;
       ep.aux = w->S[l - 1];
       ep.ldaux = Lp.ldo;
-      rc = gemm(m, EPI_DGRAD_SIG, false, true, b, Ly.n_in, Ly.n_out, dZl, Ly.ldo, adt, Wp, Ly.ldw,
-                bf ? HB_BF16 : HB_F32, ep, s);
+      rc = gemm_simt_p(EPI_DGRAD_SIG, false, true, b, Ly.n_in, Ly.n_out, dZl, Ly.ldo, HB_F32, m->master + Ly.w_off,
+                       Ly.ldw, HB_F32, ep, s);
       if (rc) return rc;
     }
-    {  // W_l -= lr * dZ_l^T A_{l-1}
+    {
       EpiArgs ep{};
       const int epi = grads_only ? EPI_WGRAD_STORE : EPI_WGRAD_SGD;
       ep.master = m->master + Ly.w_off;
-      ep.shadow = bf ? m->shadow + Ly.w_off : nullptr;
       ep.ldw = Ly.ldw;
       ep.lr = lr;
       if (grads_only) ep.out0 = w->grads + Ly.w_off;
-      const bool tr = Ly.n_out < 128 && Ly.n_out < Ly.n_in;  // small head: M = n_in instead of n_out
+      const bool tr = Ly.n_out < 128 && Ly.n_out < Ly.n_in;
       ep.transposed = tr ? 1 : 0;
       if (!tr) {
         ep.M = Ly.n_out;
         ep.N = Ly.n_in;
-        rc = gemm(m, epi, true, true, Ly.n_out, Ly.n_in, b, dZl, Ly.ldo, adt, Al, ldal, al_dt, ep, s);
+        rc = gemm_simt_p(epi, true, true, Ly.n_out, Ly.n_in, b, dZl, Ly.ldo, HB_F32, Al, ldal, al_dt, ep, s);
       } else {
         ep.M = Ly.n_in;
         ep.N = Ly.n_out;
-        rc = gemm(m, epi, true, true, Ly.n_in, Ly.n_out, b, Al, ldal, al_dt, dZl, Ly.ldo, adt, ep, s);
+        rc = gemm_simt_p(epi, true, true, Ly.n_in, Ly.n_out, b, Al, ldal, al_dt, dZl, Ly.ldo, HB_F32, ep, s);
       }
       if (rc) return rc;
     }
-    {  // b_l -= lr * 1^T dZ_l (deterministic two-pass column sum)
+    {
       const int splits = (b + 127) / 128;
       Prof pr(HB_PROF_BIAS, s);
-      dim3 g1((Ly.n_out + 63) / 64, splits), b1(64, 4);
-      if (bf)
-        colsum_partial_kernel<__nv_bfloat16><<<g1, b1, 0, s>>>(static_cast<const __nv_bfloat16*>(dZl), Ly.ldo, b,
-                                                              Ly.n_out, 128, w->partial);
-      else
-        colsum_partial_kernel<float><<<g1, b1, 0, s>>>(static_cast<const float*>(dZl), Ly.ldo, b, Ly.n_out, 128,
-                                                       w->partial);
-      bias_apply_kernel<<<(Ly.n_out + 255) / 256, 256, 0, s>>>(w->partial, splits, Ly.n_out, lr,
+      colsum_partial_kernel<float><<<dim3((Ly.n_out + 63) / 64, splits), dim3(64, 4), 0, s>>>(
+          static_cast<const float*>(dZl), Ly.ldo, b, Ly.n_out, 128, w->bpart[l]);
+      bias_apply_kernel<<<(Ly.n_out + 255) / 256, 256, 0, s>>>(w->bpart[l], splits, Ly.n_out, lr,
                                                                m->master + Ly.b_off,
                                                                grads_only ? w->grads + Ly.b_off : nullptr);
       HB_CUDA_TRY(cudaGetLastError());
-      pr.done(2, (double)b * Ly.n_out, (double)b * Ly.n_out * (bf ? 2.0 : 4.0) + 8.0 * Ly.n_out);
+      pr.done(2, (double)b * Ly.n_out, (double)b * Ly.n_out * 4.0 + 8.0 * Ly.n_out);
     }
   }
+  return HB_OK;
+}
+
+// Forward chain (Eq. (1)) of the bf16 tensor-core path.  X holds x_rows rows; the batch starts
+// at row *d_off (graph replay) or at row 0 (d_off == nullptr).  With want_grad the head writes
+// dZ_L and its bias partials; otherwise only the per-row losses (mlp_loss).
+static int forward_tc(hb_worker* w, const void* X, int64_t ldx, int64_t x_rows, const int32_t* y, const int* d_off,
+                      int b, bool want_grad, cudaStream_t s) {
+  hb_model* m = w->m;
+  const int L = (int)m->layers.size();
+  int rc;
+  TcOp A{X, ldx, x_rows, d_off};
+  for (int l = 0; l < L; ++l) {
+    const Layer& Ly = m->layers[l];
+    TcOp B{m->shadow + Ly.w_off, Ly.ldw, 0, nullptr};
+    EpiArgs ep{};
+    ep.M = b;
+    ep.N = Ly.n_out;
+    ep.bias = m->master + Ly.b_off;
+    if (l < L - 1) {
+      ep.out0 = w->H[l];
+      ep.ld0 = Ly.ldo;
+      ep.out1 = want_grad ? w->S[l] : nullptr;
+      ep.ld1 = Ly.ldo;
+      rc = gemm_tc_p(EPI_FWD_SIG, false, false, b, Ly.n_out, Ly.n_in, A, B, ep, s);
+      if (rc) return rc;
+      A = TcOp{w->H[l], Ly.ldo, b, nullptr};
+      continue;
+    }
+    // output layer + softmax cross-entropy: dZ_L = (softmax(z) - onehot(y)) / b, per-row loss
+    if (Ly.n_out <= 16) {
+      ep.out0 = want_grad ? w->dZ[l] : nullptr;
+      ep.ld0 = Ly.ldo;
+      ep.y = y;
+      ep.yoff = d_off;
+      ep.row_loss = w->row_loss;
+      ep.inv_b = 1.0f / (float)b;
+      ep.bpart_out = want_grad ? w->bpart[l] : nullptr;
+      ep.ldp = Ly.n_out;
+      rc = gemm_tc_p(EPI_HEAD_XENT, false, false, b, Ly.n_out, Ly.n_in, A, B, ep, s);
+      if (rc) return rc;
+    } else {
+      ep.out0 = w->logits;
+      ep.ld0 = w->ldc;
+      rc = gemm_tc_p(EPI_FWD_LOGITS, false, false, b, Ly.n_out, Ly.n_in, A, B, ep, s);
+      if (rc) return rc;
+      Prof pr(HB_PROF_SOFTMAX, s);
+      softmax_xent_kernel<__nv_bfloat16><<<(b * 32 + 255) / 256, 256, 0, s>>>(
+          w->logits, w->ldc, y, d_off, b, Ly.n_out, want_grad ? static_cast<__nv_bfloat16*>(w->dZ[l]) : nullptr,
+          Ly.ldo, w->row_loss, 1.0f / (float)b);
+      int nl = 1;
+      if (want_grad) {
+        colsum_partial_kernel<__nv_bfloat16><<<dim3((Ly.n_out + 63) / 64, (b + 127) / 128), dim3(64, 4), 0, s>>>(
+            static_cast<const __nv_bfloat16*>(w->dZ[l]), Ly.ldo, b, Ly.n_out, 128, w->bpart[l]);
+        nl = 2;
+      }
+      HB_CUDA_TRY(cudaGetLastError());
+      pr.done(nl, 0.0, (double)b * Ly.n_out * 8.0 + 8.0 * b);
+    }
+  }
+  return HB_OK;
+}
+
+// One SGD step of the bf16 tensor-core path: forward + fused head, then for l = L..1
+// dgrad (reads W_l before it is updated) and wgrad with the fused in-place SGD of W_l and b_l.
+// 3L - 1 kernel launches for C <= 16 (L fwd incl. head, L-1 dgrad, L wgrad).
+static int run_step_tc(hb_worker* w, const void* X, int64_t ldx, int64_t x_rows, const int32_t* y, const int* d_off,
+                       int b, float lr, bool grads_only, cudaStream_t s) {
+  hb_model* m = w->m;
+  const int L = (int)m->layers.size();
+  int rc = forward_tc(w, X, ldx, x_rows, y, d_off, b, true, s);
+  if (rc) return rc;
+  const int mt = (b + TC_BM - 1) / TC_BM;
+  for (int l = L - 1; l >= 0; --l) {
+    const Layer& Ly = m->layers[l];
+    TcOp dZl{w->dZ[l], Ly.ldo, b, nullptr};
+    TcOp Al = l == 0 ? TcOp{X, ldx, x_rows, d_off} : TcOp{w->H[l - 1], m->layers[l - 1].ldo, b, nullptr};
+    TcOp Wl{m->shadow + Ly.w_off, Ly.ldw, 0, nullptr};
+    if (l > 0) {  // dZ_{l-1} = (dZ_l W_l) * sigma'(Z_{l-1}) and its bias partials
+      const Layer& Lp = m->layers[l - 1];
+      EpiArgs ep{};
+      ep.M = b;
+      ep.N = Ly.n_in;
+      ep.out0 = w->dZ[l - 1];
+      ep.ld0 = Lp.ldo;
+      ep.aux = w->S[l - 1];
+      ep.ldaux = Lp.ldo;
+      ep.bpart_out = w->bpart[l - 1];
+      ep.ldp = Lp.n_out;
+      rc = gemm_tc_p(EPI_DGRAD_SIG, false, true, b, Ly.n_in, Ly.n_out, dZl, Wl, ep, s);
+      if (rc) return rc;
+    }
+    // W_l -= lr * dZ_l^T A_{l-1};  b_l -= lr * 1^T dZ_l  (from the partials)
+    EpiArgs ep{};
+    const int epi = grads_only ? EPI_WGRAD_STORE : EPI_WGRAD_SGD;
+    ep.master = m->master + Ly.w_off;
+    ep.shadow = m->shadow + Ly.w_off;
+    ep.ldw = Ly.ldw;
+    ep.lr = lr;
+    if (grads_only) ep.out0 = w->grads + Ly.w_off;
+    ep.bpart_in = w->bpart[l];
+    ep.ldp = Ly.n_out;
+    ep.n_mtiles = mt;
+    ep.bias_upd = m->master + Ly.b_off;
+    ep.bias_grad = grads_only ? w->grads + Ly.b_off : nullptr;
+    const bool tr = Ly.n_out < 128 && Ly.n_out < Ly.n_in;  // small head: M = n_in instead of n_out
+    ep.transposed = tr ? 1 : 0;
+    if (!tr) {
+      ep.M = Ly.n_out;
+      ep.N = Ly.n_in;
+      rc = gemm_tc_p(epi, true, true, Ly.n_out, Ly.n_in, b, dZl, Al, ep, s);
+    } else {
+      ep.M = Ly.n_in;
+      ep.N = Ly.n_out;
+      rc = gemm_tc_p(epi, true, true, Ly.n_in, Ly.n_out, b, Al, dZl, ep, s);
+    }
+    if (rc) return rc;
+  }
+  return HB_OK;
+}
+
+int run_step(hb_worker* w, const void* X, int64_t ldx, int32_t xdt, int64_t x_rows, const int32_t* y,
+             const int* d_off, int b, float lr, bool grads_only, cudaStream_t s) {
+  if (w->m->prec == HB_PREC_BF16) return run_step_tc(w, X, ldx, x_rows, y, d_off, b, lr, grads_only, s);
+  if (d_off) return fail(HB_EUNSUPPORTED, "device row offsets are a tensor-core-path feature");
+  return run_step_simt(w, X, ldx, xdt, y, b, lr, grads_only, s);
+}
+
+void clear_graphs(hb_worker* w) {
+  for (auto& kv : w->graphs)
+    if (kv.second.exec) cudaGraphExecDestroy(kv.second.exec);
+  w->graphs.clear();
+}
+
+int step_graph(hb_worker* w, const void* X, int64_t ldx, int64_t x_rows, const int32_t* y, int64_t off, int b,
+               float lr) {
+  if (w->g_X != X || w->g_y != y || w->g_ldx != ldx || w->g_rows != x_rows) {
+    clear_graphs(w);
+    w->g_X = X;
+    w->g_y = y;
+    w->g_ldx = ldx;
+    w->g_rows = x_rows;
+  }
+  uint32_t lrbits;
+  std::memcpy(&lrbits, &lr, 4);
+  auto key = std::make_pair(b, lrbits);
+  auto it = w->graphs.find(key);
+  if (it == w->graphs.end()) {
+    cudaStream_t s = w->stream;
+    const int64_t l0 = g_launches.load();
+    HB_CUDA_TRY(cudaStreamBeginCapture(s, cudaStreamCaptureModeThreadLocal));
+    cudaMemcpyAsync(w->d_off, w->h_off, sizeof(int), cudaMemcpyHostToDevice, s);
+    int rc = run_step(w, X, ldx, HB_BF16, x_rows, y, w->d_off, b, lr, false, s);
+    cudaGraph_t graph = nullptr;
+    cudaError_t ce = cudaStreamEndCapture(s, &graph);
+    if (rc) {
+      if (graph) cudaGraphDestroy(graph);
+      return rc;
+    }
+    if (ce != cudaSuccess) return fail(HB_ECUDA, std::string("graph capture: ") + cudaGetErrorString(ce));
+    hb_worker::Graph gr;
+    ce = cudaGraphInstantiate(&gr.exec, graph, 0);
+    cudaGraphDestroy(graph);
+    if (ce != cudaSuccess) return fail(HB_ECUDA, std::string("graph instantiate: ") + cudaGetErrorString(ce));
+    gr.launches = (int)(g_launches.load() - l0);
+    g_launches.fetch_sub(gr.launches);  // counted when replayed
+    it = w->graphs.emplace(key, gr).first;
+  }
+  *w->h_off = (int)off;  // the previous replay of this worker has completed (caller synchronises)
+  HB_CUDA_TRY(cudaGraphLaunch(it->second.exec, w->stream));
+  g_launches.fetch_add(it->second.launches);
   return HB_OK;
 }
 
@@ -688,7 +871,7 @@ int mlp_step(hb_worker* w, const void* X, int64_t ldx, int32_t x_dtype, const in
   int rc = check_step_args(w, X, ldx, x_dtype, y, batch);
   if (rc) return rc;
   HB_CUDA_TRY(cudaSetDevice(w->m->device));
-  rc = run_step(w, X, ldx, x_dtype, y, batch, lr, false, w->stream);
+  rc = run_step(w, X, ldx, x_dtype, batch, y, nullptr, batch, lr, false, w->stream);
   if (rc) return rc;
   if (loss_out) return finish_loss(w, batch, loss_out, w->stream);
   return HB_OK;
@@ -705,7 +888,7 @@ int mlp_step_grads(hb_worker* w, const void* X, int64_t ldx, int32_t x_dtype, co
   HB_CUDA_TRY(cudaSetDevice(m->device));
   if (!w->grads) HB_CUDA_TRY(cudaMalloc(&w->grads, m->total * 4));
   HB_CUDA_TRY(cudaMemsetAsync(w->grads, 0, m->total * 4, w->stream));
-  rc = run_step(w, X, ldx, x_dtype, y, batch, 0.f, true, w->stream);
+  rc = run_step(w, X, ldx, x_dtype, batch, y, nullptr, batch, 0.f, true, w->stream);
   if (rc) return rc;
   std::vector<float> h(m->total);
   HB_CUDA_TRY(cudaMemcpyAsync(h.data(), w->grads, m->total * 4, cudaMemcpyDeviceToHost, w->stream));
@@ -749,38 +932,42 @@ int mlp_loss(hb_model* m, const void* X, int64_t ldx, int32_t x_dtype, const int
   for (int64_t c = 0; c < nchunks; ++c) {
     const int64_t r0 = c * chunk;
     const int b = (int)std::min<int64_t>(chunk, n - r0);
-    const void* Ain = static_cast<const char*>(X) + r0 * ldx * xes;
-    int64_t lda = ldx;
-    int adt = x_dtype;
-    for (int l = 0; l < L; ++l) {
-      const Layer& Ly = m->layers[l];
-      EpiArgs ep{};
-      ep.M = b;
-      ep.N = Ly.n_out;
-      ep.bias = m->master + Ly.b_off;
-      int epi;
-      if (l < L - 1) {
-        epi = EPI_FWD_SIG;
-        ep.out0 = w->H[l];
-        ep.ld0 = Ly.ldo;
-      } else {
-        epi = EPI_FWD_LOGITS;
-        ep.out0 = w->logits;
-        ep.ld0 = w->ldc;
-      }
-      const void* Wp = bf ? (const void*)(m->shadow + Ly.w_off) : (const void*)(m->master + Ly.w_off);
-      rc = gemm(m, epi, false, false, b, Ly.n_out, Ly.n_in, Ain, lda, adt, Wp, Ly.ldw, bf ? HB_BF16 : HB_F32, ep, s);
+    const void* Xc = static_cast<const char*>(X) + r0 * ldx * xes;
+    if (bf) {
+      rc = forward_tc(w, Xc, ldx, b, y + r0, nullptr, b, false, s);
       if (rc) return rc;
-      if (l < L - 1) {
+    } else {
+      const void* Ain = Xc;
+      int64_t lda = ldx;
+      int adt = x_dtype;
+      for (int l = 0; l < L; ++l) {
+        const Layer& Ly = m->layers[l];
+        EpiArgs ep{};
+        ep.M = b;
+        ep.N = Ly.n_out;
+        ep.bias = m->master + Ly.b_off;
+        int epi = EPI_FWD_SIG;
+        if (l < L - 1) {
+          ep.out0 = w->H[l];
+          ep.ld0 = Ly.ldo;
+        } else {
+          epi = EPI_FWD_LOGITS;
+          ep.out0 = w->logits;
+          ep.ld0 = w->ldc;
+        }
+        rc = gemm_simt_p(epi, false, false, b, Ly.n_out, Ly.n_in, Ain, lda, adt, m->master + Ly.w_off, Ly.ldw,
+                         HB_F32, ep, s);
+        if (rc) return rc;
         Ain = w->H[l];
         lda = Ly.ldo;
-        adt = act_dt(m);
+        adt = HB_F32;
       }
+      softmax_xent_kernel<float><<<(b * 32 + 255) / 256, 256, 0, s>>>(
+          w->logits, w->ldc, y + r0, nullptr, b, m->layers.back().n_out, (float*)nullptr, 0, w->row_loss, 1.0f);
+      g_launches.fetch_add(1, std::memory_order_relaxed);
     }
-    const int blocks = (b * 32 + 255) / 256;
-    softmax_xent_kernel<float><<<blocks, 256, 0, s>>>(w->logits, w->ldc, y + r0, b, m->layers.back().n_out,
-                                                     (float*)nullptr, 0, w->row_loss, 1.0f);
     sum_rows_kernel<<<1, 1024, 0, s>>>(w->row_loss, b, m->chunk_sums, (int)c);
+    g_launches.fetch_add(1, std::memory_order_relaxed);
     HB_CUDA_TRY(cudaGetLastError());
   }
   std::vector<double> h(nchunks);

@@ -4,6 +4,7 @@
 #include <cuda_bf16.h>
 #include <cuda_runtime.h>
 
+#include <map>
 #include <mutex>
 #include <vector>
 
@@ -61,16 +62,34 @@ struct hb_worker {
   float* logits = nullptr;      // [max_b x ldc] fp32
   int ldc = 0;
   float* row_loss = nullptr;    // [max_b]
-  float* partial = nullptr;     // [splits x max width] bias-gradient partial sums
-  int splits_max = 0;
+  std::vector<float*> bpart;    // per layer [ceil(max_b/128) x n_out] bias-gradient partial sums
+  int* d_off = nullptr;         // device row offset of the current batch (graph replay)
+  int* h_off = nullptr;         // pinned host source of d_off
+  // CUDA graphs of one SGD step, per (batch size, lr), for the dataset they were captured on
+  struct Graph {
+    cudaGraphExec_t exec = nullptr;
+    int launches = 0;
+  };
+  std::map<std::pair<int, uint32_t>, Graph> graphs;
+  const void* g_X = nullptr;
+  const void* g_y = nullptr;
+  int64_t g_ldx = 0, g_rows = 0;
   double* dsum = nullptr;
   double* h_dsum = nullptr;     // pinned
   float* grads = nullptr;       // mlp_step_grads output (flat padded layout)
 };
 
 namespace hb {
-int run_step(hb_worker* w, const void* X, int64_t ldx, int32_t xdt, const int32_t* y, int b, float lr,
-             bool grads_only, cudaStream_t s);
+// One SGD step.  X / y: the batch's first row, or (d_off != nullptr, tensor-core path) the
+// dataset base with the batch's first row read from *d_off on the device.  x_rows = rows of X.
+int run_step(hb_worker* w, const void* X, int64_t ldx, int32_t xdt, int64_t x_rows, const int32_t* y,
+             const int* d_off, int b, float lr, bool grads_only, cudaStream_t s);
+// One SGD step replayed from a CUDA graph captured for (b, lr) on the dataset (X, y): the
+// batch's row offset is copied from pinned host memory by the graph's first node.
+int step_graph(hb_worker* w, const void* X, int64_t ldx, int64_t x_rows, const int32_t* y, int64_t off, int b,
+               float lr);
+void clear_graphs(hb_worker* w);
+bool prof_enabled();
 int finish_loss(hb_worker* w, int b, float* loss_out, cudaStream_t s);
 // enqueue sum of the last step's per-row losses into *dst (device double)
 void sum_rows_into(hb_worker* w, int b, double* dst, cudaStream_t s);

@@ -5,15 +5,21 @@
 //
 // The three contractions of one SGD step (Eq. (1)/(2), L43/L49) map onto it as
 //   forward  H_l  = sigma(H_{l-1} W_l^T + b_l)   A = H_{l-1} (K-major), B = W_l (K-major)
+//   head     dZ_L = softmax(H W_L^T + b_L) - Y    (fused cross-entropy epilogue, C <= 16)
 //   dgrad    dZ   = (dZ_l W_l) * S               A = dZ_l   (K-major), B = W_l (MN-major)
 //   wgrad    W_l -= lr * dZ_l^T H_{l-1}          A = dZ_l   (MN-major), B = H_{l-1} (MN-major)
 // so the same kernel serves all of them; the operand major-ness is a template parameter and is
 // handled entirely by the TMA box shape and the UMMA shared-memory descriptor, never by a copy.
+// The bias gradient db_l = 1^T dZ_l is fused as well: the epilogue that PRODUCES dZ (dgrad /
+// head) writes per-128-row column sums, and the wgrad epilogue reduces them in fixed order and
+// applies b_l -= lr * db_l — no separate reduction kernel, deterministic.
 //
 // CTA = 256 threads: warp 0 TMA producer, warp 1 MMA issuer (one elected thread), warp 2 TMEM
 // allocator, warps 4..7 epilogue (warp w reads TMEM lanes 32*(w%4)..+31 = tile rows).
 // Tile: BLOCK_M = 128 (UMMA M = 128, cta_group::1), BLOCK_N = BN (16..256), BLOCK_K = 64 (one
 // 128-byte swizzle atom of bf16).  smem stages form an mbarrier ring (full/empty).
+// offA / offB (nullable, device) add a row offset to the stored-row coordinate of A / B: the
+// batch's first row inside the HBM-resident dataset, written once per step (graph replay).
 #pragma once
 
 #include "common.cuh"
@@ -31,16 +37,51 @@ struct TcCfg {
   static constexpr int B_ROWS = B_MN ? (BN < 64 ? 64 : BN) : BN;        // MN-major loads 64-wide boxes
   static constexpr int B_BYTES = B_ROWS * TC_BK * 2;
   static constexpr int STAGE_BYTES = A_BYTES + B_BYTES;
-  static constexpr int STAGES_RAW = (196 * 1024) / STAGE_BYTES;
+  static constexpr int STAGES_RAW = (192 * 1024) / STAGE_BYTES;
   static constexpr int STAGES = STAGES_RAW > 8 ? 8 : STAGES_RAW;
   static constexpr int TMEM_COLS = BN <= 32 ? 32 : BN;                  // power of two >= 32
-  static constexpr int SMEM_BYTES = STAGES * STAGE_BYTES + 1024 /*align*/ + 256 /*barriers*/;
+  static constexpr int RED_BYTES = 4 * BN * 4;                          // per-warp column sums
+  static constexpr int SMEM_BYTES = STAGES * STAGE_BYTES + 1024 /*align*/ + 256 /*barriers*/ + RED_BYTES;
 };
+
+__device__ __forceinline__ void epi_bar_sync() { asm volatile("bar.sync 1, 128;" ::: "memory"); }
+
+// Column sums of a 32-row x 16-column register tile (one row per lane) in 16 shuffles
+// (reduce-scatter): afterwards lane L holds the total of column
+// 8*b4(L) + 4*b3(L) + 2*b2(L) + b1(L), where bk(L) is bit k of L (pairs L, L^1 agree).
+__device__ __forceinline__ float warp_colsum16(const float (&v)[16], int lane) {
+  float a[8], b[4], c[2];
+  bool up = lane & 16;
+#pragma unroll
+  for (int j = 0; j < 8; ++j) {
+    float send = up ? v[j] : v[j + 8], keep = up ? v[j + 8] : v[j];
+    a[j] = keep + __shfl_xor_sync(0xffffffffu, send, 16);
+  }
+  up = lane & 8;
+#pragma unroll
+  for (int j = 0; j < 4; ++j) {
+    float send = up ? a[j] : a[j + 4], keep = up ? a[j + 4] : a[j];
+    b[j] = keep + __shfl_xor_sync(0xffffffffu, send, 8);
+  }
+  up = lane & 4;
+#pragma unroll
+  for (int j = 0; j < 2; ++j) {
+    float send = up ? b[j] : b[j + 2], keep = up ? b[j + 2] : b[j];
+    c[j] = keep + __shfl_xor_sync(0xffffffffu, send, 4);
+  }
+  up = lane & 2;
+  float d = (up ? c[1] : c[0]) + __shfl_xor_sync(0xffffffffu, up ? c[0] : c[1], 2);
+  return d + __shfl_xor_sync(0xffffffffu, d, 1);
+}
+
+__device__ __forceinline__ int colsum16_col(int lane) {
+  return ((lane >> 4) & 1) * 8 + ((lane >> 3) & 1) * 4 + ((lane >> 2) & 1) * 2 + ((lane >> 1) & 1);
+}
 
 template <int BN, bool A_MN, bool B_MN, int EPI>
 __global__ void __launch_bounds__(TC_THREADS, 1)
     tc_gemm_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUtensorMap tmB,
-                   int K, EpiArgs ep) {
+                   int K, const int* __restrict__ offA, const int* __restrict__ offB, EpiArgs ep) {
   using Cfg = TcCfg<BN, B_MN>;
   constexpr int STAGES = Cfg::STAGES;
   extern __shared__ uint8_t smem_raw[];
@@ -49,6 +90,7 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
   uint64_t* empty_bar = full_bar + STAGES;
   uint64_t* tmem_full_bar = empty_bar + STAGES;
   uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(tmem_full_bar + 1);
+  float* red = reinterpret_cast<float*>(smem + STAGES * Cfg::STAGE_BYTES + 256);  // [4][BN]
 
   const int warp = threadIdx.x >> 5;
   const int lane = threadIdx.x & 31;
@@ -74,6 +116,8 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
 
   if (warp == 0 && lane == 0) {
     // ===== TMA producer =====
+    const int oa = offA ? __ldg(offA) : 0;
+    const int ob = offB ? __ldg(offB) : 0;
     for (int kb = 0; kb < num_kb; ++kb) {
       const int s = kb % STAGES;
       const uint32_t ph = (kb / STAGES) & 1;
@@ -83,16 +127,17 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
       mbar_arrive_expect_tx(&full_bar[s], Cfg::STAGE_BYTES);
       const int k0 = kb * TC_BK;
       if (!A_MN) {
-        tma_load_2d(sA, &tmA, &full_bar[s], k0, m0);
+        tma_load_2d(sA, &tmA, &full_bar[s], k0, m0 + oa);
       } else {
-        tma_load_2d(sA, &tmA, &full_bar[s], m0, k0);
-        tma_load_2d(sA + 8192, &tmA, &full_bar[s], m0 + 64, k0);
+        tma_load_2d(sA, &tmA, &full_bar[s], m0, k0 + oa);
+        tma_load_2d(sA + 8192, &tmA, &full_bar[s], m0 + 64, k0 + oa);
       }
       if (!B_MN) {
-        tma_load_2d(sB, &tmB, &full_bar[s], k0, n0);
+        tma_load_2d(sB, &tmB, &full_bar[s], k0, n0 + ob);
       } else {
 #pragma unroll
-        for (int j = 0; j < Cfg::B_ROWS / 64; ++j) tma_load_2d(sB + j * 8192, &tmB, &full_bar[s], n0 + 64 * j, k0);
+        for (int j = 0; j < Cfg::B_ROWS / 64; ++j)
+          tma_load_2d(sB + j * 8192, &tmB, &full_bar[s], n0 + 64 * j, k0 + ob);
       }
     }
   } else if (warp == 1 && lane == 0) {
@@ -124,28 +169,144 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
     mbar_wait(tmem_full_bar, 0);
     tc_fence_after();
     const int q = warp & 3;
-    const int r = m0 + q * 32 + lane;
+    const int rl = q * 32 + lane;  // row within the tile
+    const int r = m0 + rl;
     const bool row_ok = r < ep.M;
-#pragma unroll 1
-    for (int c = 0; c < BN; c += 16) {
-      if (n0 + c >= ep.N) break;  // warp-uniform
+    const uint32_t tbase = tmem_base + ((uint32_t)(q * 32) << 16);
+
+    if (EPI == EPI_HEAD_XENT) {
+      // ---- softmax cross-entropy on the thread's own row of logits (N = C <= BN = 16) ----
       uint32_t raw[16];
-      tmem_ld_32x32b_x16(tmem_base + ((uint32_t)(q * 32) << 16) + (uint32_t)c, raw);
+      tmem_ld_32x32b_x16(tbase, raw);
       tmem_ld_wait();
-      float v[16];
+      const int C = ep.N;
+      float z[16], dz[16];
+      float mx = -INFINITY;
 #pragma unroll
-      for (int j = 0; j < 16; ++j) v[j] = __uint_as_float(raw[j]);
+      for (int j = 0; j < 16; ++j) {
+        z[j] = j < C ? __uint_as_float(raw[j]) + ep.bias[j] : -INFINITY;
+        mx = fmaxf(mx, z[j]);
+      }
+      float se = 0.f;
+#pragma unroll
+      for (int j = 0; j < 16; ++j) se += j < C ? expf(z[j] - mx) : 0.f;
+      const float lse = mx + logf(se);
+      const int yo = ep.yoff ? __ldg(ep.yoff) : 0;
+      const int yi = row_ok ? __ldg(ep.y + yo + r) : -1;
+#pragma unroll
+      for (int j = 0; j < 16; ++j)
+        dz[j] = (row_ok && j < C) ? (expf(z[j] - lse) - (j == yi ? 1.f : 0.f)) * ep.inv_b : 0.f;
       if (row_ok) {
+        float zy = 0.f;
+#pragma unroll
+        for (int j = 0; j < 16; ++j) zy = j == yi ? z[j] : zy;
+        ep.row_loss[r] = lse - zy;
+        if (ep.out0) {
+          uint4* D = reinterpret_cast<uint4*>(static_cast<__nv_bfloat16*>(ep.out0) + (int64_t)r * ep.ld0);
+          D[0] = make_uint4(pack_bf16x2(dz[0], dz[1]), pack_bf16x2(dz[2], dz[3]), pack_bf16x2(dz[4], dz[5]),
+                            pack_bf16x2(dz[6], dz[7]));
+          if (ep.ld0 >= 16)
+            D[1] = make_uint4(pack_bf16x2(dz[8], dz[9]), pack_bf16x2(dz[10], dz[11]),
+                              pack_bf16x2(dz[12], dz[13]), pack_bf16x2(dz[14], dz[15]));
+        }
+      }
+      if (ep.bpart_out) {
+        const float t = warp_colsum16(dz, lane);
+        if (!(lane & 1)) red[q * BN + colsum16_col(lane)] = t;
+        epi_bar_sync();
+        if (rl < C)
+          ep.bpart_out[(int64_t)blockIdx.y * ep.ldp + rl] = (red[rl] + red[BN + rl]) + (red[2 * BN + rl] + red[3 * BN + rl]);
+      }
+    } else {
+#pragma unroll 1
+      for (int c = 0; c < BN; c += 16) {
+        if (n0 + c >= ep.N) break;  // warp-uniform
+        uint32_t raw[16];
+        tmem_ld_32x32b_x16(tbase + (uint32_t)c, raw);
+        tmem_ld_wait();
+        float v[16];
+#pragma unroll
+        for (int j = 0; j < 16; ++j) v[j] = __uint_as_float(raw[j]);
         const int nc = n0 + c;
-        const bool vec_ok = (nc + 16 <= ep.N) && !((EPI == EPI_WGRAD_SGD || EPI == EPI_WGRAD_STORE) && ep.transposed) &&
-                            (EPI != EPI_WGRAD_SGD || ep.shadow != nullptr) && EPI != EPI_FWD_LOGITS &&
-                            EPI != EPI_WGRAD_STORE;
-        if (vec_ok) {
-          epi_row16_bf16<EPI>(ep, r, nc, v);
-        } else {
+        const bool full = nc + 16 <= ep.N;
+        if (EPI == EPI_DGRAD_SIG) {
+          // dZ = acc * sigma'(Z) (stashed S), stored bf16; fp32 values feed the bias partials
+          if (row_ok) {
+            if (full) {
+              const uint4* S = reinterpret_cast<const uint4*>(static_cast<const __nv_bfloat16*>(ep.aux) +
+                                                              (int64_t)r * ep.ldaux + nc);
+              uint4 s0 = S[0], s1 = S[1];
+              const __nv_bfloat162* sv0 = reinterpret_cast<const __nv_bfloat162*>(&s0);
+              const __nv_bfloat162* sv1 = reinterpret_cast<const __nv_bfloat162*>(&s1);
+#pragma unroll
+              for (int qq = 0; qq < 4; ++qq) {
+                float2 a = __bfloat1622float2(sv0[qq]);
+                v[2 * qq] *= a.x;
+                v[2 * qq + 1] *= a.y;
+                float2 cc = __bfloat1622float2(sv1[qq]);
+                v[8 + 2 * qq] *= cc.x;
+                v[8 + 2 * qq + 1] *= cc.y;
+              }
+              uint4* D = reinterpret_cast<uint4*>(static_cast<__nv_bfloat16*>(ep.out0) + (int64_t)r * ep.ld0 + nc);
+              D[0] = make_uint4(pack_bf16x2(v[0], v[1]), pack_bf16x2(v[2], v[3]), pack_bf16x2(v[4], v[5]),
+                                pack_bf16x2(v[6], v[7]));
+              D[1] = make_uint4(pack_bf16x2(v[8], v[9]), pack_bf16x2(v[10], v[11]), pack_bf16x2(v[12], v[13]),
+                                pack_bf16x2(v[14], v[15]));
+            } else {
+              const __nv_bfloat16* S = static_cast<const __nv_bfloat16*>(ep.aux) + (int64_t)r * ep.ldaux;
+              __nv_bfloat16* D = static_cast<__nv_bfloat16*>(ep.out0) + (int64_t)r * ep.ld0;
+#pragma unroll
+              for (int j = 0; j < 16; ++j) {
+                if (nc + j < ep.N) {
+                  v[j] *= __bfloat162float(S[nc + j]);
+                  D[nc + j] = __float2bfloat16_rn(v[j]);
+                } else {
+                  v[j] = 0.f;
+                }
+              }
+            }
+          } else {
+#pragma unroll
+            for (int j = 0; j < 16; ++j) v[j] = 0.f;
+          }
+          if (ep.bpart_out) {
+            const float t = warp_colsum16(v, lane);
+            if (!(lane & 1)) red[q * BN + c + colsum16_col(lane)] = t;
+          }
+        } else if (row_ok) {
+          const bool vec_ok = full && !((EPI == EPI_WGRAD_SGD || EPI == EPI_WGRAD_STORE) && ep.transposed) &&
+                              (EPI != EPI_WGRAD_SGD || ep.shadow != nullptr) && EPI != EPI_FWD_LOGITS &&
+                              EPI != EPI_WGRAD_STORE;
+          if (vec_ok) {
+            epi_row16_bf16<EPI>(ep, r, nc, v);
+          } else {
 #pragma unroll 4
-          for (int j = 0; j < 16; ++j)
-            if (nc + j < ep.N) epi_elem<EPI, __nv_bfloat16, false>(ep, r, nc + j, v[j]);
+            for (int j = 0; j < 16; ++j)
+              if (nc + j < ep.N) epi_elem<EPI, __nv_bfloat16, false>(ep, r, nc + j, v[j]);
+          }
+        }
+      }
+      if (EPI == EPI_DGRAD_SIG && ep.bpart_out) {
+        epi_bar_sync();
+        if (rl < BN && n0 + rl < ep.N)
+          ep.bpart_out[(int64_t)blockIdx.y * ep.ldp + n0 + rl] =
+              (red[rl] + red[BN + rl]) + (red[2 * BN + rl] + red[3 * BN + rl]);
+      }
+      if ((EPI == EPI_WGRAD_SGD || EPI == EPI_WGRAD_STORE) && ep.bpart_in) {
+        // db = sum of the dZ producer's per-tile partials, fixed order; bias index = W row
+        int bi = -1;
+        if (!ep.transposed) {
+          if (blockIdx.x == 0 && row_ok) bi = r;
+        } else if (blockIdx.y == 0 && rl < BN && n0 + rl < ep.N) {
+          bi = n0 + rl;
+        }
+        if (bi >= 0) {
+          float sdb = 0.f;
+          for (int t = 0; t < ep.n_mtiles; ++t) sdb += ep.bpart_in[(int64_t)t * ep.ldp + bi];
+          if (EPI == EPI_WGRAD_SGD)
+            ep.bias_upd[bi] -= ep.lr * sdb;
+          else
+            ep.bias_grad[bi] = sdb;
         }
       }
     }
