@@ -281,9 +281,6 @@ def main():
     torch.cuda.synchronize()
     if world > 1:
         dist.barrier()
-    if not args.no_prof:
-        hb.prof_read(reset=True)
-        hb.prof_enable(True)
     clocks = ClockSampler(local)
     clocks.start()
     l0 = hb.kernel_launches()
@@ -304,8 +301,6 @@ def main():
         share += st["updates"][0]
     launches = hb.kernel_launches() - l0
     clk = clocks.stop()
-    prof = hb.prof_read(reset=True) if not args.no_prof else None
-    hb.prof_enable(False)
     tot_ms = sum(ms)
     t = torch.tensor([tot_ms], device=f"cuda:{local}")
     s = torch.tensor([float(samples)], device=f"cuda:{local}")
@@ -340,6 +335,20 @@ def main():
         dist.all_reduce(te, op=dist.ReduceOp.MAX)
         dist.all_reduce(se, op=dist.ReduceOp.SUM)
     e2e_value = se.item() / (te.item() * 1e-3) if args.e2e_steps else None
+
+    # ---- per-kernel roofline: the same steps re-run with every hot-path launch bracketed by
+    #      CUDA events on its own stream (hb_prof_enable; graphs off so each launch is visible).
+    #      Kept out of the timed region above: the event records cost host time per launch.
+    prof = None
+    if not args.no_prof:
+        model.set_params(params0)
+        hb.prof_read(reset=True)
+        hb.prof_enable(True)
+        for _ in range(max(1, min(args.steps, 3))):
+            flush.zero_()
+            run_epoch()
+        prof = hb.prof_read(reset=True)
+        hb.prof_enable(False)
 
     if rank == 0:
         peaks = load_peaks()

@@ -66,7 +66,8 @@ int hb_merge_begin(hb_model* m) {
   if (!m->base) HB_CUDA_TRY(cudaMalloc(&m->base, m->total * 4));
   if (!m->delta) HB_CUDA_TRY(cudaMalloc(&m->delta, m->total * 4));
   HB_CUDA_TRY(cudaDeviceSynchronize());
-  HB_CUDA_TRY(cudaMemcpy(m->base, m->master, m->total * 4, cudaMemcpyDeviceToDevice));
+  HB_CUDA_TRY(cudaMemcpyAsync(m->base, m->master, m->total * 4, cudaMemcpyDeviceToDevice, m->stream));
+  HB_CUDA_TRY(cudaStreamSynchronize(m->stream));
   return HB_OK;
 }
 

@@ -743,7 +743,8 @@ int mlp_create(const int32_t* dims, int32_t n_dims, int32_t activation, int32_t 
     delete m;
     return fail(HB_ENOMEM, "model alloc");
   }
-  if (cudaStreamCreateWithFlags(&m->stream, cudaStreamNonBlocking) != cudaSuccess) {
+  // blocking stream: ordered after the caller's legacy-stream work (e.g. torch copies)
+  if (cudaStreamCreate(&m->stream) != cudaSuccess) {
     cudaFree(m->master);
     cudaFree(m->shadow);
     delete m;
@@ -759,12 +760,14 @@ int mlp_create(const int32_t* dims, int32_t n_dims, int32_t activation, int32_t 
       for (int j = 0; j < Ly.n_in; ++j) h[Ly.w_off + (size_t)i * Ly.ldw + j] = (float)(nd(gen) * sd);
   }
   int rc = [&]() -> int {
-    HB_CUDA_TRY(cudaMemcpy(m->master, h.data(), m->total * 4, cudaMemcpyHostToDevice));
+    // copy and shadow refresh on the same stream: a pageable cudaMemcpy may return before its
+    // DMA lands, so the refresh must be stream-ordered after it
+    HB_CUDA_TRY(cudaMemcpyAsync(m->master, h.data(), m->total * 4, cudaMemcpyHostToDevice, m->stream));
     if (m->shadow) {
       refresh_shadow_kernel<<<256, 256, 0, m->stream>>>(m->master, m->shadow, (int64_t)m->total);
       HB_CUDA_TRY(cudaGetLastError());
-      HB_CUDA_TRY(cudaStreamSynchronize(m->stream));
     }
+    HB_CUDA_TRY(cudaStreamSynchronize(m->stream));
     return HB_OK;
   }();
   if (rc) {
@@ -804,7 +807,9 @@ int mlp_get_params(const hb_model* m, float* host_dst, int64_t n) {
   HB_CHECK_ARG(host_dst && n == need, "n must equal mlp_num_params");
   HB_CUDA_TRY(cudaSetDevice(m->device));
   std::vector<float> h(m->total);
-  HB_CUDA_TRY(cudaMemcpy(h.data(), m->master, m->total * 4, cudaMemcpyDeviceToHost));
+  HB_CUDA_TRY(cudaDeviceSynchronize());  // every worker's in-place updates are visible
+  HB_CUDA_TRY(cudaMemcpyAsync(h.data(), m->master, m->total * 4, cudaMemcpyDeviceToHost, m->stream));
+  HB_CUDA_TRY(cudaStreamSynchronize(m->stream));
   int64_t o = 0;
   for (const Layer& Ly : m->layers) {
     for (int i = 0; i < Ly.n_out; ++i)
@@ -828,7 +833,7 @@ int mlp_set_params(hb_model* m, const float* host_src, int64_t n) {
     for (int i = 0; i < Ly.n_out; ++i) h[Ly.b_off + i] = host_src[o++];
   }
   HB_CUDA_TRY(cudaDeviceSynchronize());
-  HB_CUDA_TRY(cudaMemcpy(m->master, h.data(), m->total * 4, cudaMemcpyHostToDevice));
+  HB_CUDA_TRY(cudaMemcpyAsync(m->master, h.data(), m->total * 4, cudaMemcpyHostToDevice, m->stream));
   if (m->shadow) {
     refresh_shadow_kernel<<<256, 256, 0, m->stream>>>(m->master, m->shadow, (int64_t)m->total);
     HB_CUDA_TRY(cudaGetLastError());

@@ -288,26 +288,26 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
       }
       if (EPI == EPI_DGRAD_SIG && ep.bpart_out) {
         epi_bar_sync();
-        if (rl < BN && n0 + rl < ep.N)
-          ep.bpart_out[(int64_t)blockIdx.y * ep.ldp + n0 + rl] =
-              (red[rl] + red[BN + rl]) + (red[2 * BN + rl] + red[3 * BN + rl]);
+        for (int cc = rl; cc < BN && n0 + cc < ep.N; cc += 128)
+          ep.bpart_out[(int64_t)blockIdx.y * ep.ldp + n0 + cc] =
+              (red[cc] + red[BN + cc]) + (red[2 * BN + cc] + red[3 * BN + cc]);
       }
       if ((EPI == EPI_WGRAD_SGD || EPI == EPI_WGRAD_STORE) && ep.bpart_in) {
         // db = sum of the dZ producer's per-tile partials, fixed order; bias index = W row
-        int bi = -1;
-        if (!ep.transposed) {
-          if (blockIdx.x == 0 && row_ok) bi = r;
-        } else if (blockIdx.y == 0 && rl < BN && n0 + rl < ep.N) {
-          bi = n0 + rl;
-        }
-        if (bi >= 0) {
-          float sdb = 0.f;
-          for (int t = 0; t < ep.n_mtiles; ++t) sdb += ep.bpart_in[(int64_t)t * ep.ldp + bi];
-          if (EPI == EPI_WGRAD_SGD)
-            ep.bias_upd[bi] -= ep.lr * sdb;
-          else
-            ep.bias_grad[bi] = sdb;
-        }
+        // non-transposed: the n-tile-0 CTA owns bias rows m0..m0+127 (one per thread);
+        // transposed (small head): the m-tile-0 CTA owns bias entries n0..n0+BN-1
+        const bool own = !ep.transposed ? (blockIdx.x == 0) : (blockIdx.y == 0);
+        const int lo = !ep.transposed ? r : n0 + rl;
+        const int hi = !ep.transposed ? min(ep.M, m0 + TC_BM) : min(ep.N, n0 + BN);
+        if (own)
+          for (int bi = lo; bi < hi; bi += 128) {
+            float sdb = 0.f;
+            for (int t = 0; t < ep.n_mtiles; ++t) sdb += ep.bpart_in[(int64_t)t * ep.ldp + bi];
+            if (EPI == EPI_WGRAD_SGD)
+              ep.bias_upd[bi] -= ep.lr * sdb;
+            else
+              ep.bias_grad[bi] = sdb;
+          }
       }
     }
   }

