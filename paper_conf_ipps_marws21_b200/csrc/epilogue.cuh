@@ -37,6 +37,7 @@ struct EpiArgs {
   int n_mtiles;         // WGRAD: number of partial rows (ceil(b / 128))
   float* bias_upd;      // WGRAD_SGD: b_l -= lr * db_l in place
   float* bias_grad;     // WGRAD_STORE: db_l written out
+  float* ws;            // WGRAD split-K: fp32 partial tiles [tiles][splits][128][BN]
   // softmax cross-entropy head fused into the output-layer GEMM (C <= 16):
   const int32_t* y;     // labels (dataset base when yoff != nullptr)
   const int* yoff;      // device row offset of the batch (graph replay), nullable

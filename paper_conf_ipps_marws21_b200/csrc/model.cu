@@ -128,7 +128,7 @@ static std::set<std::pair<const void*, int>> g_attr_done;
 
 template <int BN, bool A_MN, bool B_MN, int EPI>
 static int launch_tc(const CUtensorMap& ma, const CUtensorMap& mb, int M, int N, int K, const int* offA,
-                     const int* offB, const EpiArgs& ep, cudaStream_t s) {
+                     const int* offB, const EpiArgs& ep, cudaStream_t s, int splits = 1) {
   using Cfg = TcCfg<BN, B_MN>;
   auto kern = tc_gemm_kernel<BN, A_MN, B_MN, EPI>;
   int dev = 0;
@@ -141,22 +141,48 @@ static int launch_tc(const CUtensorMap& ma, const CUtensorMap& mb, int M, int N,
       g_attr_done.insert(key);
     }
   }
-  dim3 grid((N + BN - 1) / BN, (M + TC_BM - 1) / TC_BM);
-  kern<<<grid, TC_THREADS, Cfg::SMEM_BYTES, s>>>(ma, mb, K, offA, offB, ep);
+  dim3 grid((N + BN - 1) / BN, (M + TC_BM - 1) / TC_BM, splits);
+  if (splits == 1) {
+    kern<<<grid, TC_THREADS, Cfg::SMEM_BYTES, s>>>(ma, mb, K, offA, offB, ep);
+  } else {  // split-K: the `splits` CTAs of a tile form one thread-block cluster along z
+    cudaLaunchConfig_t cfg{};
+    cfg.gridDim = grid;
+    cfg.blockDim = dim3(TC_THREADS);
+    cfg.dynamicSmemBytes = Cfg::SMEM_BYTES;
+    cfg.stream = s;
+    cudaLaunchAttribute attr[1];
+    attr[0].id = cudaLaunchAttributeClusterDimension;
+    attr[0].val.clusterDim.x = 1;
+    attr[0].val.clusterDim.y = 1;
+    attr[0].val.clusterDim.z = splits;
+    cfg.attrs = attr;
+    cfg.numAttrs = 1;
+    HB_CUDA_TRY(cudaLaunchKernelEx(&cfg, kern, ma, mb, K, offA, offB, ep));
+  }
   HB_CUDA_TRY(cudaGetLastError());
   return HB_OK;
 }
 
 template <bool A_MN, bool B_MN, int EPI>
 static int launch_tc_bn(int bn, const CUtensorMap& ma, const CUtensorMap& mb, int M, int N, int K,
-                        const int* offA, const int* offB, const EpiArgs& ep, cudaStream_t s) {
+                        const int* offA, const int* offB, const EpiArgs& ep, cudaStream_t s, int splits = 1) {
   switch (bn) {
-    case 16: return launch_tc<16, A_MN, B_MN, EPI>(ma, mb, M, N, K, offA, offB, ep, s);
-    case 32: return launch_tc<32, A_MN, B_MN, EPI>(ma, mb, M, N, K, offA, offB, ep, s);
-    case 64: return launch_tc<64, A_MN, B_MN, EPI>(ma, mb, M, N, K, offA, offB, ep, s);
-    case 128: return launch_tc<128, A_MN, B_MN, EPI>(ma, mb, M, N, K, offA, offB, ep, s);
-    default: return launch_tc<256, A_MN, B_MN, EPI>(ma, mb, M, N, K, offA, offB, ep, s);
+    case 16: return launch_tc<16, A_MN, B_MN, EPI>(ma, mb, M, N, K, offA, offB, ep, s, splits);
+    case 32: return launch_tc<32, A_MN, B_MN, EPI>(ma, mb, M, N, K, offA, offB, ep, s, splits);
+    case 64: return launch_tc<64, A_MN, B_MN, EPI>(ma, mb, M, N, K, offA, offB, ep, s, splits);
+    case 128: return launch_tc<128, A_MN, B_MN, EPI>(ma, mb, M, N, K, offA, offB, ep, s, splits);
+    default: return launch_tc<256, A_MN, B_MN, EPI>(ma, mb, M, N, K, offA, offB, ep, s, splits);
   }
+}
+
+// split-K factor of a dW GEMM (K = batch): enough CTAs to cover the 148 SMs, power of two
+// <= 8 (portable cluster size), at least one k-block per split
+int choose_splits(int M, int N, int K, int bn) {
+  const long tiles = (long)((M + TC_BM - 1) / TC_BM) * ((N + bn - 1) / bn);
+  const int nkb = (K + TC_BK - 1) / TC_BK;
+  int S = 1;
+  while (S * 2 <= 8 && tiles * S * 2 <= 148 && S * 2 <= nkb) S *= 2;
+  return S;
 }
 
 int choose_bn(int M, int N) {
@@ -197,9 +223,11 @@ static int gemm_tc(int epi, bool a_mn, bool b_mn, int M, int N, int K, TcOp A, T
   } else if (!a_mn && b_mn) {
     if (epi == EPI_DGRAD_SIG) return launch_tc_bn<false, true, EPI_DGRAD_SIG>(bn, ma, mb, M, N, K, A.off, B.off, ep, s);
   } else if (a_mn && b_mn) {
-    if (epi == EPI_WGRAD_SGD) return launch_tc_bn<true, true, EPI_WGRAD_SGD>(bn, ma, mb, M, N, K, A.off, B.off, ep, s);
+    const int S = ep.ws ? choose_splits(M, N, K, bn) : 1;
+    if (epi == EPI_WGRAD_SGD)
+      return launch_tc_bn<true, true, EPI_WGRAD_SGD>(bn, ma, mb, M, N, K, A.off, B.off, ep, s, S);
     if (epi == EPI_WGRAD_STORE)
-      return launch_tc_bn<true, true, EPI_WGRAD_STORE>(bn, ma, mb, M, N, K, A.off, B.off, ep, s);
+      return launch_tc_bn<true, true, EPI_WGRAD_STORE>(bn, ma, mb, M, N, K, A.off, B.off, ep, s, S);
   }
   return fail(HB_EUNSUPPORTED, "gemm_tc: unsupported epilogue/major combination");
 }
@@ -297,6 +325,8 @@ static void free_worker_buffers(hb_worker* w) {
   if (w->h_off) cudaFreeHost(w->h_off);
   w->d_off = nullptr;
   w->h_off = nullptr;
+  cudaFree(w->ws);
+  w->ws = nullptr;
   cudaFree(w->logits);
   cudaFree(w->row_loss);
   cudaFree(w->dsum);
@@ -345,6 +375,8 @@ static int alloc_worker(hb_model* m, int max_b, cudaStream_t stream, bool own, h
       return fail_free(fail(HB_ENOMEM, "bias partial alloc"));
     w->bpart.push_back(p);
   }
+  if (m->prec == HB_PREC_BF16 && cudaMalloc(&w->ws, (size_t)148 * TC_BM * 256 * 4) != cudaSuccess)
+    return fail_free(fail(HB_ENOMEM, "split-K workspace alloc"));
   if (cudaMalloc(&w->logits, (size_t)max_b * w->ldc * 4) != cudaSuccess ||
       cudaMalloc(&w->row_loss, (size_t)max_b * 4) != cudaSuccess ||
       cudaMalloc(&w->d_off, sizeof(int)) != cudaSuccess || cudaMallocHost(&w->h_off, sizeof(int)) != cudaSuccess ||
@@ -563,6 +595,7 @@ static int run_step_tc(hb_worker* w, const void* X, int64_t ldx, int64_t x_rows,
     ep.n_mtiles = mt;
     ep.bias_upd = m->master + Ly.b_off;
     ep.bias_grad = grads_only ? w->grads + Ly.b_off : nullptr;
+    ep.ws = w->ws;
     const bool tr = Ly.n_out < 128 && Ly.n_out < Ly.n_in;  // small head: M = n_in instead of n_out
     ep.transposed = tr ? 1 : 0;
     if (!tr) {

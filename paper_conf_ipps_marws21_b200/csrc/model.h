@@ -77,6 +77,7 @@ struct hb_worker {
   double* dsum = nullptr;
   double* h_dsum = nullptr;     // pinned
   float* grads = nullptr;       // mlp_step_grads output (flat padded layout)
+  float* ws = nullptr;          // split-K partial tiles of the dW GEMMs (148 x 128 x 256 fp32)
 };
 
 namespace hb {

@@ -14,8 +14,10 @@
 // head) writes per-128-row column sums, and the wgrad epilogue reduces them in fixed order and
 // applies b_l -= lr * db_l — no separate reduction kernel, deterministic.
 //
-// CTA = 256 threads: warp 0 TMA producer, warp 1 MMA issuer (one elected thread), warp 2 TMEM
-// allocator, warps 4..7 epilogue (warp w reads TMEM lanes 32*(w%4)..+31 = tile rows).
+// CTA = 384 threads: warp 0 TMA producer, warp 1 MMA issuer (one elected thread), warp 2 TMEM
+// allocator, warps 4..11 epilogue (warp w reads TMEM lanes 32*(w%4)..+31 = tile rows, and one
+// half of the tile's columns); the epilogue warps stage the bias and prefetch the sigma' stash
+// while the mainloop runs.
 // Tile: BLOCK_M = 128 (UMMA M = 128, cta_group::1), BLOCK_N = BN (16..256), BLOCK_K = 64 (one
 // 128-byte swizzle atom of bf16).  smem stages form an mbarrier ring (full/empty).
 // offA / offB (nullable, device) add a row offset to the stored-row coordinate of A / B: the
@@ -29,7 +31,7 @@ namespace hb {
 
 constexpr int TC_BM = 128;
 constexpr int TC_BK = 64;
-constexpr int TC_THREADS = 256;
+constexpr int TC_THREADS = 384;  // 4 control warps + 8 epilogue warps
 
 template <int BN, bool B_MN>
 struct TcCfg {
@@ -40,11 +42,12 @@ struct TcCfg {
   static constexpr int STAGES_RAW = (192 * 1024) / STAGE_BYTES;
   static constexpr int STAGES = STAGES_RAW > 8 ? 8 : STAGES_RAW;
   static constexpr int TMEM_COLS = BN <= 32 ? 32 : BN;                  // power of two >= 32
-  static constexpr int RED_BYTES = 4 * BN * 4;                          // per-warp column sums
-  static constexpr int SMEM_BYTES = STAGES * STAGE_BYTES + 1024 /*align*/ + 256 /*barriers*/ + RED_BYTES;
+  static constexpr int RED_BYTES = 4 * BN * 4;                          // per-quadrant column sums
+  static constexpr int BIAS_BYTES = BN * 4;                             // staged bias of the tile
+  static constexpr int SMEM_BYTES = STAGES * STAGE_BYTES + 1024 /*align*/ + 256 /*barriers*/ + RED_BYTES + BIAS_BYTES;
 };
 
-__device__ __forceinline__ void epi_bar_sync() { asm volatile("bar.sync 1, 128;" ::: "memory"); }
+__device__ __forceinline__ void epi_bar_sync() { asm volatile("bar.sync 1, 256;" ::: "memory"); }
 
 // Column sums of a 32-row x 16-column register tile (one row per lane) in 16 shuffles
 // (reduce-scatter): afterwards lane L holds the total of column
@@ -91,12 +94,20 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
   uint64_t* tmem_full_bar = empty_bar + STAGES;
   uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(tmem_full_bar + 1);
   float* red = reinterpret_cast<float*>(smem + STAGES * Cfg::STAGE_BYTES + 256);  // [4][BN]
+  float* sbias = red + 4 * BN;                                                      // [BN]
 
   const int warp = threadIdx.x >> 5;
   const int lane = threadIdx.x & 31;
   const int n0 = blockIdx.x * BN;
   const int m0 = blockIdx.y * TC_BM;
-  const int num_kb = (K + TC_BK - 1) / TC_BK;
+  // split-K (dW GEMMs with K = batch): the gridDim.z CTAs of one output tile form a cluster,
+  // each accumulates k-blocks [kb_lo, kb_hi) in its own TMEM
+  const int splits = gridDim.z;
+  const int kz = blockIdx.z;
+  const int num_kb_all = (K + TC_BK - 1) / TC_BK;
+  const int kpb = (num_kb_all + splits - 1) / splits;
+  const int kb_lo = min(num_kb_all, kz * kpb);
+  const int num_kb = min(num_kb_all, kb_lo + kpb) - kb_lo;
 
   if (warp == 0 && lane == 0) {
     tma_prefetch_desc(&tmA);
@@ -125,7 +136,7 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
       uint8_t* sA = smem + s * Cfg::STAGE_BYTES;
       uint8_t* sB = sA + Cfg::A_BYTES;
       mbar_arrive_expect_tx(&full_bar[s], Cfg::STAGE_BYTES);
-      const int k0 = kb * TC_BK;
+      const int k0 = (kb_lo + kb) * TC_BK;
       if (!A_MN) {
         tma_load_2d(sA, &tmA, &full_bar[s], k0, m0 + oa);
       } else {
@@ -165,142 +176,289 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
     }
     umma_commit(tmem_full_bar);     // accumulator ready
   } else if (warp >= 4) {
-    // ===== epilogue: TMEM -> registers -> fused epilogue -> global =====
-    mbar_wait(tmem_full_bar, 0);
-    tc_fence_after();
+    // ===== epilogue (8 warps): TMEM -> registers -> fused epilogue -> global =====
+    // warp w reads TMEM lanes 32*(w%4).. (tile rows) and handles column half h = (w-4)/4
     const int q = warp & 3;
-    const int rl = q * 32 + lane;  // row within the tile
+    const int h = (warp - 4) >> 2;
+    const int et = threadIdx.x - 128;  // 0..255
+    const int rl = q * 32 + lane;      // row within the tile
     const int r = m0 + rl;
     const bool row_ok = r < ep.M;
     const uint32_t tbase = tmem_base + ((uint32_t)(q * 32) << 16);
+    constexpr int HALF = BN >= 32 ? BN / 2 : BN;  // columns per warp
+    const bool active = BN >= 32 || h == 0;
+    const int c_lo = BN >= 32 ? h * HALF : 0;
+
+    // stage the bias of the tile's columns in shared memory while the mainloop runs
+    if (EPI == EPI_FWD_SIG || EPI == EPI_FWD_LOGITS || EPI == EPI_HEAD_XENT) {
+      for (int c = et; c < BN; c += 256) sbias[c] = n0 + c < ep.N ? ep.bias[n0 + c] : 0.f;
+    }
+    // DGRAD: prefetch this thread's row of sigma'(Z) (the S stash) for all of its columns
+    constexpr int NCH = (HALF + 15) / 16;
+    uint4 spre[EPI == EPI_DGRAD_SIG ? NCH : 1][2];
+    if (EPI == EPI_DGRAD_SIG && active && row_ok) {
+#pragma unroll
+      for (int i = 0; i < NCH; ++i) {
+        const int nc = n0 + c_lo + 16 * i;
+        if (nc + 16 <= ep.N) {
+          const uint4* S = reinterpret_cast<const uint4*>(static_cast<const __nv_bfloat16*>(ep.aux) +
+                                                          (int64_t)r * ep.ldaux + nc);
+          spre[i][0] = __ldg(S);
+          spre[i][1] = __ldg(S + 1);
+        }
+      }
+    }
+    epi_bar_sync();  // sbias visible
+    mbar_wait(tmem_full_bar, 0);
+    tc_fence_after();
 
     if (EPI == EPI_HEAD_XENT) {
       // ---- softmax cross-entropy on the thread's own row of logits (N = C <= BN = 16) ----
-      uint32_t raw[16];
-      tmem_ld_32x32b_x16(tbase, raw);
-      tmem_ld_wait();
-      const int C = ep.N;
-      float z[16], dz[16];
-      float mx = -INFINITY;
+      float dz[16];
 #pragma unroll
-      for (int j = 0; j < 16; ++j) {
-        z[j] = j < C ? __uint_as_float(raw[j]) + ep.bias[j] : -INFINITY;
-        mx = fmaxf(mx, z[j]);
-      }
-      float se = 0.f;
+      for (int j = 0; j < 16; ++j) dz[j] = 0.f;
+      if (h == 0) {
+        uint32_t raw[16];
+        tmem_ld_32x32b_x16(tbase, raw);
+        tmem_ld_wait();
+        const int C = ep.N;
+        float z[16];
+        float mx = -INFINITY;
 #pragma unroll
-      for (int j = 0; j < 16; ++j) se += j < C ? expf(z[j] - mx) : 0.f;
-      const float lse = mx + logf(se);
-      const int yo = ep.yoff ? __ldg(ep.yoff) : 0;
-      const int yi = row_ok ? __ldg(ep.y + yo + r) : -1;
+        for (int j = 0; j < 16; ++j) {
+          z[j] = j < C ? __uint_as_float(raw[j]) + sbias[j] : -INFINITY;
+          mx = fmaxf(mx, z[j]);
+        }
+        float se = 0.f;
 #pragma unroll
-      for (int j = 0; j < 16; ++j)
-        dz[j] = (row_ok && j < C) ? (expf(z[j] - lse) - (j == yi ? 1.f : 0.f)) * ep.inv_b : 0.f;
-      if (row_ok) {
-        float zy = 0.f;
+        for (int j = 0; j < 16; ++j) se += j < C ? expf(z[j] - mx) : 0.f;
+        const float lse = mx + logf(se);
+        const int yo = ep.yoff ? __ldg(ep.yoff) : 0;
+        const int yi = row_ok ? __ldg(ep.y + yo + r) : -1;
 #pragma unroll
-        for (int j = 0; j < 16; ++j) zy = j == yi ? z[j] : zy;
-        ep.row_loss[r] = lse - zy;
-        if (ep.out0) {
-          uint4* D = reinterpret_cast<uint4*>(static_cast<__nv_bfloat16*>(ep.out0) + (int64_t)r * ep.ld0);
-          D[0] = make_uint4(pack_bf16x2(dz[0], dz[1]), pack_bf16x2(dz[2], dz[3]), pack_bf16x2(dz[4], dz[5]),
-                            pack_bf16x2(dz[6], dz[7]));
-          if (ep.ld0 >= 16)
-            D[1] = make_uint4(pack_bf16x2(dz[8], dz[9]), pack_bf16x2(dz[10], dz[11]),
-                              pack_bf16x2(dz[12], dz[13]), pack_bf16x2(dz[14], dz[15]));
+        for (int j = 0; j < 16; ++j)
+          dz[j] = (row_ok && j < C) ? (expf(z[j] - lse) - (j == yi ? 1.f : 0.f)) * ep.inv_b : 0.f;
+        if (row_ok) {
+          float zy = 0.f;
+#pragma unroll
+          for (int j = 0; j < 16; ++j) zy = j == yi ? z[j] : zy;
+          ep.row_loss[r] = lse - zy;
+          if (ep.out0) {
+            uint4* D = reinterpret_cast<uint4*>(static_cast<__nv_bfloat16*>(ep.out0) + (int64_t)r * ep.ld0);
+            D[0] = make_uint4(pack_bf16x2(dz[0], dz[1]), pack_bf16x2(dz[2], dz[3]), pack_bf16x2(dz[4], dz[5]),
+                              pack_bf16x2(dz[6], dz[7]));
+            if (ep.ld0 >= 16)
+              D[1] = make_uint4(pack_bf16x2(dz[8], dz[9]), pack_bf16x2(dz[10], dz[11]),
+                                pack_bf16x2(dz[12], dz[13]), pack_bf16x2(dz[14], dz[15]));
+          }
+        }
+        if (ep.bpart_out) {
+          const float t = warp_colsum16(dz, lane);
+          if (!(lane & 1)) red[q * BN + colsum16_col(lane)] = t;
         }
       }
       if (ep.bpart_out) {
-        const float t = warp_colsum16(dz, lane);
-        if (!(lane & 1)) red[q * BN + colsum16_col(lane)] = t;
         epi_bar_sync();
-        if (rl < C)
-          ep.bpart_out[(int64_t)blockIdx.y * ep.ldp + rl] = (red[rl] + red[BN + rl]) + (red[2 * BN + rl] + red[3 * BN + rl]);
+        if (et < ep.N)
+          ep.bpart_out[(int64_t)blockIdx.y * ep.ldp + et] = (red[et] + red[BN + et]) + (red[2 * BN + et] + red[3 * BN + et]);
       }
     } else {
+      if (active) {
 #pragma unroll 1
-      for (int c = 0; c < BN; c += 16) {
-        if (n0 + c >= ep.N) break;  // warp-uniform
-        uint32_t raw[16];
-        tmem_ld_32x32b_x16(tbase + (uint32_t)c, raw);
-        tmem_ld_wait();
-        float v[16];
+        for (int cc = 0; cc < HALF; cc += 16) {
+          const int c = c_lo + cc;
+          if (n0 + c >= ep.N) break;  // warp-uniform
+          uint32_t raw[16];
+          tmem_ld_32x32b_x16(tbase + (uint32_t)c, raw);
+          tmem_ld_wait();
+          float v[16];
 #pragma unroll
-        for (int j = 0; j < 16; ++j) v[j] = __uint_as_float(raw[j]);
-        const int nc = n0 + c;
-        const bool full = nc + 16 <= ep.N;
-        if (EPI == EPI_DGRAD_SIG) {
-          // dZ = acc * sigma'(Z) (stashed S), stored bf16; fp32 values feed the bias partials
-          if (row_ok) {
-            if (full) {
-              const uint4* S = reinterpret_cast<const uint4*>(static_cast<const __nv_bfloat16*>(ep.aux) +
-                                                              (int64_t)r * ep.ldaux + nc);
-              uint4 s0 = S[0], s1 = S[1];
-              const __nv_bfloat162* sv0 = reinterpret_cast<const __nv_bfloat162*>(&s0);
-              const __nv_bfloat162* sv1 = reinterpret_cast<const __nv_bfloat162*>(&s1);
+          for (int j = 0; j < 16; ++j) v[j] = __uint_as_float(raw[j]);
+          const int nc = n0 + c;
+          const bool full = nc + 16 <= ep.N;
+          if (EPI == EPI_DGRAD_SIG) {
+            // dZ = acc * sigma'(Z) (prefetched S), stored bf16; fp32 values feed the bias partials
+            if (row_ok) {
+              if (full) {
+                const uint4 s0 = spre[0][0], s1 = spre[0][1];
+                const __nv_bfloat162* sv0 = reinterpret_cast<const __nv_bfloat162*>(&s0);
+                const __nv_bfloat162* sv1 = reinterpret_cast<const __nv_bfloat162*>(&s1);
 #pragma unroll
-              for (int qq = 0; qq < 4; ++qq) {
-                float2 a = __bfloat1622float2(sv0[qq]);
-                v[2 * qq] *= a.x;
-                v[2 * qq + 1] *= a.y;
-                float2 cc = __bfloat1622float2(sv1[qq]);
-                v[8 + 2 * qq] *= cc.x;
-                v[8 + 2 * qq + 1] *= cc.y;
-              }
-              uint4* D = reinterpret_cast<uint4*>(static_cast<__nv_bfloat16*>(ep.out0) + (int64_t)r * ep.ld0 + nc);
-              D[0] = make_uint4(pack_bf16x2(v[0], v[1]), pack_bf16x2(v[2], v[3]), pack_bf16x2(v[4], v[5]),
-                                pack_bf16x2(v[6], v[7]));
-              D[1] = make_uint4(pack_bf16x2(v[8], v[9]), pack_bf16x2(v[10], v[11]), pack_bf16x2(v[12], v[13]),
-                                pack_bf16x2(v[14], v[15]));
-            } else {
-              const __nv_bfloat16* S = static_cast<const __nv_bfloat16*>(ep.aux) + (int64_t)r * ep.ldaux;
-              __nv_bfloat16* D = static_cast<__nv_bfloat16*>(ep.out0) + (int64_t)r * ep.ld0;
+                for (int qq = 0; qq < 4; ++qq) {
+                  float2 a = __bfloat1622float2(sv0[qq]);
+                  v[2 * qq] *= a.x;
+                  v[2 * qq + 1] *= a.y;
+                  float2 b2 = __bfloat1622float2(sv1[qq]);
+                  v[8 + 2 * qq] *= b2.x;
+                  v[8 + 2 * qq + 1] *= b2.y;
+                }
+                uint4* D = reinterpret_cast<uint4*>(static_cast<__nv_bfloat16*>(ep.out0) + (int64_t)r * ep.ld0 + nc);
+                D[0] = make_uint4(pack_bf16x2(v[0], v[1]), pack_bf16x2(v[2], v[3]), pack_bf16x2(v[4], v[5]),
+                                  pack_bf16x2(v[6], v[7]));
+                D[1] = make_uint4(pack_bf16x2(v[8], v[9]), pack_bf16x2(v[10], v[11]), pack_bf16x2(v[12], v[13]),
+                                  pack_bf16x2(v[14], v[15]));
+              } else {
+                const __nv_bfloat16* S = static_cast<const __nv_bfloat16*>(ep.aux) + (int64_t)r * ep.ldaux;
+                __nv_bfloat16* D = static_cast<__nv_bfloat16*>(ep.out0) + (int64_t)r * ep.ld0;
 #pragma unroll
-              for (int j = 0; j < 16; ++j) {
-                if (nc + j < ep.N) {
-                  v[j] *= __bfloat162float(S[nc + j]);
-                  D[nc + j] = __float2bfloat16_rn(v[j]);
-                } else {
-                  v[j] = 0.f;
+                for (int j = 0; j < 16; ++j) {
+                  if (nc + j < ep.N) {
+                    v[j] *= __bfloat162float(S[nc + j]);
+                    D[nc + j] = __float2bfloat16_rn(v[j]);
+                  } else {
+                    v[j] = 0.f;
+                  }
                 }
               }
-            }
-          } else {
+            } else {
 #pragma unroll
-            for (int j = 0; j < 16; ++j) v[j] = 0.f;
-          }
-          if (ep.bpart_out) {
-            const float t = warp_colsum16(v, lane);
-            if (!(lane & 1)) red[q * BN + c + colsum16_col(lane)] = t;
-          }
-        } else if (row_ok) {
-          const bool vec_ok = full && !((EPI == EPI_WGRAD_SGD || EPI == EPI_WGRAD_STORE) && ep.transposed) &&
-                              (EPI != EPI_WGRAD_SGD || ep.shadow != nullptr) && EPI != EPI_FWD_LOGITS &&
-                              EPI != EPI_WGRAD_STORE;
-          if (vec_ok) {
-            epi_row16_bf16<EPI>(ep, r, nc, v);
-          } else {
+              for (int j = 0; j < 16; ++j) v[j] = 0.f;
+            }
+            if (ep.bpart_out) {
+              const float t = warp_colsum16(v, lane);
+              if (!(lane & 1)) red[q * BN + c + colsum16_col(lane)] = t;
+            }
+            // advance the prefetched-S ring (static register indexing)
+#pragma unroll
+            for (int i = 0; i + 1 < NCH; ++i) {
+              spre[i][0] = spre[i + 1][0];
+              spre[i][1] = spre[i + 1][1];
+            }
+          } else if ((EPI == EPI_WGRAD_SGD || EPI == EPI_WGRAD_STORE) && splits > 1) {
+            // split-K: park the fp32 partial tile; reduced after the cluster barrier below
+            float4* wsp = reinterpret_cast<float4*>(
+                ep.ws + ((((size_t)blockIdx.y * gridDim.x + blockIdx.x) * splits + kz) * TC_BM + rl) * BN + c);
+            if (num_kb == 0) {
+#pragma unroll
+              for (int j = 0; j < 16; ++j) v[j] = 0.f;
+            }
+#pragma unroll
+            for (int qq = 0; qq < 4; ++qq) wsp[qq] = make_float4(v[4 * qq], v[4 * qq + 1], v[4 * qq + 2], v[4 * qq + 3]);
+          } else if (row_ok) {
+            if (EPI == EPI_FWD_SIG && full) {
+              uint32_t hp[8], sp[8];
+#pragma unroll
+              for (int qq = 0; qq < 8; ++qq) {
+                const float z0 = v[2 * qq] + sbias[c + 2 * qq], z1 = v[2 * qq + 1] + sbias[c + 2 * qq + 1];
+                const float h0 = sigmoidf_(z0), h1 = sigmoidf_(z1);
+                hp[qq] = pack_bf16x2(h0, h1);
+                sp[qq] = pack_bf16x2(h0 * (1.f - h0), h1 * (1.f - h1));
+              }
+              uint4* H = reinterpret_cast<uint4*>(static_cast<__nv_bfloat16*>(ep.out0) + (int64_t)r * ep.ld0 + nc);
+              H[0] = make_uint4(hp[0], hp[1], hp[2], hp[3]);
+              H[1] = make_uint4(hp[4], hp[5], hp[6], hp[7]);
+              if (ep.out1) {
+                uint4* S = reinterpret_cast<uint4*>(static_cast<__nv_bfloat16*>(ep.out1) + (int64_t)r * ep.ld1 + nc);
+                S[0] = make_uint4(sp[0], sp[1], sp[2], sp[3]);
+                S[1] = make_uint4(sp[4], sp[5], sp[6], sp[7]);
+              }
+            } else if (EPI == EPI_FWD_SIG || EPI == EPI_FWD_LOGITS) {
 #pragma unroll 4
-            for (int j = 0; j < 16; ++j)
-              if (nc + j < ep.N) epi_elem<EPI, __nv_bfloat16, false>(ep, r, nc + j, v[j]);
+              for (int j = 0; j < 16; ++j)
+                if (nc + j < ep.N) {
+                  const float z = v[j] + sbias[c + j];
+                  if (EPI == EPI_FWD_LOGITS) {
+                    static_cast<float*>(ep.out0)[(int64_t)r * ep.ld0 + nc + j] = z;
+                  } else {
+                    const float hv = sigmoidf_(z);
+                    static_cast<__nv_bfloat16*>(ep.out0)[(int64_t)r * ep.ld0 + nc + j] = __float2bfloat16_rn(hv);
+                    if (ep.out1)
+                      static_cast<__nv_bfloat16*>(ep.out1)[(int64_t)r * ep.ld1 + nc + j] =
+                          __float2bfloat16_rn(hv * (1.f - hv));
+                  }
+                }
+            } else {
+              const bool vec_ok = full && !ep.transposed && (EPI != EPI_WGRAD_SGD || ep.shadow != nullptr) &&
+                                  EPI != EPI_WGRAD_STORE;
+              if (vec_ok) {
+                epi_row16_bf16<EPI>(ep, r, nc, v);
+              } else {
+#pragma unroll 4
+                for (int j = 0; j < 16; ++j)
+                  if (nc + j < ep.N) epi_elem<EPI, __nv_bfloat16, false>(ep, r, nc + j, v[j]);
+              }
+            }
           }
         }
       }
       if (EPI == EPI_DGRAD_SIG && ep.bpart_out) {
         epi_bar_sync();
-        for (int cc = rl; cc < BN && n0 + cc < ep.N; cc += 128)
+        for (int cc = et; cc < BN && n0 + cc < ep.N; cc += 256)
           ep.bpart_out[(int64_t)blockIdx.y * ep.ldp + n0 + cc] =
               (red[cc] + red[BN + cc]) + (red[2 * BN + cc] + red[3 * BN + cc]);
       }
-      if ((EPI == EPI_WGRAD_SGD || EPI == EPI_WGRAD_STORE) && ep.bpart_in) {
-        // db = sum of the dZ producer's per-tile partials, fixed order; bias index = W row
-        // non-transposed: the n-tile-0 CTA owns bias rows m0..m0+127 (one per thread);
+      if ((EPI == EPI_WGRAD_SGD || EPI == EPI_WGRAD_STORE) && ep.bpart_in && splits == 1) {
+        // db = sum of the dZ producer's per-tile partials, fixed order; bias index = W row.
+        // non-transposed: the n-tile-0 CTA owns bias rows m0..m0+127;
         // transposed (small head): the m-tile-0 CTA owns bias entries n0..n0+BN-1
         const bool own = !ep.transposed ? (blockIdx.x == 0) : (blockIdx.y == 0);
-        const int lo = !ep.transposed ? r : n0 + rl;
+        const int lo = !ep.transposed ? m0 + et : n0 + et;
         const int hi = !ep.transposed ? min(ep.M, m0 + TC_BM) : min(ep.N, n0 + BN);
         if (own)
-          for (int bi = lo; bi < hi; bi += 128) {
+          for (int bi = lo; bi < hi; bi += 256) {
+            float sdb = 0.f;
+            for (int t = 0; t < ep.n_mtiles; ++t) sdb += ep.bpart_in[(int64_t)t * ep.ldp + bi];
+            if (EPI == EPI_WGRAD_SGD)
+              ep.bias_upd[bi] -= ep.lr * sdb;
+            else
+              ep.bias_grad[bi] = sdb;
+          }
+      }
+    }
+  }
+
+  if ((EPI == EPI_WGRAD_SGD || EPI == EPI_WGRAD_STORE) && splits > 1) {
+    // ---- split-K reduce-scatter: CTA kz of the cluster reduces rows [kz*rps, (kz+1)*rps) of the
+    //      tile over the `splits` partials in fixed order and applies the fused SGD update ----
+    __threadfence();
+    cluster_sync_all();
+    if (warp >= 4) {
+      const int tid = threadIdx.x - 128;  // 0..255
+      const int rps = TC_BM / splits;
+      const size_t tile_base = ((size_t)blockIdx.y * gridDim.x + blockIdx.x) * splits * TC_BM * BN;
+      for (int e = tid * 4; e < rps * BN; e += 256 * 4) {
+        const int rloc = kz * rps + e / BN, col = e % BN;
+        float4 acc = make_float4(0.f, 0.f, 0.f, 0.f);
+        for (int sp = 0; sp < splits; ++sp) {
+          const float4 t = *reinterpret_cast<const float4*>(ep.ws + tile_base + ((size_t)sp * TC_BM + rloc) * BN + col);
+          acc.x += t.x;
+          acc.y += t.y;
+          acc.z += t.z;
+          acc.w += t.w;
+        }
+        const int gm = m0 + rloc, gn = n0 + col;
+        if (gm >= ep.M || gn >= ep.N) continue;
+        const float a4[4] = {acc.x, acc.y, acc.z, acc.w};
+        if (!ep.transposed && gn + 4 <= ep.N && EPI == EPI_WGRAD_SGD) {
+          float4* W = reinterpret_cast<float4*>(ep.master + (int64_t)gm * ep.ldw + gn);
+          float4 w = *W;
+          w.x -= ep.lr * acc.x;
+          w.y -= ep.lr * acc.y;
+          w.z -= ep.lr * acc.z;
+          w.w -= ep.lr * acc.w;
+          *W = w;
+          uint2 sh = make_uint2(pack_bf16x2(w.x, w.y), pack_bf16x2(w.z, w.w));
+          *reinterpret_cast<uint2*>(ep.shadow + (int64_t)gm * ep.ldw + gn) = sh;
+        } else {
+#pragma unroll
+          for (int j = 0; j < 4; ++j)
+            if (gn + j < ep.N) epi_elem<EPI, __nv_bfloat16, false>(ep, gm, gn + j, a4[j]);
+        }
+      }
+      if (ep.bpart_in) {  // bias: rows of this CTA's slice (or, transposed, the tile's columns)
+        int lo, hi;
+        bool own;
+        if (!ep.transposed) {
+          own = blockIdx.x == 0;
+          lo = m0 + kz * rps + tid;
+          hi = min(ep.M, m0 + (kz + 1) * rps);
+        } else {
+          own = blockIdx.y == 0 && kz == 0;
+          lo = n0 + tid;
+          hi = min(ep.N, n0 + BN);
+        }
+        if (own)
+          for (int bi = lo; bi < hi; bi += 256) {
             float sdb = 0.f;
             for (int t = 0; t < ep.n_mtiles; ++t) sdb += ep.bpart_in[(int64_t)t * ep.ldp + bi];
             if (EPI == EPI_WGRAD_SGD)
