@@ -214,6 +214,11 @@ typedef struct hb_prof_entry {
 int64_t hb_kernel_launches(void);
 int hb_prof_enable(int32_t on);
 int hb_prof_read(hb_prof_entry* out, int32_t n, int32_t reset);
+/* tuning only: mean device microseconds of one tensor-core GEMM launch of the given kind
+ * (0 forward+sigmoid, 1 dgrad+sigma', 2 wgrad+SGD) and shape on zero-filled scratch buffers */
+int hb_bench_gemm(int32_t kind, int32_t M, int32_t N, int32_t K, int32_t iters, float* us_out);
+/* tuning only: per-CTA phase timestamps (8 globaltimer ns values per CTA, cap entries) of one launch */
+int hb_bench_gemm_phases(int32_t kind, int32_t M, int32_t N, int32_t K, unsigned long long* host_ts, int64_t cap);
 
 /* ---- multi-GPU replica merge over NCCL (future work L277) -------- */
 int hb_nccl_unique_id(uint8_t out[128]);

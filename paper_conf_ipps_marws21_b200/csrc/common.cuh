@@ -167,6 +167,22 @@ __device__ __forceinline__ void cluster_sync_all() {
   asm volatile("barrier.cluster.wait.acquire.aligned;" ::: "memory");
 }
 
-__device__ __forceinline__ float sigmoidf_(float z) { return 1.0f / (1.0f + __expf(-z)); }
+__device__ __forceinline__ unsigned long long gtimer() {
+  unsigned long long t;
+  asm volatile("mov.u64 %0, %globaltimer;" : "=l"(t));
+  return t;
+}
+
+__device__ __forceinline__ float sigmoidf_(float z) { return __fdividef(1.0f, 1.0f + __expf(-z)); }
+
+// h = sigma(z) and d = sigma'(z) = sigma(z) (1 - sigma(z)) without cancellation or overflow:
+// with e = exp(-|z|) <= 1 and s = 1 / (1 + e):  sigma(|z|) = s, sigma(-|z|) = e s,  d = e s^2.
+__device__ __forceinline__ void sigmoid_d(float z, float& h, float& d) {
+  const float e = __expf(-fabsf(z));
+  const float s = __fdividef(1.0f, 1.0f + e);
+  const float es = e * s;
+  h = z >= 0.f ? s : es;
+  d = es * s;
+}
 
 }  // namespace hb

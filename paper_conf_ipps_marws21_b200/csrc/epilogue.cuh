@@ -38,6 +38,7 @@ struct EpiArgs {
   float* bias_upd;      // WGRAD_SGD: b_l -= lr * db_l in place
   float* bias_grad;     // WGRAD_STORE: db_l written out
   float* ws;            // WGRAD split-K: fp32 partial tiles [tiles][splits][128][BN]
+  unsigned long long* dbg;  // tuning only: per-CTA phase timestamps (globaltimer ns), nullable
   // softmax cross-entropy head fused into the output-layer GEMM (C <= 16):
   const int32_t* y;     // labels (dataset base when yoff != nullptr)
   const int* yoff;      // device row offset of the batch (graph replay), nullable
@@ -62,9 +63,16 @@ template <int EPI, typename TAct, bool PRECISE>
 __device__ __forceinline__ void epi_elem(const EpiArgs& ep, int r, int n, float v) {
   if (EPI == EPI_FWD_SIG) {
     float z = v + ep.bias[n];
-    float h = PRECISE ? 1.0f / (1.0f + expf(-z)) : sigmoidf_(z);
+    float h, d;
+    if (PRECISE) {  // check mode: IEEE exp/div, same cancellation-free form
+      const float e = expf(-fabsf(z)), s = 1.0f / (1.0f + e);
+      h = z >= 0.f ? s : e * s;
+      d = e * s * s;
+    } else {
+      sigmoid_d(z, h, d);
+    }
     static_cast<TAct*>(ep.out0)[(int64_t)r * ep.ld0 + n] = to_act<TAct>(h);
-    if (ep.out1) static_cast<TAct*>(ep.out1)[(int64_t)r * ep.ld1 + n] = to_act<TAct>(h * (1.0f - h));
+    if (ep.out1) static_cast<TAct*>(ep.out1)[(int64_t)r * ep.ld1 + n] = to_act<TAct>(d);
   } else if (EPI == EPI_FWD_LOGITS) {
     static_cast<float*>(ep.out0)[(int64_t)r * ep.ld0 + n] = v + ep.bias[n];
   } else if (EPI == EPI_DGRAD_SIG) {
@@ -98,11 +106,15 @@ __device__ __forceinline__ void epi_row16_bf16(const EpiArgs& ep, int r, int n0,
       float4 bb = __ldg(b4 + q);
       float z0 = v[4 * q] + bb.x, z1 = v[4 * q + 1] + bb.y, z2 = v[4 * q + 2] + bb.z,
             z3 = v[4 * q + 3] + bb.w;
-      float h0 = sigmoidf_(z0), h1 = sigmoidf_(z1), h2 = sigmoidf_(z2), h3 = sigmoidf_(z3);
+      float h0, h1, h2, h3, d0, d1, d2, d3;
+      sigmoid_d(z0, h0, d0);
+      sigmoid_d(z1, h1, d1);
+      sigmoid_d(z2, h2, d2);
+      sigmoid_d(z3, h3, d3);
       hp[2 * q] = pack_bf16x2(h0, h1);
       hp[2 * q + 1] = pack_bf16x2(h2, h3);
-      sp[2 * q] = pack_bf16x2(h0 * (1.f - h0), h1 * (1.f - h1));
-      sp[2 * q + 1] = pack_bf16x2(h2 * (1.f - h2), h3 * (1.f - h3));
+      sp[2 * q] = pack_bf16x2(d0, d1);
+      sp[2 * q + 1] = pack_bf16x2(d2, d3);
     }
     uint4* H = reinterpret_cast<uint4*>(static_cast<__nv_bfloat16*>(ep.out0) + (int64_t)r * ep.ld0 + n0);
     H[0] = make_uint4(hp[0], hp[1], hp[2], hp[3]);

@@ -941,6 +941,120 @@ int mlp_step_grads(hb_worker* w, const void* X, int64_t ldx, int32_t x_dtype, co
   return HB_OK;
 }
 
+// Test/tuning only: times `iters` launches of one tensor-core GEMM configuration on scratch
+// buffers (bf16 operands filled with zeros, fp32 master); kind 0 = forward (bias+sigmoid),
+// 1 = dgrad (sigma'), 2 = wgrad + SGD.  Reports the mean device microseconds per launch.
+static int bench_gemm_impl(int32_t kind, int32_t M, int32_t N, int32_t K, int32_t iters, float* us_out,
+                           unsigned long long* host_ts, int64_t cap);
+int hb_bench_gemm(int32_t kind, int32_t M, int32_t N, int32_t K, int32_t iters, float* us_out) {
+  return bench_gemm_impl(kind, M, N, K, iters, us_out, nullptr, 0);
+}
+// tuning only: per-CTA phase timestamps of one launch (8 globaltimer values per CTA)
+int hb_bench_gemm_phases(int32_t kind, int32_t M, int32_t N, int32_t K, unsigned long long* host_ts, int64_t cap) {
+  float us = 0.f;
+  return bench_gemm_impl(kind, M, N, K, 1, &us, host_ts, cap);
+}
+static int bench_gemm_impl(int32_t kind, int32_t M, int32_t N, int32_t K, int32_t iters, float* us_out,
+                           unsigned long long* host_ts, int64_t cap) {
+  HB_CHECK_ARG(us_out && M > 0 && N > 0 && K > 0 && iters > 0 && kind >= 0 && kind <= 3, "bad args");
+  const bool nostore = kind == 3;  // forward without output stores (epilogue cost probe)
+  if (nostore) kind = 0;
+  const int64_t lda = round_up(kind == 2 ? M : K, 8), ldb = round_up(kind == 0 ? K : N, 8);
+  const int64_t ldo = round_up(N, 8);
+  const int64_t arows = kind == 2 ? K : M, brows = kind == 0 ? N : K;
+  void *A = nullptr, *B = nullptr, *O = nullptr, *S = nullptr;
+  float *W = nullptr, *bias = nullptr, *ws = nullptr, *bp = nullptr;
+  __nv_bfloat16* Wsh = nullptr;
+  size_t out_elems = (size_t)std::max<int64_t>(M, 1) * ldo;
+  if (cudaMalloc(&A, arows * lda * 2) || cudaMalloc(&B, brows * ldb * 2) || cudaMalloc(&O, out_elems * 2) ||
+      cudaMalloc(&S, out_elems * 2) || cudaMalloc(&W, out_elems * 4) || cudaMalloc(&Wsh, out_elems * 2) ||
+      cudaMalloc(&bias, ldo * 4 + 64) || cudaMalloc(&ws, (size_t)148 * TC_BM * 256 * 4) ||
+      cudaMalloc(&bp, (size_t)((std::max(M, K) + 127) / 128) * ldo * 4 + 4096))
+    return fail(HB_ENOMEM, "bench alloc");
+  cudaMemset(A, 0, arows * lda * 2);
+  cudaMemset(B, 0, brows * ldb * 2);
+  cudaMemset(W, 0, out_elems * 4);
+  cudaMemset(bias, 0, ldo * 4 + 64);
+  cudaMemset(S, 0, out_elems * 2);
+  cudaMemset(bp, 0, (size_t)((std::max(M, K) + 127) / 128) * ldo * 4 + 4096);
+  cudaStream_t s;
+  cudaStreamCreate(&s);
+  EpiArgs ep{};
+  ep.M = M;
+  ep.N = N;
+  int epi;
+  bool a_mn = false, b_mn = false;
+  if (kind == 0) {
+    epi = EPI_FWD_SIG;
+    ep.bias = bias;
+    ep.out0 = O;
+    ep.out1 = S;
+    ep.ld0 = ep.ld1 = ldo;
+    if (nostore) ep.ld0 = -1;
+  } else if (kind == 1) {
+    epi = EPI_DGRAD_SIG;
+    b_mn = true;
+    ep.out0 = O;
+    ep.ld0 = ldo;
+    ep.aux = S;
+    ep.ldaux = ldo;
+    ep.bpart_out = bp;
+    ep.ldp = N;
+  } else {
+    epi = EPI_WGRAD_SGD;
+    a_mn = b_mn = true;
+    ep.master = W;
+    ep.shadow = Wsh;
+    ep.ldw = ldo;
+    ep.lr = 0.f;
+    ep.ws = ws;
+    ep.bpart_in = bp;
+    ep.ldp = M;
+    ep.n_mtiles = (K + 127) / 128;
+    ep.bias_upd = bias;
+  }
+  TcOp a{A, lda, arows, nullptr}, b{B, ldb, brows, nullptr};
+  int rc = gemm_tc(epi, a_mn, b_mn, M, N, K, a, b, ep, s);  // warm-up (sets kernel attributes)
+  if (host_ts && !rc) {
+    unsigned long long* d = nullptr;
+    cudaMalloc(&d, cap * sizeof(unsigned long long));
+    cudaMemsetAsync(d, 0, cap * sizeof(unsigned long long), s);
+    EpiArgs e2 = ep;
+    e2.dbg = d;
+    rc = gemm_tc(epi, a_mn, b_mn, M, N, K, a, b, e2, s);
+    cudaMemcpyAsync(host_ts, d, cap * sizeof(unsigned long long), cudaMemcpyDeviceToHost, s);
+    cudaStreamSynchronize(s);
+    cudaFree(d);
+  }
+  // capture the launches in a graph so the timing is device time, not host launch cost
+  cudaGraph_t g = nullptr;
+  cudaGraphExec_t ge = nullptr;
+  cudaStreamBeginCapture(s, cudaStreamCaptureModeThreadLocal);
+  for (int i = 0; i < iters && !rc; ++i) rc = gemm_tc(epi, a_mn, b_mn, M, N, K, a, b, ep, s);
+  cudaStreamEndCapture(s, &g);
+  if (!rc && g) cudaGraphInstantiate(&ge, g, 0);
+  if (ge) cudaGraphLaunch(ge, s);
+  cudaEvent_t e0, e1;
+  cudaEventCreate(&e0);
+  cudaEventCreate(&e1);
+  cudaEventRecord(e0, s);
+  if (ge) cudaGraphLaunch(ge, s);
+  cudaEventRecord(e1, s);
+  cudaStreamSynchronize(s);
+  if (ge) cudaGraphExecDestroy(ge);
+  if (g) cudaGraphDestroy(g);
+  float ms = 0.f;
+  cudaEventElapsedTime(&ms, e0, e1);
+  *us_out = ms * 1000.f / iters;
+  cudaEventDestroy(e0);
+  cudaEventDestroy(e1);
+  cudaStreamDestroy(s);
+  cudaFree(A); cudaFree(B); cudaFree(O); cudaFree(S); cudaFree(W); cudaFree(Wsh); cudaFree(bias); cudaFree(ws);
+  cudaFree(bp);
+  if (!rc && cudaGetLastError() != cudaSuccess) return fail(HB_ECUDA, "bench kernel failed");
+  return rc;
+}
+
 int mlp_loss(hb_model* m, const void* X, int64_t ldx, int32_t x_dtype, const int32_t* y, int64_t n,
              double* loss_out) {
   HB_CHECK_ARG(m && loss_out, "null arg");

@@ -42,9 +42,7 @@ struct TcCfg {
   static constexpr int STAGES_RAW = (192 * 1024) / STAGE_BYTES;
   static constexpr int STAGES = STAGES_RAW > 8 ? 8 : STAGES_RAW;
   static constexpr int TMEM_COLS = BN <= 32 ? 32 : BN;                  // power of two >= 32
-  static constexpr int RED_BYTES = 4 * BN * 4;                          // per-quadrant column sums
-  static constexpr int BIAS_BYTES = BN * 4;                             // staged bias of the tile
-  static constexpr int SMEM_BYTES = STAGES * STAGE_BYTES + 1024 /*align*/ + 256 /*barriers*/ + RED_BYTES + BIAS_BYTES;
+  static constexpr int SMEM_BYTES = STAGES * STAGE_BYTES + 1024 /*align*/ + 256 /*barriers*/;
 };
 
 __device__ __forceinline__ void epi_bar_sync() { asm volatile("bar.sync 1, 256;" ::: "memory"); }
@@ -93,11 +91,13 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
   uint64_t* empty_bar = full_bar + STAGES;
   uint64_t* tmem_full_bar = empty_bar + STAGES;
   uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(tmem_full_bar + 1);
-  float* red = reinterpret_cast<float*>(smem + STAGES * Cfg::STAGE_BYTES + 256);  // [4][BN]
-  float* sbias = red + 4 * BN;                                                      // [BN]
+  __shared__ float red[4 * BN];  // per-quadrant column sums (bias-gradient partials)
+  __shared__ float sbias[BN];    // the tile's bias
 
   const int warp = threadIdx.x >> 5;
   const int lane = threadIdx.x & 31;
+  unsigned long long* dbg = ep.dbg ? ep.dbg + 8 * ((size_t)(blockIdx.z * gridDim.y + blockIdx.y) * gridDim.x + blockIdx.x) : nullptr;
+  if (dbg && threadIdx.x == 0) dbg[0] = gtimer();
   const int n0 = blockIdx.x * BN;
   const int m0 = blockIdx.y * TC_BM;
   // split-K (dW GEMMs with K = batch): the gridDim.z CTAs of one output tile form a cluster,
@@ -124,6 +124,7 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
   __syncthreads();
   tc_fence_after();
   const uint32_t tmem_base = *tmem_slot;
+  if (dbg && threadIdx.x == 0) dbg[1] = gtimer();
 
   if (warp == 0 && lane == 0) {
     // ===== TMA producer =====
@@ -159,6 +160,7 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
       const uint32_t ph = (kb / STAGES) & 1;
       mbar_wait(&full_bar[s], ph);
       tc_fence_after();
+      if (dbg && kb == 0) dbg[2] = gtimer();
       const uint32_t a_base = smem_u32(smem + s * Cfg::STAGE_BYTES);
       const uint32_t b_base = a_base + Cfg::A_BYTES;
 #pragma unroll
@@ -175,6 +177,7 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
       umma_commit(&empty_bar[s]);  // frees the smem slot when these MMAs complete
     }
     umma_commit(tmem_full_bar);     // accumulator ready
+    if (dbg) dbg[3] = gtimer();
   } else if (warp >= 4) {
     // ===== epilogue (8 warps): TMEM -> registers -> fused epilogue -> global =====
     // warp w reads TMEM lanes 32*(w%4).. (tile rows) and handles column half h = (w-4)/4
@@ -209,8 +212,10 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
       }
     }
     epi_bar_sync();  // sbias visible
+    if (dbg && et == 0) dbg[4] = gtimer();
     mbar_wait(tmem_full_bar, 0);
     tc_fence_after();
+    if (dbg && et == 0) dbg[5] = gtimer();
 
     if (EPI == EPI_HEAD_XENT) {
       // ---- softmax cross-entropy on the thread's own row of logits (N = C <= BN = 16) ----
@@ -264,7 +269,7 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
       }
     } else {
       if (active) {
-#pragma unroll 1
+#pragma unroll
         for (int cc = 0; cc < HALF; cc += 16) {
           const int c = c_lo + cc;
           if (n0 + c >= ep.N) break;  // warp-uniform
@@ -335,14 +340,24 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
 #pragma unroll
             for (int qq = 0; qq < 4; ++qq) wsp[qq] = make_float4(v[4 * qq], v[4 * qq + 1], v[4 * qq + 2], v[4 * qq + 3]);
           } else if (row_ok) {
-            if (EPI == EPI_FWD_SIG && full) {
+            if (EPI == EPI_FWD_SIG && ep.ld0 < 0) {  // tuning probe: epilogue math, no stores
+              float acc = 0.f;
+#pragma unroll
+              for (int qq = 0; qq < 16; ++qq) {
+                float hv, dv;
+                sigmoid_d(v[qq] + sbias[c + qq], hv, dv);
+                acc += hv + dv;
+              }
+              if (acc == 12345.f) static_cast<float*>(ep.bias_upd)[0] = acc;
+            } else if (EPI == EPI_FWD_SIG && full) {
               uint32_t hp[8], sp[8];
 #pragma unroll
               for (int qq = 0; qq < 8; ++qq) {
-                const float z0 = v[2 * qq] + sbias[c + 2 * qq], z1 = v[2 * qq + 1] + sbias[c + 2 * qq + 1];
-                const float h0 = sigmoidf_(z0), h1 = sigmoidf_(z1);
+                float h0, d0, h1, d1;
+                sigmoid_d(v[2 * qq] + sbias[c + 2 * qq], h0, d0);
+                sigmoid_d(v[2 * qq + 1] + sbias[c + 2 * qq + 1], h1, d1);
                 hp[qq] = pack_bf16x2(h0, h1);
-                sp[qq] = pack_bf16x2(h0 * (1.f - h0), h1 * (1.f - h1));
+                sp[qq] = pack_bf16x2(d0, d1);
               }
               uint4* H = reinterpret_cast<uint4*>(static_cast<__nv_bfloat16*>(ep.out0) + (int64_t)r * ep.ld0 + nc);
               H[0] = make_uint4(hp[0], hp[1], hp[2], hp[3]);
@@ -353,18 +368,18 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
                 S[1] = make_uint4(sp[4], sp[5], sp[6], sp[7]);
               }
             } else if (EPI == EPI_FWD_SIG || EPI == EPI_FWD_LOGITS) {
-#pragma unroll 4
+#pragma unroll
               for (int j = 0; j < 16; ++j)
                 if (nc + j < ep.N) {
                   const float z = v[j] + sbias[c + j];
                   if (EPI == EPI_FWD_LOGITS) {
                     static_cast<float*>(ep.out0)[(int64_t)r * ep.ld0 + nc + j] = z;
                   } else {
-                    const float hv = sigmoidf_(z);
+                    float hv, dv;
+                    sigmoid_d(z, hv, dv);
                     static_cast<__nv_bfloat16*>(ep.out0)[(int64_t)r * ep.ld0 + nc + j] = __float2bfloat16_rn(hv);
                     if (ep.out1)
-                      static_cast<__nv_bfloat16*>(ep.out1)[(int64_t)r * ep.ld1 + nc + j] =
-                          __float2bfloat16_rn(hv * (1.f - hv));
+                      static_cast<__nv_bfloat16*>(ep.out1)[(int64_t)r * ep.ld1 + nc + j] = __float2bfloat16_rn(dv);
                   }
                 }
             } else {
@@ -373,7 +388,7 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
               if (vec_ok) {
                 epi_row16_bf16<EPI>(ep, r, nc, v);
               } else {
-#pragma unroll 4
+#pragma unroll
                 for (int j = 0; j < 16; ++j)
                   if (nc + j < ep.N) epi_elem<EPI, __nv_bfloat16, false>(ep, r, nc + j, v[j]);
               }
@@ -470,12 +485,14 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
     }
   }
 
+  if (dbg && threadIdx.x == 128) dbg[6] = gtimer();
   tc_fence_before();
   __syncthreads();
   if (warp == 2) {
     tc_fence_after();
     tmem_dealloc<Cfg::TMEM_COLS>(tmem_base);
   }
+  if (dbg && threadIdx.x == 64) dbg[7] = gtimer();
 }
 
 }  // namespace hb
