@@ -109,7 +109,8 @@ class ClockSampler:
                 "reasons": sorted(reasons), "samples": len(sm)}
 
 
-def make_data(cfg, rank, N):
+def make_data(cfg, rank, N, dense=True):
+    """Seeded synthetic dataset (synth/).  dense=False returns the CSR of sparse-shaped data."""
     from synth import covtype_like, pad_cols
     from synth.data import csr_to_dense, sparse_like
     d = cfg["dims"][0]
@@ -120,7 +121,29 @@ def make_data(cfg, rank, N):
         csr, y = sparse_like(N, 300, 11.6, 0.03, True, seed=rank)
     else:
         csr, y = sparse_like(N, 20958, 51.5, 0.31, False, seed=rank)
-    return csr_to_dense(csr, d, (d + 7) // 8 * 8), y
+    return (csr_to_dense(csr, d, (d + 7) // 8 * 8) if dense else csr), y
+
+
+def device_data(cfg, rank, N, device):
+    """(X_host pinned bf16, y_host pinned int32, X_dev, y_dev).  Sparse-shaped data is
+    densified on the device ("processed in dense format"); the host copy used
+    by the e2e leg is then a pinned copy of the same dense matrix."""
+    import torch
+    d = cfg["dims"][0]
+    ld = (d + 7) // 8 * 8
+    if cfg["data"] == "covtype" or (N * ld * 4) < (4 << 30):
+        Xp, y = make_data(cfg, rank, N)
+        X_host = torch.from_numpy(Xp).to(torch.bfloat16).pin_memory()
+        Xd = X_host.to(device)
+    else:
+        (indptr, indices, vals), y = make_data(cfg, rank, N, dense=False)
+        rows = torch.from_numpy(np.repeat(np.arange(N), np.diff(indptr))).to(device)
+        Xd = torch.zeros(N, ld, dtype=torch.bfloat16, device=device)
+        Xd[rows, torch.from_numpy(indices.astype(np.int64)).to(device)] = torch.from_numpy(vals).to(device).to(torch.bfloat16)
+        X_host = torch.empty(N, ld, dtype=torch.bfloat16, pin_memory=True)
+        X_host.copy_(Xd)
+    y_host = torch.from_numpy(y.astype(np.int32)).pin_memory()
+    return X_host, y_host, Xd, y_host.to(device)
 
 
 # --------------------------------------------------------------------------------------------
@@ -134,6 +157,7 @@ def oracle_arm(cfg, args, rows_per_step, budget_note):
     b = min(8192, rows_per_step)
     Xp, y = make_data(cfg, 0, rows_per_step)
     X = Xp[:, :dims[0]].astype(np.float64)
+    y = y[:rows_per_step]
     params = init_params(dims, seed=2)
     lr = args.eta0 * b / args.b0
 
@@ -217,12 +241,7 @@ def main():
     from synth import init_params, params_to_flat
 
     # ---- data + model (resident in HBM before timing) ----
-    Xp, y = make_data(cfg, rank, N)
-    ld = Xp.shape[1]
-    X_host = torch.from_numpy(Xp).to(torch.bfloat16).pin_memory()
-    y_host = torch.from_numpy(y.astype(np.int32)).pin_memory()
-    Xd = X_host.to(f"cuda:{local}")
-    yd = y_host.to(f"cuda:{local}")
+    X_host, y_host, Xd, yd = device_data(cfg, rank, N, f"cuda:{local}")
     model = hb.MLP(dims, precision="bf16", seed=0, device=local)
     model.set_params(params_to_flat(init_params(dims, seed=2)))
     big_max = 8192

@@ -9,6 +9,7 @@
 
 #include <atomic>
 #include <cmath>
+#include <cstdlib>
 #include <cstring>
 #include <mutex>
 #include <random>
@@ -177,12 +178,28 @@ static int launch_tc_bn(int bn, const CUtensorMap& ma, const CUtensorMap& mb, in
 
 // split-K factor of a dW GEMM (K = batch): enough CTAs to cover the 148 SMs, power of two
 // <= 8 (portable cluster size), at least one k-block per split
+static int env_int(const char* name, int dflt) {
+  const char* v = getenv(name);
+  return v && *v ? atoi(v) : dflt;
+}
+
 int choose_splits(int M, int N, int K, int bn) {
+  static const int max_s = env_int("HB_MAX_SPLITS", 4);  // 8-CTA clusters of 200 KB CTAs do not all co-reside
   const long tiles = (long)((M + TC_BM - 1) / TC_BM) * ((N + bn - 1) / bn);
   const int nkb = (K + TC_BK - 1) / TC_BK;
   int S = 1;
-  while (S * 2 <= 8 && tiles * S * 2 <= 148 && S * 2 <= nkb) S *= 2;
+  while (S * 2 <= max_s && tiles * S * 2 <= 148 && S * 2 <= nkb) S *= 2;
+  if (S == 4 && tiles * 8 <= 64 && 8 <= nkb) S = 8;  // a few 8-CTA clusters still co-reside
   return S;
+}
+
+// tile width of a dW GEMM: narrow enough that tiles x splits fill the SMs
+static int choose_bn_wgrad(int M, int N, int K) {
+  static const int forced = env_int("HB_WGRAD_BN", 0);
+  if (forced) return forced;
+  int bn = choose_bn(M, N);
+  while (bn > 64 && (long)((M + TC_BM - 1) / TC_BM) * ((N + bn - 1) / bn) * 4 < 148 && K >= 2048) bn /= 2;
+  return bn;
 }
 
 int choose_bn(int M, int N) {
@@ -207,7 +224,9 @@ struct TcOp {
 
 static int gemm_tc(int epi, bool a_mn, bool b_mn, int M, int N, int K, TcOp A, TcOp B, const EpiArgs& ep,
                    cudaStream_t s) {
-  const int bn = epi == EPI_HEAD_XENT ? 16 : choose_bn(M, N);
+  const int bn = epi == EPI_HEAD_XENT                          ? 16
+                 : (epi == EPI_WGRAD_SGD || epi == EPI_WGRAD_STORE) ? choose_bn_wgrad(M, N, K)
+                                                                    : choose_bn(M, N);
   CUtensorMap ma, mb;
   const int64_t ar = A.rows ? A.rows : (a_mn ? K : M);
   const int64_t br = B.rows ? B.rows : (b_mn ? K : N);
