@@ -142,24 +142,39 @@ static int launch_tc(const CUtensorMap& ma, const CUtensorMap& mb, int M, int N,
       g_attr_done.insert(key);
     }
   }
-  dim3 grid((N + BN - 1) / BN, (M + TC_BM - 1) / TC_BM, splits);
-  if (splits == 1) {
-    kern<<<grid, TC_THREADS, Cfg::SMEM_BYTES, s>>>(ma, mb, K, offA, offB, ep);
-  } else {  // split-K: the `splits` CTAs of a tile form one thread-block cluster along z
-    cudaLaunchConfig_t cfg{};
-    cfg.gridDim = grid;
-    cfg.blockDim = dim3(TC_THREADS);
-    cfg.dynamicSmemBytes = Cfg::SMEM_BYTES;
-    cfg.stream = s;
-    cudaLaunchAttribute attr[1];
-    attr[0].id = cudaLaunchAttributeClusterDimension;
-    attr[0].val.clusterDim.x = 1;
-    attr[0].val.clusterDim.y = 1;
-    attr[0].val.clusterDim.z = splits;
-    cfg.attrs = attr;
-    cfg.numAttrs = 1;
-    HB_CUDA_TRY(cudaLaunchKernelEx(&cfg, kern, ma, mb, K, offA, offB, ep));
+  // persistent: one CTA per SM (at most one per tile) walking the tiles; split-K: one CTA per
+  // (tile, split) with the splits of a tile in one cluster
+  const int tiles = ((N + BN - 1) / BN) * ((M + TC_BM - 1) / TC_BM);
+  static int nsm = 0;
+  if (!nsm) {
+    cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, dev);
+    if (nsm <= 0) nsm = 148;
   }
+  dim3 grid = splits == 1 ? dim3(std::min(tiles, nsm), 1, 1)
+                          : dim3((N + BN - 1) / BN, (M + TC_BM - 1) / TC_BM, splits);
+  cudaLaunchConfig_t cfg{};
+  cfg.gridDim = grid;
+  cfg.blockDim = dim3(TC_THREADS);
+  cfg.dynamicSmemBytes = Cfg::SMEM_BYTES;
+  cfg.stream = s;
+  cudaLaunchAttribute attr[2];
+  int na = 0;
+  static const bool pdl = !(getenv("HB_NO_PDL") && getenv("HB_NO_PDL")[0] == '1');
+  if (pdl) {  // programmatic dependent launch: prologue overlaps the previous kernel's tail
+    attr[na].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+    attr[na].val.programmaticStreamSerializationAllowed = 1;
+    ++na;
+  }
+  if (splits > 1) {
+    attr[na].id = cudaLaunchAttributeClusterDimension;
+    attr[na].val.clusterDim.x = 1;
+    attr[na].val.clusterDim.y = 1;
+    attr[na].val.clusterDim.z = splits;
+    ++na;
+  }
+  cfg.attrs = attr;
+  cfg.numAttrs = na;
+  HB_CUDA_TRY(cudaLaunchKernelEx(&cfg, kern, ma, mb, K, offA, offB, ep));
   HB_CUDA_TRY(cudaGetLastError());
   return HB_OK;
 }

@@ -41,7 +41,7 @@ struct TcCfg {
   static constexpr int STAGE_BYTES = A_BYTES + B_BYTES;
   static constexpr int STAGES_RAW = (192 * 1024) / STAGE_BYTES;
   static constexpr int STAGES = STAGES_RAW > 8 ? 8 : STAGES_RAW;
-  static constexpr int TMEM_COLS = BN <= 32 ? 32 : BN;                  // power of two >= 32
+  static constexpr int TMEM_COLS = 2 * BN < 32 ? 32 : 2 * BN;          // two accumulators (double buffer)
   static constexpr int SMEM_BYTES = STAGES * STAGE_BYTES + 1024 /*align*/ + 256 /*barriers*/;
 };
 
@@ -89,20 +89,26 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
   uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
   uint64_t* full_bar = reinterpret_cast<uint64_t*>(smem + STAGES * Cfg::STAGE_BYTES);
   uint64_t* empty_bar = full_bar + STAGES;
-  uint64_t* tmem_full_bar = empty_bar + STAGES;
-  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(tmem_full_bar + 1);
-  __shared__ float red[4 * BN];  // per-quadrant column sums (bias-gradient partials)
-  __shared__ float sbias[BN];    // the tile's bias
+  uint64_t* tmem_full_bar = empty_bar + STAGES;   // [2]: accumulator a ready (MMA -> epilogue)
+  uint64_t* tmem_empty_bar = tmem_full_bar + 2;    // [2]: accumulator a drained (epilogue -> MMA)
+  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(tmem_empty_bar + 2);
+  __shared__ float red[4 * BN];    // per-quadrant column sums (bias-gradient partials)
+  __shared__ float sbias[2][BN];   // bias of the tile, double-buffered across tiles
 
   const int warp = threadIdx.x >> 5;
   const int lane = threadIdx.x & 31;
   unsigned long long* dbg = ep.dbg ? ep.dbg + 8 * ((size_t)(blockIdx.z * gridDim.y + blockIdx.y) * gridDim.x + blockIdx.x) : nullptr;
   if (dbg && threadIdx.x == 0) dbg[0] = gtimer();
-  const int n0 = blockIdx.x * BN;
-  const int m0 = blockIdx.y * TC_BM;
+  // Tiles: persistent CTAs walk tiles t = blockIdx.x, +gridDim.x, ... (n fastest, so CTAs running
+  // together share the A row panel in L2).  Split-K launches (gridDim.z > 1) are one tile per CTA.
+  const int tiles_n = (ep.N + BN - 1) / BN;
+  const int tiles_m = (ep.M + TC_BM - 1) / TC_BM;
+  const int num_tiles = tiles_n * tiles_m;
   // split-K (dW GEMMs with K = batch): the gridDim.z CTAs of one output tile form a cluster,
   // each accumulates k-blocks [kb_lo, kb_hi) in its own TMEM
   const int splits = gridDim.z;
+  const int t_first = splits == 1 ? (int)blockIdx.x : (int)(blockIdx.y * gridDim.x + blockIdx.x);
+  const int t_step = splits == 1 ? (int)gridDim.x : num_tiles;
   const int kz = blockIdx.z;
   const int num_kb_all = (K + TC_BK - 1) / TC_BK;
   const int kpb = (num_kb_all + splits - 1) / splits;
@@ -116,7 +122,10 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
       mbar_init(&full_bar[s], 1);
       mbar_init(&empty_bar[s], 1);
     }
-    mbar_init(tmem_full_bar, 1);
+    for (int a = 0; a < 2; ++a) {
+      mbar_init(&tmem_full_bar[a], 1);
+      mbar_init(&tmem_empty_bar[a], 8);  // one arrive per epilogue warp
+    }
     fence_barrier_init();
   }
   if (warp == 2) tmem_alloc<Cfg::TMEM_COLS>(tmem_slot);
@@ -124,15 +133,22 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
   __syncthreads();
   tc_fence_after();
   const uint32_t tmem_base = *tmem_slot;
+  // programmatic dependent launch: everything above overlapped the previous kernel's tail;
+  // no global memory produced by it is touched before this point
+  asm volatile("griddepcontrol.wait;" ::: "memory");
+  asm volatile("griddepcontrol.launch_dependents;" ::: "memory");
   if (dbg && threadIdx.x == 0) dbg[1] = gtimer();
 
   if (warp == 0 && lane == 0) {
     // ===== TMA producer =====
     const int oa = offA ? __ldg(offA) : 0;
     const int ob = offB ? __ldg(offB) : 0;
-    for (int kb = 0; kb < num_kb; ++kb) {
-      const int s = kb % STAGES;
-      const uint32_t ph = (kb / STAGES) & 1;
+    int it = 0;  // k-blocks issued by this CTA (ring position across tiles)
+    for (int t = t_first; t < num_tiles; t += t_step) {
+    const int m0 = (t / tiles_n) * TC_BM, n0 = (t % tiles_n) * BN;
+    for (int kb = 0; kb < num_kb; ++kb, ++it) {
+      const int s = it % STAGES;
+      const uint32_t ph = (it / STAGES) & 1;
       mbar_wait(&empty_bar[s], ph ^ 1);
       uint8_t* sA = smem + s * Cfg::STAGE_BYTES;
       uint8_t* sB = sA + Cfg::A_BYTES;
@@ -152,15 +168,22 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
           tma_load_2d(sB + j * 8192, &tmB, &full_bar[s], n0 + 64 * j, k0 + ob);
       }
     }
+    }
   } else if (warp == 1 && lane == 0) {
     // ===== MMA issuer (single thread) =====
     constexpr uint32_t idesc = make_idesc_bf16(TC_BM, BN, A_MN, B_MN);
-    for (int kb = 0; kb < num_kb; ++kb) {
-      const int s = kb % STAGES;
-      const uint32_t ph = (kb / STAGES) & 1;
+    int it = 0, i = 0;
+    for (int t = t_first; t < num_tiles; t += t_step, ++i) {
+    const int acc = i & 1;
+    mbar_wait(&tmem_empty_bar[acc], ((i >> 1) & 1) ^ 1);  // epilogue has drained this accumulator
+    tc_fence_after();
+    const uint32_t tacc = tmem_base + (uint32_t)(acc * BN);
+    for (int kb = 0; kb < num_kb; ++kb, ++it) {
+      const int s = it % STAGES;
+      const uint32_t ph = (it / STAGES) & 1;
       mbar_wait(&full_bar[s], ph);
       tc_fence_after();
-      if (dbg && kb == 0) dbg[2] = gtimer();
+      if (dbg && it == 0) dbg[2] = gtimer();
       const uint32_t a_base = smem_u32(smem + s * Cfg::STAGE_BYTES);
       const uint32_t b_base = a_base + Cfg::A_BYTES;
 #pragma unroll
@@ -172,12 +195,13 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
                                  : make_sw128_desc(a_base + kk * 32, 16, 1024);
         const uint64_t bd = B_MN ? make_sw128_desc(b_base + kk * 2048, 8192, 1024)
                                  : make_sw128_desc(b_base + kk * 32, 16, 1024);
-        umma_bf16(tmem_base, ad, bd, idesc, (kb | kk) != 0);
+        umma_bf16(tacc, ad, bd, idesc, (kb | kk) != 0);
       }
       umma_commit(&empty_bar[s]);  // frees the smem slot when these MMAs complete
     }
-    umma_commit(tmem_full_bar);     // accumulator ready
-    if (dbg) dbg[3] = gtimer();
+    umma_commit(&tmem_full_bar[acc]);  // accumulator ready (arrives even if num_kb == 0)
+    if (dbg && i == 0) dbg[3] = gtimer();
+    }
   } else if (warp >= 4) {
     // ===== epilogue (8 warps): TMEM -> registers -> fused epilogue -> global =====
     // warp w reads TMEM lanes 32*(w%4).. (tile rows) and handles column half h = (w-4)/4
@@ -185,16 +209,22 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
     const int h = (warp - 4) >> 2;
     const int et = threadIdx.x - 128;  // 0..255
     const int rl = q * 32 + lane;      // row within the tile
-    const int r = m0 + rl;
-    const bool row_ok = r < ep.M;
-    const uint32_t tbase = tmem_base + ((uint32_t)(q * 32) << 16);
     constexpr int HALF = BN >= 32 ? BN / 2 : BN;  // columns per warp
     const bool active = BN >= 32 || h == 0;
     const int c_lo = BN >= 32 ? h * HALF : 0;
+    int i = 0;
+    for (int t = t_first; t < num_tiles; t += t_step, ++i) {
+    const int acc = i & 1;
+    const int m_tile = t / tiles_n, n_tile = t % tiles_n;
+    const int m0 = m_tile * TC_BM, n0 = n_tile * BN;
+    const int r = m0 + rl;
+    const bool row_ok = r < ep.M;
+    const uint32_t tbase = tmem_base + (uint32_t)(acc * BN) + ((uint32_t)(q * 32) << 16);
+    float* sb = sbias[acc];
 
     // stage the bias of the tile's columns in shared memory while the mainloop runs
     if (EPI == EPI_FWD_SIG || EPI == EPI_FWD_LOGITS || EPI == EPI_HEAD_XENT) {
-      for (int c = et; c < BN; c += 256) sbias[c] = n0 + c < ep.N ? ep.bias[n0 + c] : 0.f;
+      for (int c = et; c < BN; c += 256) sb[c] = n0 + c < ep.N ? ep.bias[n0 + c] : 0.f;
     }
     // DGRAD: prefetch this thread's row of sigma'(Z) (the S stash) for all of its columns
     constexpr int NCH = (HALF + 15) / 16;
@@ -211,11 +241,11 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
         }
       }
     }
-    epi_bar_sync();  // sbias visible
-    if (dbg && et == 0) dbg[4] = gtimer();
-    mbar_wait(tmem_full_bar, 0);
+    epi_bar_sync();  // sbias visible; previous tile's partial sums consumed
+    if (dbg && et == 0 && i == 0) dbg[4] = gtimer();
+    mbar_wait(&tmem_full_bar[acc], (i >> 1) & 1);
     tc_fence_after();
-    if (dbg && et == 0) dbg[5] = gtimer();
+    if (dbg && et == 0 && i == 0) dbg[5] = gtimer();
 
     if (EPI == EPI_HEAD_XENT) {
       // ---- softmax cross-entropy on the thread's own row of logits (N = C <= BN = 16) ----
@@ -231,7 +261,7 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
         float mx = -INFINITY;
 #pragma unroll
         for (int j = 0; j < 16; ++j) {
-          z[j] = j < C ? __uint_as_float(raw[j]) + sbias[j] : -INFINITY;
+          z[j] = j < C ? __uint_as_float(raw[j]) + sb[j] : -INFINITY;
           mx = fmaxf(mx, z[j]);
         }
         float se = 0.f;
@@ -265,7 +295,7 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
       if (ep.bpart_out) {
         epi_bar_sync();
         if (et < ep.N)
-          ep.bpart_out[(int64_t)blockIdx.y * ep.ldp + et] = (red[et] + red[BN + et]) + (red[2 * BN + et] + red[3 * BN + et]);
+          ep.bpart_out[(int64_t)m_tile * ep.ldp + et] = (red[et] + red[BN + et]) + (red[2 * BN + et] + red[3 * BN + et]);
       }
     } else {
       if (active) {
@@ -332,7 +362,7 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
           } else if ((EPI == EPI_WGRAD_SGD || EPI == EPI_WGRAD_STORE) && splits > 1) {
             // split-K: park the fp32 partial tile; reduced after the cluster barrier below
             float4* wsp = reinterpret_cast<float4*>(
-                ep.ws + ((((size_t)blockIdx.y * gridDim.x + blockIdx.x) * splits + kz) * TC_BM + rl) * BN + c);
+                ep.ws + ((((size_t)t) * splits + kz) * TC_BM + rl) * BN + c);
             if (num_kb == 0) {
 #pragma unroll
               for (int j = 0; j < 16; ++j) v[j] = 0.f;
@@ -345,7 +375,7 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
 #pragma unroll
               for (int qq = 0; qq < 16; ++qq) {
                 float hv, dv;
-                sigmoid_d(v[qq] + sbias[c + qq], hv, dv);
+                sigmoid_d(v[qq] + sb[c + qq], hv, dv);
                 acc += hv + dv;
               }
               if (acc == 12345.f) static_cast<float*>(ep.bias_upd)[0] = acc;
@@ -354,8 +384,8 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
 #pragma unroll
               for (int qq = 0; qq < 8; ++qq) {
                 float h0, d0, h1, d1;
-                sigmoid_d(v[2 * qq] + sbias[c + 2 * qq], h0, d0);
-                sigmoid_d(v[2 * qq + 1] + sbias[c + 2 * qq + 1], h1, d1);
+                sigmoid_d(v[2 * qq] + sb[c + 2 * qq], h0, d0);
+                sigmoid_d(v[2 * qq + 1] + sb[c + 2 * qq + 1], h1, d1);
                 hp[qq] = pack_bf16x2(h0, h1);
                 sp[qq] = pack_bf16x2(d0, d1);
               }
@@ -371,7 +401,7 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
 #pragma unroll
               for (int j = 0; j < 16; ++j)
                 if (nc + j < ep.N) {
-                  const float z = v[j] + sbias[c + j];
+                  const float z = v[j] + sb[c + j];
                   if (EPI == EPI_FWD_LOGITS) {
                     static_cast<float*>(ep.out0)[(int64_t)r * ep.ld0 + nc + j] = z;
                   } else {
@@ -399,14 +429,14 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
       if (EPI == EPI_DGRAD_SIG && ep.bpart_out) {
         epi_bar_sync();
         for (int cc = et; cc < BN && n0 + cc < ep.N; cc += 256)
-          ep.bpart_out[(int64_t)blockIdx.y * ep.ldp + n0 + cc] =
+          ep.bpart_out[(int64_t)m_tile * ep.ldp + n0 + cc] =
               (red[cc] + red[BN + cc]) + (red[2 * BN + cc] + red[3 * BN + cc]);
       }
       if ((EPI == EPI_WGRAD_SGD || EPI == EPI_WGRAD_STORE) && ep.bpart_in && splits == 1) {
         // db = sum of the dZ producer's per-tile partials, fixed order; bias index = W row.
         // non-transposed: the n-tile-0 CTA owns bias rows m0..m0+127;
         // transposed (small head): the m-tile-0 CTA owns bias entries n0..n0+BN-1
-        const bool own = !ep.transposed ? (blockIdx.x == 0) : (blockIdx.y == 0);
+        const bool own = !ep.transposed ? (n_tile == 0) : (m_tile == 0);
         const int lo = !ep.transposed ? m0 + et : n0 + et;
         const int hi = !ep.transposed ? min(ep.M, m0 + TC_BM) : min(ep.N, n0 + BN);
         if (own)
@@ -420,6 +450,11 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
           }
       }
     }
+    // release this accumulator to the MMA warp (all TMEM reads of the tile have completed)
+    tc_fence_before();
+    __syncwarp();
+    if (lane == 0) mbar_arrive(&tmem_empty_bar[acc]);
+    }  // tile loop
   }
 
   if ((EPI == EPI_WGRAD_SGD || EPI == EPI_WGRAD_STORE) && splits > 1) {
@@ -428,9 +463,11 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
     __threadfence();
     cluster_sync_all();
     if (warp >= 4) {
+      const int t = t_first;
+      const int m0 = (t / tiles_n) * TC_BM, n0 = (t % tiles_n) * BN;
       const int tid = threadIdx.x - 128;  // 0..255
       const int rps = TC_BM / splits;
-      const size_t tile_base = ((size_t)blockIdx.y * gridDim.x + blockIdx.x) * splits * TC_BM * BN;
+      const size_t tile_base = (size_t)t * splits * TC_BM * BN;
       for (int e = tid * 4; e < rps * BN; e += 256 * 4) {
         const int rloc = kz * rps + e / BN, col = e % BN;
         float4 acc = make_float4(0.f, 0.f, 0.f, 0.f);
@@ -464,11 +501,11 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
         int lo, hi;
         bool own;
         if (!ep.transposed) {
-          own = blockIdx.x == 0;
+          own = (t % tiles_n) == 0;
           lo = m0 + kz * rps + tid;
           hi = min(ep.M, m0 + (kz + 1) * rps);
         } else {
-          own = blockIdx.y == 0 && kz == 0;
+          own = (t / tiles_n) == 0 && kz == 0;
           lo = n0 + tid;
           hi = min(ep.N, n0 + BN);
         }
