@@ -79,6 +79,20 @@ __device__ __forceinline__ int colsum16_col(int lane) {
   return ((lane >> 4) & 1) * 8 + ((lane >> 3) & 1) * 4 + ((lane >> 2) & 1) * 2 + ((lane >> 1) & 1);
 }
 
+// Grouped tile rasterisation: consecutive tile indices walk down GROUP_M row tiles before moving
+// to the next column tile, so the ~148 tiles resident at once cover a compact block of the
+// output and share both their A row panels and their B column panels through L2.
+constexpr int TC_GROUP_M = 8;
+__device__ __forceinline__ void tile_coords(int t, int tiles_m, int tiles_n, int& m_tile, int& n_tile) {
+  const int per_group = TC_GROUP_M * tiles_n;
+  const int g = t / per_group;
+  const int first_m = g * TC_GROUP_M;
+  const int gm = min(tiles_m - first_m, TC_GROUP_M);
+  const int r = t - g * per_group;
+  m_tile = first_m + r % gm;
+  n_tile = r / gm;
+}
+
 template <int BN, bool A_MN, bool B_MN, int EPI>
 __global__ void __launch_bounds__(TC_THREADS, 1)
     tc_gemm_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUtensorMap tmB,
@@ -145,7 +159,9 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
     const int ob = offB ? __ldg(offB) : 0;
     int it = 0;  // k-blocks issued by this CTA (ring position across tiles)
     for (int t = t_first; t < num_tiles; t += t_step) {
-    const int m0 = (t / tiles_n) * TC_BM, n0 = (t % tiles_n) * BN;
+    int mt_, nt_;
+    tile_coords(t, tiles_m, tiles_n, mt_, nt_);
+    const int m0 = mt_ * TC_BM, n0 = nt_ * BN;
     for (int kb = 0; kb < num_kb; ++kb, ++it) {
       const int s = it % STAGES;
       const uint32_t ph = (it / STAGES) & 1;
@@ -215,7 +231,8 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
     int i = 0;
     for (int t = t_first; t < num_tiles; t += t_step, ++i) {
     const int acc = i & 1;
-    const int m_tile = t / tiles_n, n_tile = t % tiles_n;
+    int m_tile, n_tile;
+    tile_coords(t, tiles_m, tiles_n, m_tile, n_tile);
     const int m0 = m_tile * TC_BM, n0 = n_tile * BN;
     const int r = m0 + rl;
     const bool row_ok = r < ep.M;
@@ -464,7 +481,9 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
     cluster_sync_all();
     if (warp >= 4) {
       const int t = t_first;
-      const int m0 = (t / tiles_n) * TC_BM, n0 = (t % tiles_n) * BN;
+      int m_tile, n_tile;
+      tile_coords(t, tiles_m, tiles_n, m_tile, n_tile);
+      const int m0 = m_tile * TC_BM, n0 = n_tile * BN;
       const int tid = threadIdx.x - 128;  // 0..255
       const int rps = TC_BM / splits;
       const size_t tile_base = (size_t)t * splits * TC_BM * BN;
@@ -501,11 +520,11 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
         int lo, hi;
         bool own;
         if (!ep.transposed) {
-          own = (t % tiles_n) == 0;
+          own = n_tile == 0;
           lo = m0 + kz * rps + tid;
           hi = min(ep.M, m0 + (kz + 1) * rps);
         } else {
-          own = (t / tiles_n) == 0 && kz == 0;
+          own = m_tile == 0 && kz == 0;
           lo = n0 + tid;
           hi = min(ep.N, n0 + BN);
         }
