@@ -207,6 +207,10 @@ def main():
     ap.add_argument("--e2e-steps", type=int, default=3)
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-prof", action="store_true")
+    ap.add_argument("--ttt-epochs", type=int, default=40,
+                    help="epochs per algorithm for time-to-target (0 disables; N=1 only)")
+    ap.add_argument("--eta-grid", default="0.001,0.01,0.1,1",
+                    help="powers-of-10 learning-rate grid for time-to-target (PAPER.md L258)")
     args = ap.parse_args()
     cfg = CONFIGS[args.config]
     world = int(os.environ.get("WORLD_SIZE", "1"))
@@ -235,9 +239,9 @@ def main():
     import torch
     import torch.distributed as dist
     torch.cuda.set_device(local)
-    if world > 1:
-        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
     import paper_conf_ipps_marws21_b200 as hb
+    from paper_conf_ipps_marws21_b200 import dist as hbd
+    hbd.init("nccl", torch.device("cuda", local))
     from synth import init_params, params_to_flat
 
     # ---- data + model (resident in HBM before timing) ----
@@ -283,9 +287,8 @@ def main():
         pol = hb.Policy(kind=hb.HB_MINIBATCH, workers=specs, eta0=args.eta0, b0=args.b0)
     comm = None
     if world > 1:
-        uid = [hb.Comm.unique_id() if rank == 0 else None]
-        dist.broadcast_object_list(uid, src=0)
-        comm = hb.Comm(uid[0], world, rank, local)
+        uid = hbd.share_bytes(hb.Comm.unique_id() if rank == 0 else None)
+        comm = hb.Comm(uid, world, rank, local)
         model.merge_begin()
         pol.comm = comm
         pol.merges_per_epoch = args.merges
@@ -320,13 +323,10 @@ def main():
         share += st["updates"][0]
     launches = hb.kernel_launches() - l0
     clk = clocks.stop()
-    tot_ms = sum(ms)
-    t = torch.tensor([tot_ms], device=f"cuda:{local}")
-    s = torch.tensor([float(samples)], device=f"cuda:{local}")
-    if world > 1:
-        dist.all_reduce(t, op=dist.ReduceOp.MAX)
-        dist.all_reduce(s, op=dist.ReduceOp.SUM)
-    value = s.item() / (t.item() * 1e-3)
+    dev = torch.device("cuda", local)
+    t_max = hbd.reduce_scalar(sum(ms), "max", dev)            # device ms, max over ranks
+    s_tot = hbd.reduce_scalar(float(samples), "sum", dev)     # samples of all ranks
+    value = s_tot / (t_max * 1e-3)
 
     # ---- e2e: host (pinned) -> device copy of the step's inputs + the step + D2H of the
     #      trained parameters, through the public API, every step ----
@@ -348,12 +348,9 @@ def main():
         torch.cuda.synchronize()
         e2e_ms.append(e0.elapsed_time(e1))
         e2e_samples += st["total_samples"]
-    te = torch.tensor([sum(e2e_ms)], device=f"cuda:{local}")
-    se = torch.tensor([float(e2e_samples)], device=f"cuda:{local}")
-    if world > 1:
-        dist.all_reduce(te, op=dist.ReduceOp.MAX)
-        dist.all_reduce(se, op=dist.ReduceOp.SUM)
-    e2e_value = se.item() / (te.item() * 1e-3) if args.e2e_steps else None
+    te = hbd.reduce_scalar(sum(e2e_ms), "max", dev)
+    se = hbd.reduce_scalar(float(e2e_samples), "sum", dev)
+    e2e_value = se / (te * 1e-3) if args.e2e_steps else None
 
     # ---- per-kernel roofline: the same steps re-run with every hot-path launch bracketed by
     #      CUDA events on its own stream (hb_prof_enable; graphs off so each launch is visible).
@@ -368,6 +365,42 @@ def main():
             run_epoch()
         prof = hb.prof_read(reset=True)
         hb.prof_enable(False)
+
+    # ---- time to target loss (PAPER.md L258 methodology): every algorithm runs the same budget
+    #      of epochs from the same initial model; eta0 is chosen on a powers-of-10 grid by the
+    #      lowest loss reached by any algorithm; the minimum loss across algorithms is the basis
+    #      and the target is 1.1x that minimum ("90% of the minimum loss", L264).  Training time
+    #      only (loss evaluation excluded, L258); runs outside the throughput measurement.
+    ttt = None
+    if args.ttt_epochs > 0 and world == 1:
+        algos = {"minibatch": (hb.HB_MINIBATCH, [workers[0]], [hb.WorkerSpec(big_max, big_max, big_max)])}
+        if len(workers) > 1:
+            algos["adaptive"] = (hb.HB_ADAPTIVE, workers, specs)
+        curves = {}
+        for eta in [float(x) for x in args.eta_grid.split(",")]:
+            for name, (kind, ws_, sp) in algos.items():
+                model.set_params(params0)
+                p2 = hb.Policy(kind=kind, workers=sp, eta0=eta, b0=args.b0, eval_loss=True)
+                st = hb.hogbatch_run(ws_, p2, Xd, yd, epochs=args.ttt_epochs)
+                t_cum = np.cumsum(st["epoch_train_s"]).tolist()
+                curves[(eta, name)] = (t_cum, st["epoch_loss"])
+        def best(eta):
+            return min(min([l for l in curves[(eta, a)][1] if l == l] or [float("inf")]) for a in algos)
+        etas = sorted({e for e, _ in curves})
+        eta_star = min(etas, key=best)
+        l_min = best(eta_star)
+        target = 1.1 * l_min
+        res = {}
+        for a in algos:
+            t_cum, ls = curves[(eta_star, a)]
+            hit = next((t for t, l in zip(t_cum, ls) if l <= target), None)
+            res[a] = {"time_to_target_s": hit, "final_loss": ls[-1] if ls else None,
+                      "epoch_loss": [round(x, 5) for x in ls], "epoch_end_s": [round(x, 4) for x in t_cum]}
+        ttt = {"eta0": eta_star, "b0": args.b0, "epochs": args.ttt_epochs, "min_loss": l_min,
+               "target_loss": target, "grid": {str(e): round(best(e), 5) for e in etas}, "algorithms": res,
+               "method": "same epoch budget per algorithm, eta0 from the powers-of-10 grid with the lowest loss, "
+                         "target = 1.1 x min loss across algorithms, training time only (PAPER.md L258, L264)"}
+        model.set_params(params0)
 
     if rank == 0:
         peaks = load_peaks()
@@ -403,7 +436,7 @@ def main():
         line = {
             "metric": f"MLP SGD samples/sec ({'Adaptive Hogbatch' if args.policy == 'adaptive' else 'mini-batch'}, {args.config})",
             "value": value, "unit": "samples/s", "n_gpus": world, "steps": args.steps, "warmup": args.warmup,
-            "ms_per_step": t.item() / args.steps, "higher_is_better": True, "scaling": "weak", "vs_baseline": None,
+            "ms_per_step": t_max / args.steps, "higher_is_better": True, "scaling": "weak", "vs_baseline": None,
             "dtype": "bf16", "data": "synthetic",
             "config": {"workload": cfg["workload"] + (", Adaptive Hogbatch: large worker [%d, %d] init %d + small "
                                                       "worker [32, 2048] init 32, shared model (Hogwild)"
@@ -419,6 +452,7 @@ def main():
             "e2e": {"value": e2e_value, "unit": "samples/s", "h2d_bytes_per_step": h2d, "d2h_bytes_per_step": d2h},
             "gpu_launches": launches,
             "clocks": clk,
+            "time_to_target": ttt,
         }
         print(json.dumps(line), flush=True)
     if comm is not None:

@@ -220,6 +220,12 @@ int hb_bench_gemm(int32_t kind, int32_t M, int32_t N, int32_t K, int32_t iters, 
 /* tuning only: per-CTA phase timestamps (8 globaltimer ns values per CTA, cap entries) of one launch */
 int hb_bench_gemm_phases(int32_t kind, int32_t M, int32_t N, int32_t K, unsigned long long* host_ts, int64_t cap);
 
+/* Merge points of one rank for one epoch of served batch sizes batches[0..n):
+ * mid_epoch_out = merges due while serving, total_out = merges performed in the epoch (always
+ * merges_per_epoch, so ranks with different batch-size dynamics issue the same collectives). */
+int hb_merge_schedule(int64_t N, int32_t merges_per_epoch, const int32_t* batches, int64_t n_batches,
+                      int32_t* mid_epoch_out, int32_t* total_out);
+
 /* ---- multi-GPU replica merge over NCCL (future work L277) -------- */
 int hb_nccl_unique_id(uint8_t out[128]);
 int hb_comm_create(const uint8_t id[128], int32_t nranks, int32_t rank, int32_t device,

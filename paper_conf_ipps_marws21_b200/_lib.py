@@ -26,7 +26,7 @@ EXPORTS = ("hb_last_error", "hb_abi_version", "hb_device_ok", "mlp_create", "mlp
            "mlp_worker_destroy", "mlp_worker_stream", "mlp_step", "mlp_step_grads", "mlp_loss",
            "hb_schedule_trace", "hogbatch_run", "hb_nccl_unique_id", "hb_comm_create",
            "hb_comm_destroy", "hb_merge_begin", "hb_merge", "hb_kernel_launches", "hb_prof_enable",
-           "hb_prof_read", "hb_bench_gemm", "hb_bench_gemm_phases")
+           "hb_prof_read", "hb_bench_gemm", "hb_bench_gemm_phases", "hb_merge_schedule")
 PROF_CLASSES = ("fwd_gemm", "head_gemm", "softmax_xent", "dgrad_gemm", "wgrad_sgd_gemm", "bias_sgd", "other")
 
 
@@ -103,6 +103,7 @@ def load():
         "hb_prof_read": ([P(ProfEntry), I32, I32], C.c_int),
         "hb_bench_gemm": ([I32, I32, I32, I32, I32, P(F)], C.c_int),
         "hb_bench_gemm_phases": ([I32, I32, I32, I32, P(C.c_uint64), I64], C.c_int),
+        "hb_merge_schedule": ([I64, I32, P(I32), I64, P(I32), P(I32)], C.c_int),
     }
     for name, (args, res) in sig.items():
         fn = getattr(lib, name)
