@@ -193,6 +193,8 @@ static int launch_tc_bn(int bn, const CUtensorMap& ma, const CUtensorMap& mb, in
 
 // split-K factor of a dW GEMM (K = batch): enough CTAs to cover the 148 SMs, power of two
 // <= 8 (portable cluster size), at least one k-block per split
+static int choose_bn_base(int M, int N);
+
 static int env_int(const char* name, int dflt) {
   const char* v = getenv(name);
   return v && *v ? atoi(v) : dflt;
@@ -212,12 +214,13 @@ int choose_splits(int M, int N, int K, int bn) {
 static int choose_bn_wgrad(int M, int N, int K) {
   static const int forced = env_int("HB_WGRAD_BN", 0);
   if (forced) return forced;
-  int bn = choose_bn(M, N);
-  while (bn > 64 && (long)((M + TC_BM - 1) / TC_BM) * ((N + bn - 1) / bn) * 4 < 148 && K >= 2048) bn /= 2;
+  if (K < 2048) return choose_bn(M, N);  // short K: no split-K, spread tiles over the SMs
+  int bn = choose_bn_base(M, N);          // long K: split-K supplies the parallelism
+  while (bn > 64 && (long)((M + TC_BM - 1) / TC_BM) * ((N + bn - 1) / bn) * 4 < 148) bn /= 2;
   return bn;
 }
 
-int choose_bn(int M, int N) {
+static int choose_bn_base(int M, int N) {
   if (N <= 16) return 16;
   if (N <= 32) return 32;
   if (N <= 64) return 64;
@@ -225,6 +228,15 @@ int choose_bn(int M, int N) {
   const long mt = (M + TC_BM - 1) / TC_BM;
   if (mt * ((N + 255) / 256) >= 148) return 256;
   return 128;
+}
+
+// Tile width: the base rule, narrowed while the grid would leave most SMs idle (small batches:
+// M = b <= a few hundred rows gives 1-2 row tiles; narrower tiles spread the epilogue)
+int choose_bn(int M, int N) {
+  int bn = choose_bn_base(M, N);
+  const long mt = (M + TC_BM - 1) / TC_BM;
+  while (bn > 32 && mt * ((N + bn - 1) / bn) < 64) bn /= 2;
+  return bn;
 }
 
 // One tcgen05 GEMM launch.  A is [M x K] (K-major) or stored [K x M] (MN-major); B is [N x K]
