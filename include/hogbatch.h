@@ -158,6 +158,12 @@ int mlp_set_params(hb_model* m, const float* host_src, int64_t n);
  * be NULL (the worker creates its own non-blocking stream) or a borrowed cudaStream_t. */
 int mlp_worker_create(hb_model* m, int32_t max_batch, int32_t replica, void* cuda_stream,
                       hb_worker** out);
+/* Nested worker: the GPU form of Algorithm 2's CPU worker [L224-L235].  Each ExecuteWork(B) is
+ * split into t contiguous sub-batches (the first b mod t get ceil(b/t) rows) run concurrently on
+ * t internal streams, each updating the shared model in place (Hogwild [L229-L232]) with
+ * lr * size/b; credit it with incr = t*beta in hb_worker_policy [L234, L238].  t >= 1,
+ * max_batch >= t.  In deterministic mode the sub-batches run in order. */
+int mlp_worker_create_nested(hb_model* m, int32_t max_batch, int32_t t, void* cuda_stream, hb_worker** out);
 int mlp_worker_destroy(hb_worker* w);
 /* cudaStream_t of the worker (borrowed) */
 void* mlp_worker_stream(hb_worker* w);

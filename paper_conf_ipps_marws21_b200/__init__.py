@@ -103,11 +103,16 @@ class MLP:
 class Worker:
     """A GPU worker (§V.A): activation scratch for max_batch rows and a stream."""
 
-    def __init__(self, model: MLP, max_batch: int, stream=None):
+    def __init__(self, model: MLP, max_batch: int, stream=None, sub_batches: int = 1):
+        """sub_batches = t > 1 creates a nested worker (Alg. 2's CPU worker, L224-L235)."""
         self.model = model
         self.max_batch = max_batch
+        self.sub_batches = sub_batches
         h = C.c_void_p()
-        _check(lib.mlp_worker_create(model.h, max_batch, 0, _stream_ptr(stream), C.byref(h)))
+        if sub_batches > 1:
+            _check(lib.mlp_worker_create_nested(model.h, max_batch, sub_batches, _stream_ptr(stream), C.byref(h)))
+        else:
+            _check(lib.mlp_worker_create(model.h, max_batch, 0, _stream_ptr(stream), C.byref(h)))
         self.h = h
 
     @property

@@ -26,7 +26,8 @@ EXPORTS = ("hb_last_error", "hb_abi_version", "hb_device_ok", "mlp_create", "mlp
            "mlp_worker_destroy", "mlp_worker_stream", "mlp_step", "mlp_step_grads", "mlp_loss",
            "hb_schedule_trace", "hogbatch_run", "hb_nccl_unique_id", "hb_comm_create",
            "hb_comm_destroy", "hb_merge_begin", "hb_merge", "hb_kernel_launches", "hb_prof_enable",
-           "hb_prof_read", "hb_bench_gemm", "hb_bench_gemm_phases", "hb_merge_schedule")
+           "hb_prof_read", "hb_bench_gemm", "hb_bench_gemm_phases", "hb_merge_schedule",
+           "mlp_worker_create_nested")
 PROF_CLASSES = ("fwd_gemm", "head_gemm", "softmax_xent", "dgrad_gemm", "wgrad_sgd_gemm", "bias_sgd", "other")
 
 
@@ -87,6 +88,7 @@ def load():
         "mlp_set_params": ([VP, P(F), I64], C.c_int),
         "mlp_worker_create": ([VP, I32, I32, VP, P(VP)], C.c_int),
         "mlp_worker_destroy": ([VP], C.c_int),
+        "mlp_worker_create_nested": ([VP, I32, I32, VP, P(VP)], C.c_int),
         "mlp_worker_stream": ([VP], VP),
         "mlp_step": ([VP, VP, I64, I32, VP, I32, F, P(F)], C.c_int),
         "mlp_step_grads": ([VP, VP, I64, I32, VP, I32, P(F), I64, P(F)], C.c_int),

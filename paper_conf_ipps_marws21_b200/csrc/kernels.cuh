@@ -134,7 +134,7 @@ __global__ void __launch_bounds__(256) simt_gemm_kernel(const TA* __restrict__ A
 // ---------------------------------------------------------------------------------------
 // deterministic sum of per-row losses into one double (single block, fixed order)
 // ---------------------------------------------------------------------------------------
-static __global__ void sum_rows_kernel(const float* __restrict__ v, int n, double* out, int accumulate_slot) {
+static __global__ void sum_rows_kernel(const float* __restrict__ v, int n, double* out, int slot, int accumulate = 0) {
   __shared__ double red[1024];
   double s = 0.0;
   for (int i = threadIdx.x; i < n; i += blockDim.x) s += (double)v[i];
@@ -144,7 +144,7 @@ static __global__ void sum_rows_kernel(const float* __restrict__ v, int n, doubl
     if (threadIdx.x < w) red[threadIdx.x] += red[threadIdx.x + w];
     __syncthreads();
   }
-  if (threadIdx.x == 0) out[accumulate_slot] = red[0];
+  if (threadIdx.x == 0) out[slot] = (accumulate ? out[slot] : 0.0) + red[0];
 }
 
 // bf16 shadow := RNE(fp32 master) over the whole flat parameter buffer

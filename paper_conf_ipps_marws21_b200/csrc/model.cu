@@ -711,6 +711,52 @@ int step_graph(hb_worker* w, const void* X, int64_t ldx, int64_t x_rows, const i
   return HB_OK;
 }
 
+int worker_execute(hb_worker* w, const void* X, int64_t ldx, int32_t xdt, int64_t x_rows, const int32_t* y,
+                   int64_t off, int b, float lr, bool graphs, bool serial, double* loss_dst) {
+  const size_t xes = xdt == HB_BF16 ? 2 : 4;
+  auto xrow = [&](int64_t o) { return static_cast<const char*>(X) + o * ldx * xes; };
+  if (w->subs.empty()) {
+    int rc = graphs ? step_graph(w, X, ldx, x_rows, y, off, b, lr)
+                    : run_step(w, xrow(off), ldx, xdt, b, y + off, nullptr, b, lr, false, w->stream);
+    if (!rc && loss_dst) sum_rows_into(w, b, loss_dst, w->stream, false);
+    return rc;
+  }
+  const int t = (int)w->subs.size();
+  const int base = b / t, extra = b % t;
+  if (!serial) HB_CUDA_TRY(cudaEventRecord(w->ev_fork, w->stream));
+  int64_t o = off;
+  for (int i = 0; i < t; ++i) {
+    const int sz = base + (i < extra ? 1 : 0);
+    if (sz == 0) continue;
+    hb_worker* sw = w->subs[i];
+    const float lr_i = lr * (float)sz / (float)b;  // eta proportional to the (sub-)batch size (L179)
+    int rc;
+    if (serial) {
+      rc = run_step(sw, xrow(o), ldx, xdt, sz, y + o, nullptr, sz, lr_i, false, w->stream);
+      if (!rc && loss_dst) sum_rows_into(sw, sz, loss_dst, w->stream, i > 0);
+    } else {
+      HB_CUDA_TRY(cudaStreamWaitEvent(sw->stream, w->ev_fork, 0));
+      rc = graphs ? step_graph(sw, X, ldx, x_rows, y, o, sz, lr_i)
+                  : run_step(sw, xrow(o), ldx, xdt, sz, y + o, nullptr, sz, lr_i, false, sw->stream);
+      HB_CUDA_TRY(cudaEventRecord(w->ev_join[i], sw->stream));
+      HB_CUDA_TRY(cudaStreamWaitEvent(w->stream, w->ev_join[i], 0));
+    }
+    if (rc) return rc;
+    o += sz;
+  }
+  if (!serial && loss_dst) {  // after the join: the sub-batch losses in sub-worker order
+    o = off;
+    bool first = true;
+    for (int i = 0; i < t; ++i) {
+      const int sz = base + (i < extra ? 1 : 0);
+      if (sz == 0) continue;
+      sum_rows_into(w->subs[i], sz, loss_dst, w->stream, !first);
+      first = false;
+    }
+  }
+  return HB_OK;
+}
+
 static int check_step_args(hb_worker* w, const void* X, int64_t ldx, int32_t xdt, const int32_t* y, int32_t batch) {
   if (!w) return fail(HB_EINVAL, "null worker");
   hb_model* m = w->m;
@@ -726,9 +772,9 @@ static int check_step_args(hb_worker* w, const void* X, int64_t ldx, int32_t xdt
   return HB_OK;
 }
 
-void sum_rows_into(hb_worker* w, int b, double* dst, cudaStream_t s) {
+void sum_rows_into(hb_worker* w, int b, double* dst, cudaStream_t s, bool accumulate) {
   Prof pr(HB_PROF_OTHER, s);
-  sum_rows_kernel<<<1, 1024, 0, s>>>(w->row_loss, b, dst, 0);
+  sum_rows_kernel<<<1, 1024, 0, s>>>(w->row_loss, b, dst, 0, accumulate ? 1 : 0);
   pr.done(1, 0.0, 4.0 * b);
 }
 
@@ -942,6 +988,11 @@ int mlp_worker_destroy(hb_worker* w) {
   if (!w) return HB_OK;
   cudaSetDevice(w->m->device);
   cudaStreamSynchronize(w->stream);
+  for (hb_worker* sw : w->subs) mlp_worker_destroy(sw);
+  w->subs.clear();
+  if (w->ev_fork) cudaEventDestroy(w->ev_fork);
+  for (cudaEvent_t e : w->ev_join) cudaEventDestroy(e);
+  w->ev_join.clear();
   free_worker_buffers(w);
   if (w->own_stream) cudaStreamDestroy(w->stream);
   delete w;
@@ -950,11 +1001,45 @@ int mlp_worker_destroy(hb_worker* w) {
 
 void* mlp_worker_stream(hb_worker* w) { return w ? (void*)w->stream : nullptr; }
 
+int mlp_worker_create_nested(hb_model* m, int32_t max_batch, int32_t t, void* cuda_stream, hb_worker** out) {
+  HB_CHECK_ARG(m && out, "null arg");
+  *out = nullptr;
+  HB_CHECK_ARG(t >= 1 && max_batch >= t, "need 1 <= t <= max_batch");
+  hb_worker* w = nullptr;
+  int rc = mlp_worker_create(m, 1, 0, cuda_stream, &w);  // parent: stream + events only
+  if (rc) return rc;
+  w->max_b = max_batch;
+  const int sub_max = (max_batch + t - 1) / t;
+  for (int i = 0; i < t; ++i) {
+    hb_worker* sw = nullptr;
+    rc = mlp_worker_create(m, sub_max, 0, nullptr, &sw);
+    if (rc) {
+      mlp_worker_destroy(w);
+      return rc;
+    }
+    w->subs.push_back(sw);
+    cudaEvent_t e;
+    cudaEventCreateWithFlags(&e, cudaEventDisableTiming);
+    w->ev_join.push_back(e);
+  }
+  cudaEventCreateWithFlags(&w->ev_fork, cudaEventDisableTiming);
+  *out = w;
+  return HB_OK;
+}
+
 int mlp_step(hb_worker* w, const void* X, int64_t ldx, int32_t x_dtype, const int32_t* y, int32_t batch, float lr,
              float* loss_out) {
   int rc = check_step_args(w, X, ldx, x_dtype, y, batch);
   if (rc) return rc;
   HB_CUDA_TRY(cudaSetDevice(w->m->device));
+  if (!w->subs.empty()) {  // nested worker: t concurrent sub-batches
+    rc = worker_execute(w, X, ldx, x_dtype, batch, y, 0, batch, lr, false, false, loss_out ? w->dsum : nullptr);
+    if (rc || !loss_out) return rc;
+    HB_CUDA_TRY(cudaMemcpyAsync(w->h_dsum, w->dsum, sizeof(double), cudaMemcpyDeviceToHost, w->stream));
+    HB_CUDA_TRY(cudaStreamSynchronize(w->stream));
+    *loss_out = (float)(w->h_dsum[0] / (double)batch);
+    return HB_OK;
+  }
   rc = run_step(w, X, ldx, x_dtype, batch, y, nullptr, batch, lr, false, w->stream);
   if (rc) return rc;
   if (loss_out) return finish_loss(w, batch, loss_out, w->stream);
@@ -966,6 +1051,7 @@ int mlp_step_grads(hb_worker* w, const void* X, int64_t ldx, int32_t x_dtype, co
   int rc = check_step_args(w, X, ldx, x_dtype, y, batch);
   if (rc) return rc;
   hb_model* m = w->m;
+  if (!w->subs.empty()) return fail(HB_EUNSUPPORTED, "mlp_step_grads on a nested worker");
   int64_t need;
   mlp_num_params(m, &need);
   HB_CHECK_ARG(host_grads && n == need, "n must equal mlp_num_params");

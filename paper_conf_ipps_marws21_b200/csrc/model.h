@@ -78,6 +78,11 @@ struct hb_worker {
   double* h_dsum = nullptr;     // pinned
   float* grads = nullptr;       // mlp_step_grads output (flat padded layout)
   float* ws = nullptr;          // split-K partial tiles of the dW GEMMs (148 x 128 x 256 fp32)
+  // nested worker (Alg. 2 "CPU worker", L224-L235): t sub-workers run the sub-batches of one
+  // ExecuteWork concurrently, each updating the shared model in place
+  std::vector<hb_worker*> subs;
+  cudaEvent_t ev_fork = nullptr;
+  std::vector<cudaEvent_t> ev_join;
 };
 
 namespace hb {
@@ -90,8 +95,15 @@ int run_step(hb_worker* w, const void* X, int64_t ldx, int32_t xdt, int64_t x_ro
 int step_graph(hb_worker* w, const void* X, int64_t ldx, int64_t x_rows, const int32_t* y, int64_t off, int b,
                float lr);
 void clear_graphs(hb_worker* w);
+// One ExecuteWork(B) of a worker on rows [off, off + b) of the dataset (X, y with x_rows rows):
+// a plain worker runs one SGD step; a nested worker splits B into its t sub-batches (the first
+// b mod t get ceil(b/t) rows, R6) with lr scaled to each sub-batch (lr * size / b),
+// concurrently on the sub-workers' streams (serial = in order on w->stream, deterministic).
+// If loss_dst != nullptr the summed per-row losses of the batch are written to *loss_dst (device).
+int worker_execute(hb_worker* w, const void* X, int64_t ldx, int32_t xdt, int64_t x_rows, const int32_t* y,
+                   int64_t off, int b, float lr, bool graphs, bool serial, double* loss_dst);
 bool prof_enabled();
 int finish_loss(hb_worker* w, int b, float* loss_out, cudaStream_t s);
 // enqueue sum of the last step's per-row losses into *dst (device double)
-void sum_rows_into(hb_worker* w, int b, double* dst, cudaStream_t s);
+void sum_rows_into(hb_worker* w, int b, double* dst, cudaStream_t s, bool accumulate = false);
 }  // namespace hb

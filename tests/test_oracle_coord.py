@@ -203,3 +203,26 @@ def test_serial_run_equals_manual_sgd_loop():
     assert losses == exp_l
     for (a, b), (c, d) in zip(got, P):
         assert np.array_equal(a, c) and np.array_equal(b, d)
+
+
+def test_nested_split_sizes_and_t1_reduces_to_serial():
+    # R6 reading of Alg. 2 line 1 [L229]
+    assert serial.split_sizes(10, 4) == [3, 3, 2, 2]
+    assert serial.split_sizes(8, 4) == [2, 2, 2, 2]
+    assert sum(serial.split_sizes(1000, 56)) == 1000
+    rng = np.random.default_rng(2)
+    dims = [5, 4, 3]
+    params = [(rng.standard_normal((dims[l], dims[l - 1])), np.zeros(dims[l])) for l in (1, 2)]
+    X = rng.standard_normal((64, 5))
+    y = rng.integers(0, 3, 64)
+    recs = coord.run(Policy(kind=MINIBATCH, eta0=0.2, b0=8, workers=[WorkerSpec(16, 16, 16)]), 64, 1)
+    a, la = serial.run_trace(params, X, y, recs)
+    b, lb = serial.run_trace_nested(params, X, y, recs, [1])
+    assert la == lb and all(np.array_equal(p[0], q[0]) for p, q in zip(a, b))
+    # t = 2: each batch = two half-size SGD steps with half the learning rate
+    c, lc = serial.run_trace_nested(params, X, y, recs, [2])
+    P = params
+    for s in range(0, 64, 16):
+        P, _ = mlp64.sgd_step(P, X[s:s + 8], y[s:s + 8], 0.2 * 16 / 8 * 0.5)
+        P, _ = mlp64.sgd_step(P, X[s + 8:s + 16], y[s + 8:s + 16], 0.2 * 16 / 8 * 0.5)
+    np.testing.assert_allclose(c[0][0], P[0][0], atol=1e-14)
