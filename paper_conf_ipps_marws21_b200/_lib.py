@@ -9,7 +9,7 @@ import ctypes as C
 import os
 
 HERE = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(HERE, "libhogbatch.so")
+LIB_PATH = os.environ.get("HB_LIB") or os.path.join(HERE, "libhogbatch.so")  # HB_LIB: A/B builds
 
 HB_OK, HB_EINVAL, HB_ENOMEM, HB_ECUDA, HB_ENCCL, HB_ESTATE, HB_EUNSUPPORTED = 0, -1, -2, -3, -4, -5, -6
 HB_SIGMOID = 0

@@ -127,10 +127,21 @@ static int make_map(CUtensorMap* out, const void* base, uint64_t inner, uint64_t
 static std::mutex g_attr_mu;
 static std::set<std::pair<const void*, int>> g_attr_done;
 
+// bf16 output map for the TMA-store epilogue: [rows x cols] row stride ld elements, box 64 x 128
+static int make_out_map(CUtensorMap* out, const void* base, int64_t cols, int64_t rows, int64_t ld) {
+  return make_map(out, base, cols, rows, ld * 2, 64, TC_BM);
+}
+
 template <int BN, bool A_MN, bool B_MN, int EPI>
 static int launch_tc(const CUtensorMap& ma, const CUtensorMap& mb, int M, int N, int K, const int* offA,
                      const int* offB, const EpiArgs& ep, cudaStream_t s, int splits = 1) {
-  using Cfg = TcCfg<BN, B_MN>;
+  using Cfg = TcCfg<BN, B_MN, EPI>;
+  CUtensorMap mo0 = ma, mo1 = ma;  // unused unless the epilogue stages its outputs for TMA stores
+  if (TmaOut<BN, EPI>::on) {
+    int rc = make_out_map(&mo0, ep.out0, N, M, ep.ld0 > 0 ? ep.ld0 : round_up(N, 8));
+    if (!rc && EPI == EPI_FWD_SIG && ep.out1) rc = make_out_map(&mo1, ep.out1, N, M, ep.ld1);
+    if (rc) return rc;
+  }
   auto kern = tc_gemm_kernel<BN, A_MN, B_MN, EPI>;
   int dev = 0;
   cudaGetDevice(&dev);
@@ -174,7 +185,7 @@ static int launch_tc(const CUtensorMap& ma, const CUtensorMap& mb, int M, int N,
   }
   cfg.attrs = attr;
   cfg.numAttrs = na;
-  HB_CUDA_TRY(cudaLaunchKernelEx(&cfg, kern, ma, mb, K, offA, offB, ep));
+  HB_CUDA_TRY(cudaLaunchKernelEx(&cfg, kern, ma, mb, mo0, mo1, K, offA, offB, ep));
   HB_CUDA_TRY(cudaGetLastError());
   return HB_OK;
 }

@@ -31,21 +31,38 @@ namespace hb {
 
 constexpr int TC_BM = 128;
 constexpr int TC_BK = 64;
-constexpr int TC_THREADS = 384;  // 4 control warps + 8 epilogue warps
+#ifndef HB_EPI_WARPS
+#define HB_EPI_WARPS 8
+#endif
+constexpr int TC_EPI_WARPS = HB_EPI_WARPS;         // epilogue warps: 4 TMEM lane quadrants x column parts
+constexpr int TC_EPI_THREADS = TC_EPI_WARPS * 32;
+constexpr int TC_EPI_PARTS = TC_EPI_WARPS / 4;
+constexpr int TC_THREADS = 128 + TC_EPI_THREADS;   // 4 control warps + the epilogue warps
 
-template <int BN, bool B_MN>
+// Epilogues whose bf16 outputs are staged in swizzled shared memory and written with TMA bulk
+// stores (full 128-byte lines instead of one 16-byte piece of 32 different rows per warp store)
+template <int BN, int EPI>
+struct TmaOut {
+  static constexpr bool on = (EPI == EPI_FWD_SIG || EPI == EPI_DGRAD_SIG) && (BN == 64 || BN == 128);
+  static constexpr int NBOX = BN / 64;                     // 64-column boxes per output
+  static constexpr int NOUT = EPI == EPI_FWD_SIG ? 2 : 1;  // H and S, or dZ
+  static constexpr int BYTES = on ? NOUT * NBOX * TC_BM * 128 : 0;
+};
+
+template <int BN, bool B_MN, int EPI = EPI_WGRAD_SGD>
 struct TcCfg {
   static constexpr int A_BYTES = TC_BM * TC_BK * 2;                     // 16 KB
   static constexpr int B_ROWS = B_MN ? (BN < 64 ? 64 : BN) : BN;        // MN-major loads 64-wide boxes
   static constexpr int B_BYTES = B_ROWS * TC_BK * 2;
   static constexpr int STAGE_BYTES = A_BYTES + B_BYTES;
-  static constexpr int STAGES_RAW = (192 * 1024) / STAGE_BYTES;
+  static constexpr int OUT_BYTES = TmaOut<BN, EPI>::BYTES;
+  static constexpr int STAGES_RAW = (192 * 1024 - OUT_BYTES) / STAGE_BYTES;
   static constexpr int STAGES = STAGES_RAW > 8 ? 8 : STAGES_RAW;
   static constexpr int TMEM_COLS = 2 * BN < 32 ? 32 : 2 * BN;          // two accumulators (double buffer)
-  static constexpr int SMEM_BYTES = STAGES * STAGE_BYTES + 1024 /*align*/ + 256 /*barriers*/;
+  static constexpr int SMEM_BYTES = STAGES * STAGE_BYTES + OUT_BYTES + 1024 /*align*/ + 256 /*barriers*/;
 };
 
-__device__ __forceinline__ void epi_bar_sync() { asm volatile("bar.sync 1, 256;" ::: "memory"); }
+__device__ __forceinline__ void epi_bar_sync() { asm volatile("bar.sync 1, %0;" ::"n"(TC_EPI_THREADS) : "memory"); }
 
 // Column sums of a 32-row x 16-column register tile (one row per lane) in 16 shuffles
 // (reduce-scatter): afterwards lane L holds the total of column
@@ -93,15 +110,29 @@ __device__ __forceinline__ void tile_coords(int t, int tiles_m, int tiles_n, int
   n_tile = r / gm;
 }
 
+// Write 16 bf16 values (8 packed words) of tile row rl, tile columns c..c+15 into staging output o
+// (boxes of 128 rows x 64 columns, 128-byte rows, 16-byte chunks XOR-swizzled by row % 8 — the
+// TMA SWIZZLE_128B layout, which also makes these per-row writes bank-conflict free).
+template <int NBOX>
+__device__ __forceinline__ void stage16(uint8_t* sout, int o, int rl, int c, const uint32_t* p) {
+  const int box = c >> 6, j0 = (c & 63) >> 3;
+  uint8_t* row = sout + ((size_t)(o * NBOX + box) * TC_BM + rl) * 128;
+  *reinterpret_cast<uint4*>(row + ((j0 ^ (rl & 7)) << 4)) = make_uint4(p[0], p[1], p[2], p[3]);
+  *reinterpret_cast<uint4*>(row + (((j0 + 1) ^ (rl & 7)) << 4)) = make_uint4(p[4], p[5], p[6], p[7]);
+}
+
 template <int BN, bool A_MN, bool B_MN, int EPI>
 __global__ void __launch_bounds__(TC_THREADS, 1)
     tc_gemm_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUtensorMap tmB,
+                   const __grid_constant__ CUtensorMap tmO0, const __grid_constant__ CUtensorMap tmO1,
                    int K, const int* __restrict__ offA, const int* __restrict__ offB, EpiArgs ep) {
-  using Cfg = TcCfg<BN, B_MN>;
+  using Cfg = TcCfg<BN, B_MN, EPI>;
+  using TO = TmaOut<BN, EPI>;
   constexpr int STAGES = Cfg::STAGES;
   extern __shared__ uint8_t smem_raw[];
   uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
-  uint64_t* full_bar = reinterpret_cast<uint64_t*>(smem + STAGES * Cfg::STAGE_BYTES);
+  uint8_t* sout = smem + STAGES * Cfg::STAGE_BYTES;  // TMA-store staging [NOUT][NBOX][128 rows x 128 B]
+  uint64_t* full_bar = reinterpret_cast<uint64_t*>(sout + Cfg::OUT_BYTES);
   uint64_t* empty_bar = full_bar + STAGES;
   uint64_t* tmem_full_bar = empty_bar + STAGES;   // [2]: accumulator a ready (MMA -> epilogue)
   uint64_t* tmem_empty_bar = tmem_full_bar + 2;    // [2]: accumulator a drained (epilogue -> MMA)
@@ -138,7 +169,7 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
     }
     for (int a = 0; a < 2; ++a) {
       mbar_init(&tmem_full_bar[a], 1);
-      mbar_init(&tmem_empty_bar[a], 8);  // one arrive per epilogue warp
+      mbar_init(&tmem_empty_bar[a], TC_EPI_WARPS);  // one arrive per epilogue warp
     }
     fence_barrier_init();
   }
@@ -222,12 +253,13 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
     // ===== epilogue (8 warps): TMEM -> registers -> fused epilogue -> global =====
     // warp w reads TMEM lanes 32*(w%4).. (tile rows) and handles column half h = (w-4)/4
     const int q = warp & 3;
-    const int h = (warp - 4) >> 2;
+    const int h = (warp - 4) >> 2;  // column part 0..TC_EPI_PARTS-1
     const int et = threadIdx.x - 128;  // 0..255
     const int rl = q * 32 + lane;      // row within the tile
-    constexpr int HALF = BN >= 32 ? BN / 2 : BN;  // columns per warp
-    const bool active = BN >= 32 || h == 0;
-    const int c_lo = BN >= 32 ? h * HALF : 0;
+    constexpr int NP = BN / 16 < TC_EPI_PARTS ? BN / 16 : TC_EPI_PARTS;  // parts with columns
+    constexpr int HALF = BN / NP;                                        // columns per warp
+    const bool active = h < NP;
+    const int c_lo = active ? h * HALF : 0;
     int i = 0;
     for (int t = t_first; t < num_tiles; t += t_step, ++i) {
     const int acc = i & 1;
@@ -241,7 +273,7 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
 
     // stage the bias of the tile's columns in shared memory while the mainloop runs
     if (EPI == EPI_FWD_SIG || EPI == EPI_FWD_LOGITS || EPI == EPI_HEAD_XENT) {
-      for (int c = et; c < BN; c += 256) sb[c] = n0 + c < ep.N ? ep.bias[n0 + c] : 0.f;
+      for (int c = et; c < BN; c += TC_EPI_THREADS) sb[c] = n0 + c < ep.N ? ep.bias[n0 + c] : 0.f;
     }
     // DGRAD: prefetch this thread's row of sigma'(Z) (the S stash) for all of its columns
     constexpr int NCH = (HALF + 15) / 16;
@@ -258,7 +290,8 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
         }
       }
     }
-    epi_bar_sync();  // sbias visible; previous tile's partial sums consumed
+    if (TO::on && et == 0) tma_store_wait_read();  // staging buffer of the previous tile free
+    epi_bar_sync();  // sbias visible; previous tile's partial sums consumed; staging free
     if (dbg && et == 0 && i == 0) dbg[4] = gtimer();
     mbar_wait(&tmem_full_bar[acc], (i >> 1) & 1);
     tc_fence_after();
@@ -344,11 +377,16 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
                   v[8 + 2 * qq] *= b2.x;
                   v[8 + 2 * qq + 1] *= b2.y;
                 }
-                uint4* D = reinterpret_cast<uint4*>(static_cast<__nv_bfloat16*>(ep.out0) + (int64_t)r * ep.ld0 + nc);
-                D[0] = make_uint4(pack_bf16x2(v[0], v[1]), pack_bf16x2(v[2], v[3]), pack_bf16x2(v[4], v[5]),
-                                  pack_bf16x2(v[6], v[7]));
-                D[1] = make_uint4(pack_bf16x2(v[8], v[9]), pack_bf16x2(v[10], v[11]), pack_bf16x2(v[12], v[13]),
-                                  pack_bf16x2(v[14], v[15]));
+                uint32_t pk[8];
+#pragma unroll
+                for (int qq = 0; qq < 8; ++qq) pk[qq] = pack_bf16x2(v[2 * qq], v[2 * qq + 1]);
+                if (TO::on) {
+                  stage16<TO::NBOX>(sout, 0, rl, c, pk);
+                } else {
+                  uint4* D = reinterpret_cast<uint4*>(static_cast<__nv_bfloat16*>(ep.out0) + (int64_t)r * ep.ld0 + nc);
+                  D[0] = make_uint4(pk[0], pk[1], pk[2], pk[3]);
+                  D[1] = make_uint4(pk[4], pk[5], pk[6], pk[7]);
+                }
               } else {
                 const __nv_bfloat16* S = static_cast<const __nv_bfloat16*>(ep.aux) + (int64_t)r * ep.ldaux;
                 __nv_bfloat16* D = static_cast<__nv_bfloat16*>(ep.out0) + (int64_t)r * ep.ld0;
@@ -356,10 +394,16 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
                 for (int j = 0; j < 16; ++j) {
                   if (nc + j < ep.N) {
                     v[j] *= __bfloat162float(S[nc + j]);
-                    D[nc + j] = __float2bfloat16_rn(v[j]);
+                    if (!TO::on) D[nc + j] = __float2bfloat16_rn(v[j]);
                   } else {
                     v[j] = 0.f;
                   }
+                }
+                if (TO::on) {  // columns >= N are clipped by the TMA store
+                  uint32_t pk[8];
+#pragma unroll
+                  for (int qq = 0; qq < 8; ++qq) pk[qq] = pack_bf16x2(v[2 * qq], v[2 * qq + 1]);
+                  stage16<TO::NBOX>(sout, 0, rl, c, pk);
                 }
               }
             } else {
@@ -386,6 +430,19 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
             }
 #pragma unroll
             for (int qq = 0; qq < 4; ++qq) wsp[qq] = make_float4(v[4 * qq], v[4 * qq + 1], v[4 * qq + 2], v[4 * qq + 3]);
+          } else if (TO::on && EPI == EPI_FWD_SIG) {
+            // all rows / columns staged; rows >= M and columns >= N are clipped by the TMA store
+            uint32_t hp[8], sp[8];
+#pragma unroll
+            for (int qq = 0; qq < 8; ++qq) {
+              float h0, d0, h1, d1;
+              sigmoid_d(v[2 * qq] + sb[c + 2 * qq], h0, d0);
+              sigmoid_d(v[2 * qq + 1] + sb[c + 2 * qq + 1], h1, d1);
+              hp[qq] = pack_bf16x2(h0, h1);
+              sp[qq] = pack_bf16x2(d0, d1);
+            }
+            stage16<TO::NBOX>(sout, 0, rl, c, hp);
+            if (ep.out1) stage16<TO::NBOX>(sout, 1, rl, c, sp);
           } else if (row_ok) {
             if (EPI == EPI_FWD_SIG && ep.ld0 < 0) {  // tuning probe: epilogue math, no stores
               float acc = 0.f;
@@ -443,9 +500,23 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
           }
         }
       }
-      if (EPI == EPI_DGRAD_SIG && ep.bpart_out) {
+      if (TO::on) {  // staged tile complete -> one thread issues the bulk stores
+        fence_proxy_async();
         epi_bar_sync();
-        for (int cc = et; cc < BN && n0 + cc < ep.N; cc += 256)
+        if (et == 0) {
+#pragma unroll
+          for (int o = 0; o < TO::NOUT; ++o) {
+            if (o == 1 && !ep.out1) continue;
+#pragma unroll
+            for (int bx = 0; bx < TO::NBOX; ++bx)
+              tma_store_2d(o == 0 ? &tmO0 : &tmO1, sout + (size_t)(o * TO::NBOX + bx) * TC_BM * 128, n0 + bx * 64, m0);
+          }
+          tma_store_commit();
+        }
+      }
+      if (EPI == EPI_DGRAD_SIG && ep.bpart_out) {
+        if (!TO::on) epi_bar_sync();
+        for (int cc = et; cc < BN && n0 + cc < ep.N; cc += TC_EPI_THREADS)
           ep.bpart_out[(int64_t)m_tile * ep.ldp + n0 + cc] =
               (red[cc] + red[BN + cc]) + (red[2 * BN + cc] + red[3 * BN + cc]);
       }
@@ -457,7 +528,7 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
         const int lo = !ep.transposed ? m0 + et : n0 + et;
         const int hi = !ep.transposed ? min(ep.M, m0 + TC_BM) : min(ep.N, n0 + BN);
         if (own)
-          for (int bi = lo; bi < hi; bi += 256) {
+          for (int bi = lo; bi < hi; bi += TC_EPI_THREADS) {
             float sdb = 0.f;
             for (int t = 0; t < ep.n_mtiles; ++t) sdb += ep.bpart_in[(int64_t)t * ep.ldp + bi];
             if (EPI == EPI_WGRAD_SGD)
@@ -487,7 +558,7 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
       const int tid = threadIdx.x - 128;  // 0..255
       const int rps = TC_BM / splits;
       const size_t tile_base = (size_t)t * splits * TC_BM * BN;
-      for (int e = tid * 4; e < rps * BN; e += 256 * 4) {
+      for (int e = tid * 4; e < rps * BN; e += TC_EPI_THREADS * 4) {
         const int rloc = kz * rps + e / BN, col = e % BN;
         float4 acc = make_float4(0.f, 0.f, 0.f, 0.f);
         for (int sp = 0; sp < splits; ++sp) {
@@ -529,7 +600,7 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
           hi = min(ep.N, n0 + BN);
         }
         if (own)
-          for (int bi = lo; bi < hi; bi += 256) {
+          for (int bi = lo; bi < hi; bi += TC_EPI_THREADS) {
             float sdb = 0.f;
             for (int t = 0; t < ep.n_mtiles; ++t) sdb += ep.bpart_in[(int64_t)t * ep.ldp + bi];
             if (EPI == EPI_WGRAD_SGD)
@@ -541,6 +612,7 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
     }
   }
 
+  if (TO::on && threadIdx.x == 128) tma_store_wait_all();  // bulk stores complete before exit
   if (dbg && threadIdx.x == 128) dbg[6] = gtimer();
   tc_fence_before();
   __syncthreads();
