@@ -44,6 +44,14 @@ struct EpiArgs {
   const int* yoff;      // device row offset of the batch (graph replay), nullable
   float* row_loss;      // per-row cross-entropy
   float inv_b;          // 1 / b (gradient of the batch MEAN loss)
+  // fused dX of the output layer (HEAD_XENT, nullable): dZ_{L-1} = (dZ_L W_L) * S_{L-1}
+  const float* w_head;  // fp32 master W_L [C x ldw_head], read before the W_L update
+  int64_t ldw_head;
+  int n_prev;           // n_{L-1}
+  const __nv_bfloat16* s_prev;  // S_{L-1} (sigma' stash) [b x ld_prev]
+  __nv_bfloat16* dz_prev;       // dZ_{L-1} [b x ld_prev]
+  int64_t ld_prev;
+  float* bpart_prev;    // bias partials of dZ_{L-1} [m tiles x n_prev]
 };
 
 template <typename T>

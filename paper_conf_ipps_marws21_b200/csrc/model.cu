@@ -550,6 +550,14 @@ static int run_step_simt(hb_worker* w, const void* X, int64_t ldx, int32_t xdt, 
   return HB_OK;
 }
 
+// Optionally (HB_HEAD_FUSE=1) the output layer's dX runs in the head kernel's epilogue when C <= 16.
+// Off by default: measured slower on B200 at b = 8192 (37.5 M vs 42.5 M samples/s on C2) because
+// the head grid has only b/128 CTAs while the separate dX GEMM fills all 148 SMs.
+static bool head_dx_fused(const hb_model* m) {
+  static const bool on = env_int("HB_HEAD_FUSE", 0) != 0;
+  return on && m->layers.size() >= 2 && m->layers.back().n_out <= 16;
+}
+
 // Forward chain (Eq. (1)) of the bf16 tensor-core path.  X holds x_rows rows; the batch starts
 // at row *d_off (graph replay) or at row 0 (d_off == nullptr).  With want_grad the head writes
 // dZ_L and its bias partials; otherwise only the per-row losses (mlp_loss).
@@ -586,6 +594,16 @@ static int forward_tc(hb_worker* w, const void* X, int64_t ldx, int64_t x_rows, 
       ep.inv_b = 1.0f / (float)b;
       ep.bpart_out = want_grad ? w->bpart[l] : nullptr;
       ep.ldp = Ly.n_out;
+      if (want_grad && head_dx_fused(m)) {  // the output layer's dX runs in this kernel's epilogue
+        const Layer& Lp = m->layers[l - 1];
+        ep.w_head = m->master + Ly.w_off;
+        ep.ldw_head = Ly.ldw;
+        ep.n_prev = Lp.n_out;
+        ep.s_prev = static_cast<const __nv_bfloat16*>(w->S[l - 1]);
+        ep.dz_prev = static_cast<__nv_bfloat16*>(w->dZ[l - 1]);
+        ep.ld_prev = Lp.ldo;
+        ep.bpart_prev = w->bpart[l - 1];
+      }
       rc = gemm_tc_p(EPI_HEAD_XENT, false, false, b, Ly.n_out, Ly.n_in, A, B, ep, s);
       if (rc) return rc;
     } else {
@@ -625,7 +643,7 @@ static int run_step_tc(hb_worker* w, const void* X, int64_t ldx, int64_t x_rows,
     TcOp dZl{w->dZ[l], Ly.ldo, b, nullptr};
     TcOp Al = l == 0 ? TcOp{X, ldx, x_rows, d_off} : TcOp{w->H[l - 1], m->layers[l - 1].ldo, b, nullptr};
     TcOp Wl{m->shadow + Ly.w_off, Ly.ldw, 0, nullptr};
-    if (l > 0) {  // dZ_{l-1} = (dZ_l W_l) * sigma'(Z_{l-1}) and its bias partials
+    if (l > 0 && !(l == L - 1 && head_dx_fused(m))) {  // dZ_{l-1} = (dZ_l W_l) * sigma'(Z_{l-1}) + bias partials
       const Layer& Lp = m->layers[l - 1];
       EpiArgs ep{};
       ep.M = b;

@@ -139,6 +139,7 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
   uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(tmem_empty_bar + 2);
   __shared__ float red[4 * BN];    // per-quadrant column sums (bias-gradient partials)
   __shared__ float sbias[2][BN];   // bias of the tile, double-buffered across tiles
+  __shared__ __align__(16) float dzs[EPI == EPI_HEAD_XENT ? TC_BM * 16 : 4];  // dZ_L rows (fused head dX)
 
   const int warp = threadIdx.x >> 5;
   const int lane = threadIdx.x & 31;
@@ -346,6 +347,49 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
         epi_bar_sync();
         if (et < ep.N)
           ep.bpart_out[(int64_t)m_tile * ep.ldp + et] = (red[et] + red[BN + et]) + (red[2 * BN + et] + red[3 * BN + et]);
+      }
+      if (ep.dz_prev) {
+        // ---- fused dX of the output layer: dZ_{L-1} = (dZ_L W_L) * sigma'(Z_{L-1}) [Eq. (2), L49],
+        //      column-parallel over the tile's rows (coalesced S loads / dZ stores); each thread
+        //      owns whole columns, so its running sums are the bias partials of dZ_{L-1} ----
+        if (h == 0) {
+          float4* d4 = reinterpret_cast<float4*>(dzs + rl * 16);
+#pragma unroll
+          for (int qq = 0; qq < 4; ++qq) d4[qq] = make_float4(dz[4 * qq], dz[4 * qq + 1], dz[4 * qq + 2], dz[4 * qq + 3]);
+        }
+        epi_bar_sync();
+        const int C = ep.N;
+        const int rows = min(TC_BM, ep.M - m0);
+        for (int pc = et; 2 * pc < ep.n_prev; pc += TC_EPI_THREADS) {
+          const int n = 2 * pc;
+          const bool two = n + 1 < ep.n_prev;
+          float w0[16], w1[16];
+#pragma unroll
+          for (int j = 0; j < 16; ++j) {
+            w0[j] = j < C ? __ldg(ep.w_head + (int64_t)j * ep.ldw_head + n) : 0.f;
+            w1[j] = (j < C && two) ? __ldg(ep.w_head + (int64_t)j * ep.ldw_head + n + 1) : 0.f;
+          }
+          float cs0 = 0.f, cs1 = 0.f;
+#pragma unroll 4
+          for (int rr = 0; rr < rows; ++rr) {
+            const float4* d4 = reinterpret_cast<const float4*>(dzs + rr * 16);
+            float a0 = 0.f, a1 = 0.f;
+#pragma unroll
+            for (int qq = 0; qq < 4; ++qq) {
+              const float4 d = d4[qq];
+              a0 = fmaf(d.x, w0[4 * qq], fmaf(d.y, w0[4 * qq + 1], fmaf(d.z, w0[4 * qq + 2], fmaf(d.w, w0[4 * qq + 3], a0))));
+              a1 = fmaf(d.x, w1[4 * qq], fmaf(d.y, w1[4 * qq + 1], fmaf(d.z, w1[4 * qq + 2], fmaf(d.w, w1[4 * qq + 3], a1))));
+            }
+            const int64_t gr = (int64_t)(m0 + rr);
+            const float2 sf = __bfloat1622float2(*reinterpret_cast<const __nv_bfloat162*>(ep.s_prev + gr * ep.ld_prev + n));
+            const float o0 = a0 * sf.x, o1 = two ? a1 * sf.y : 0.f;
+            *reinterpret_cast<__nv_bfloat162*>(ep.dz_prev + gr * ep.ld_prev + n) = __floats2bfloat162_rn(o0, o1);
+            cs0 += o0;
+            cs1 += o1;
+          }
+          ep.bpart_prev[(int64_t)m_tile * ep.n_prev + n] = cs0;
+          if (two) ep.bpart_prev[(int64_t)m_tile * ep.n_prev + n + 1] = cs1;
+        }
       }
     } else {
       if (active) {

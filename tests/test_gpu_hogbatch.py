@@ -219,3 +219,24 @@ def test_nested_hogwild_worker_in_adaptive_run():
         if prev is not None and prev[9] and r[6] == "none":
             assert r[4] == prev[8] + 8.0
         prev = r
+
+
+def test_fused_head_dx_matches_oracle():
+    # opt-in fusion of the output layer's dX into the head kernel (HB_HEAD_FUSE=1), in a child
+    # process so the env knob is read fresh
+    import subprocess
+    import sys
+    code = (
+        "import numpy as np, torch, sys; sys.path.insert(0, '.');"
+        "import paper_conf_ipps_marws21_b200 as hb; from oracle import mlp64;"
+        "from tests.helpers import *;"
+        "dims=[54,256,200,7]; X,y=dataset('covtype',1000,seed=7);"
+        "m=hb.MLP(dims); p=init_params(dims); m.set_params(params_to_flat(p)); w=hb.Worker(m,1000);"
+        "tX,ty=to_device(X,y); g,l=w.step_grads(tX,ty,1000); dW,db,lr=mlp64.grads(p,X.astype(np.float64),y);"
+        "G=split_flat(g,dims); e=max(max(rel_err(G[i][0],dW[i]),rel_err(G[i][1],db[i])) for i in range(3));"
+        "print('ERR', e); assert e <= 1e-2")
+    import os
+    env = dict(os.environ, HB_HEAD_FUSE="1")
+    r = subprocess.run([sys.executable, "-c", code], capture_output=True, text=True, env=env, timeout=300,
+                       cwd=os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+    assert r.returncode == 0, r.stdout + r.stderr
