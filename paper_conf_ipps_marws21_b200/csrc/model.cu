@@ -384,6 +384,12 @@ static void free_worker_buffers(hb_worker* w) {
   w->h_off = nullptr;
   cudaFree(w->ws);
   w->ws = nullptr;
+  for (cudaEvent_t e : w->ev_bwd) cudaEventDestroy(e);
+  w->ev_bwd.clear();
+  if (w->ev_join2) cudaEventDestroy(w->ev_join2);
+  w->ev_join2 = nullptr;
+  if (w->s2) cudaStreamDestroy(w->s2);
+  w->s2 = nullptr;
   cudaFree(w->logits);
   cudaFree(w->row_loss);
   cudaFree(w->dsum);
@@ -434,6 +440,16 @@ static int alloc_worker(hb_model* m, int max_b, cudaStream_t stream, bool own, h
   }
   if (m->prec == HB_PREC_BF16 && cudaMalloc(&w->ws, (size_t)148 * TC_BM * 256 * 4) != cudaSuccess)
     return fail_free(fail(HB_ENOMEM, "split-K workspace alloc"));
+  if (m->prec == HB_PREC_BF16) {  // second stream for the dW GEMMs (backward overlap)
+    if (cudaStreamCreateWithFlags(&w->s2, cudaStreamNonBlocking) != cudaSuccess)
+      return fail_free(fail(HB_ECUDA, "stream create"));
+    for (int l = 0; l < L; ++l) {
+      cudaEvent_t e;
+      cudaEventCreateWithFlags(&e, cudaEventDisableTiming);
+      w->ev_bwd.push_back(e);
+    }
+    cudaEventCreateWithFlags(&w->ev_join2, cudaEventDisableTiming);
+  }
   if (cudaMalloc(&w->logits, (size_t)max_b * w->ldc * 4) != cudaSuccess ||
       cudaMalloc(&w->row_loss, (size_t)max_b * 4) != cudaSuccess ||
       cudaMalloc(&w->d_off, sizeof(int)) != cudaSuccess || cudaMallocHost(&w->h_off, sizeof(int)) != cudaSuccess ||
@@ -638,6 +654,10 @@ static int run_step_tc(hb_worker* w, const void* X, int64_t ldx, int64_t x_rows,
   int rc = forward_tc(w, X, ldx, x_rows, y, d_off, b, true, s);
   if (rc) return rc;
   const int mt = (b + TC_BM - 1) / TC_BM;
+  // dW_l only has to follow dX_l (the last reader of W_l): it runs on the worker's second stream,
+  // overlapping dX_{l-1} (HB_NO_BWD_OVERLAP=1 keeps everything on one stream)
+  static const bool overlap = env_int("HB_NO_BWD_OVERLAP", 0) == 0;
+  cudaStream_t s2 = overlap && w->s2 ? w->s2 : s;
   for (int l = L - 1; l >= 0; --l) {
     const Layer& Ly = m->layers[l];
     TcOp dZl{w->dZ[l], Ly.ldo, b, nullptr};
@@ -656,6 +676,10 @@ static int run_step_tc(hb_worker* w, const void* X, int64_t ldx, int64_t x_rows,
       ep.ldp = Lp.n_out;
       rc = gemm_tc_p(EPI_DGRAD_SIG, false, true, b, Ly.n_in, Ly.n_out, dZl, Wl, ep, s);
       if (rc) return rc;
+    }
+    if (s2 != s) {
+      HB_CUDA_TRY(cudaEventRecord(w->ev_bwd[l], s));
+      HB_CUDA_TRY(cudaStreamWaitEvent(s2, w->ev_bwd[l], 0));
     }
     // W_l -= lr * dZ_l^T A_{l-1};  b_l -= lr * 1^T dZ_l  (from the partials)
     EpiArgs ep{};
@@ -676,13 +700,17 @@ static int run_step_tc(hb_worker* w, const void* X, int64_t ldx, int64_t x_rows,
     if (!tr) {
       ep.M = Ly.n_out;
       ep.N = Ly.n_in;
-      rc = gemm_tc_p(epi, true, true, Ly.n_out, Ly.n_in, b, dZl, Al, ep, s);
+      rc = gemm_tc_p(epi, true, true, Ly.n_out, Ly.n_in, b, dZl, Al, ep, s2);
     } else {
       ep.M = Ly.n_in;
       ep.N = Ly.n_out;
-      rc = gemm_tc_p(epi, true, true, Ly.n_in, Ly.n_out, b, Al, dZl, ep, s);
+      rc = gemm_tc_p(epi, true, true, Ly.n_in, Ly.n_out, b, Al, dZl, ep, s2);
     }
     if (rc) return rc;
+  }
+  if (s2 != s) {  // join: the step completes on the worker's stream
+    HB_CUDA_TRY(cudaEventRecord(w->ev_join2, s2));
+    HB_CUDA_TRY(cudaStreamWaitEvent(s, w->ev_join2, 0));
   }
   return HB_OK;
 }

@@ -78,6 +78,9 @@ struct hb_worker {
   double* h_dsum = nullptr;     // pinned
   float* grads = nullptr;       // mlp_step_grads output (flat padded layout)
   float* ws = nullptr;          // split-K partial tiles of the dW GEMMs (148 x 128 x 256 fp32)
+  cudaStream_t s2 = nullptr;    // dW GEMMs overlap the next dX GEMM on this stream
+  std::vector<cudaEvent_t> ev_bwd;  // per layer: "dX_l issued" (W_l no longer read)
+  cudaEvent_t ev_join2 = nullptr;
   // nested worker (Alg. 2 "CPU worker", L224-L235): t sub-workers run the sub-batches of one
   // ExecuteWork concurrently, each updating the shared model in place
   std::vector<hb_worker*> subs;
