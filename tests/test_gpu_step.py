@@ -120,3 +120,46 @@ def test_step_argument_errors():
         w.step(tX, ty, 0, 0.1)           # empty batch
     with pytest.raises(hb.HogbatchError):
         w.step(tX.float(), ty, 8, 0.1)   # bf16 model needs bf16 X
+
+
+@pytest.mark.parametrize("prec", ["bf16", "fp32"])
+def test_single_layer_logistic_regression(prec):
+    # L = 1: the output layer reads X directly; its dW GEMM takes X as an MN-major operand
+    e, le, errs = grads_case([54, 7], "covtype", 300, prec)
+    assert e <= TOL[prec], errs
+
+
+@pytest.mark.parametrize("prec", ["bf16", "fp32"])
+def test_many_classes_uses_warp_shuffle_softmax(prec):
+    # C > 16 takes the standalone warp-per-row softmax-xent kernel (delicious-like heads)
+    dims = [64, 96, 40]
+    X, y = dataset("gauss", 257, d=64, seed=3)
+    y = np.random.default_rng(0).integers(0, 40, 257).astype(np.int32)
+    m, w, params = make(dims, prec, 257)
+    tX, ty = to_device(X, y, "bf16" if prec == "bf16" else "f32")
+    g, loss = w.step_grads(tX, ty, 257)
+    dW, db, l_ref = mlp64.grads(params, X.astype(np.float64), y)
+    got = split_flat(g, dims)
+    for l in range(2):
+        assert rel_err(got[l][0], dW[l]) <= TOL[prec]
+        assert rel_err(got[l][1], db[l]) <= TOL[prec]
+    assert abs(loss - l_ref) / l_ref <= TOL[prec]
+
+
+def test_batch_equal_to_max_batch_and_ragged_tiles():
+    # b = max_batch with a ragged last row tile (b % 128 != 0) and ragged widths
+    e, le, errs = grads_case([100, 136, 72, 3], "gauss", 1000, "bf16", d=100)
+    assert e <= TOL["bf16"], errs
+
+
+def test_mlp_create_argument_errors():
+    _need_gpu()
+    with pytest.raises(hb.HogbatchError):
+        hb.MLP([54])                  # needs n_dims >= 2
+    with pytest.raises(hb.HogbatchError):
+        hb.MLP([54, 0, 7])            # zero width
+    with pytest.raises(hb.HogbatchError):
+        hb.MLP([54, 64, 1])           # one class
+    m = hb.MLP([5, 4, 3])
+    with pytest.raises(hb.HogbatchError):
+        m.set_params(np.zeros(3, np.float32))   # wrong parameter count
