@@ -499,9 +499,11 @@ static int run_step_simt(hb_worker* w, const void* X, int64_t ldx, int32_t xdt, 
     rc = gemm_simt_p(epi, false, false, b, Ly.n_out, Ly.n_in, Ain, lda, ain_dt, m->master + Ly.w_off, Ly.ldw, HB_F32,
                      ep, s);
     if (rc) return rc;
-    Ain = w->H[l];
-    lda = Ly.ldo;
-    ain_dt = HB_F32;
+    if (l < L - 1) {
+      Ain = w->H[l];
+      lda = Ly.ldo;
+      ain_dt = HB_F32;
+    }
   }
   {
     const Layer& Ly = m->layers[L - 1];
@@ -1299,9 +1301,11 @@ int mlp_loss(hb_model* m, const void* X, int64_t ldx, int32_t x_dtype, const int
         rc = gemm_simt_p(epi, false, false, b, Ly.n_out, Ly.n_in, Ain, lda, adt, m->master + Ly.w_off, Ly.ldw,
                          HB_F32, ep, s);
         if (rc) return rc;
-        Ain = w->H[l];
-        lda = Ly.ldo;
-        adt = HB_F32;
+        if (l < L - 1) {
+          Ain = w->H[l];
+          lda = Ly.ldo;
+          adt = HB_F32;
+        }
       }
       softmax_xent_kernel<float><<<(b * 32 + 255) / 256, 256, 0, s>>>(
           w->logits, w->ldc, y + r0, nullptr, b, m->layers.back().n_out, (float*)nullptr, 0, w->row_loss, 1.0f);
