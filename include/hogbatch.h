@@ -147,6 +147,12 @@ int mlp_create(const int32_t* dims, int32_t n_dims, int32_t activation, int32_t 
 int mlp_destroy(hb_model* m);
 /* number of parameters P + sum n_l (weights + biases) */
 int mlp_num_params(const hb_model* m, int64_t* n_out);
+/* Which step implementation the model's workers use (introspection for tests / benches):
+ * returns 1 and sets *cluster_size (1 or 2 CTAs per 128-row block) if SGD steps take the fused
+ * row-block chain (one kernel for forward, softmax-xent head and the whole dX chain, then the dW
+ * GEMMs; eligible: bf16 model, uniform hidden width n <= 512, n_0 <= 512, C <= 16, 2..12 layers,
+ * not disabled with HB_ROWCHAIN=0), 0 if they take the per-layer GEMM chain, < 0 on error. */
+int mlp_fused_path(const hb_model* m, int32_t* cluster_size);
 /* host flat fp32 layout: [W_1 (n_1 x n_0 row-major, unpadded), b_1, W_2, b_2, ...]; n must equal
  * mlp_num_params.  Blocking.  set also refreshes the bf16 shadow. */
 int mlp_get_params(const hb_model* m, float* host_dst, int64_t n);
@@ -211,7 +217,8 @@ enum {
   HB_PROF_WGRAD_GEMM = 4, /* dW GEMM + fused in-place SGD epilogue                      */
   HB_PROF_BIAS = 5,       /* bias gradient + bias SGD                                   */
   HB_PROF_OTHER = 6,      /* loss reduction, shadow refresh, merge kernels              */
-  HB_PROF_N = 7
+  HB_PROF_ROWCHAIN = 7,   /* fused per-row-block forward + softmax-xent + dX chain (narrow nets) */
+  HB_PROF_N = 8
 };
 typedef struct hb_prof_entry {
   int64_t launches;

@@ -65,6 +65,14 @@ class MLP:
         _check(lib.mlp_num_params(self.h, C.byref(n)))
         return n.value
 
+    def fused_path(self) -> int:
+        """Cluster size (1 or 2) of the fused row-block step kernel, 0 if steps use the per-layer chain."""
+        cs = C.c_int32(0)
+        r = lib.mlp_fused_path(self.h, C.byref(cs))
+        if r < 0:
+            _check(r)
+        return cs.value if r == 1 else 0
+
     def get_params(self) -> np.ndarray:
         out = np.empty(self.num_params, dtype=np.float32)
         _check(lib.mlp_get_params(self.h, out.ctypes.data_as(C.POINTER(C.c_float)), out.size))

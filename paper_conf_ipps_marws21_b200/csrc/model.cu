@@ -20,6 +20,7 @@
 #include "kernels.cuh"
 #include "model.h"
 #include "tc_gemm.cuh"
+#include "rowchain.cuh"
 
 namespace hb {
 
@@ -363,6 +364,134 @@ static int gemm_simt_p(int epi, bool a_mn, bool b_mn, int M, int N, int K, const
 }
 
 // ----------------------------------------------------------------------------------------
+// fused row-block chain (rowchain.cuh): eligibility and launch
+// ----------------------------------------------------------------------------------------
+struct RcCfg {
+  bool ok = false;
+  int CS = 1, NH = 64, NCA = 1, NS = 2, tmem = 128, smem = 0;
+};
+
+static constexpr int RC_SMEM_CAP = 232448 - 4096 /*static red[]*/ - 512 /*margin*/;
+
+// n_0 - n x (L-1) - C with uniform hidden width n <= 512, n_0 <= 512, C <= 16, 2 <= L <= 12
+// (HB_ROWCHAIN=0 disables; HB_RC_CS=1|2 forces the cluster size)
+static RcCfg rowchain_cfg(const hb_model* m) {
+  RcCfg c;
+  static const int on = env_int("HB_ROWCHAIN", 1);
+  if (!on || m->prec != HB_PREC_BF16) return c;
+  const int L = (int)m->layers.size();
+  if (L < 2 || L > RC_MAX_L) return c;
+  const int n0 = m->dims[0], n = m->dims[1], C = m->dims[L];
+  for (int l = 1; l < L; ++l)
+    if (m->dims[l] != n) return c;
+  if (n0 > 512 || n > 512 || C > 16) return c;
+  static const int cs_env = env_int("HB_RC_CS", 0);
+  c.CS = cs_env == 1 || cs_env == 2 ? cs_env : (n > 128 ? 2 : 1);
+  c.NH = (int)round_up((n + c.CS - 1) / c.CS, 64);
+  if (c.NH > 256) {
+    c.CS = 2;
+    c.NH = (int)round_up((n + 1) / 2, 64);
+  }
+  if (c.NH > 256) return c;
+  c.NCA = std::max((n0 + 63) / 64, c.CS * c.NH / 64);
+  const int stb = c.NH * 128;
+  const int fixed = 1024 + (c.NCA + 1) * RC_CHUNK + 8 * (2 * 8 + c.NCA + 8) + 64;
+  c.NS = std::min(8, (RC_SMEM_CAP - fixed) / stb);
+  if (c.NS < 2) return c;
+  c.smem = 1024 + (c.NCA + 1) * RC_CHUNK + c.NS * stb + 8 * (2 * c.NS + c.NCA + 8) + 16;
+  c.tmem = 64;
+  while (c.tmem < 2 * c.NH) c.tmem *= 2;
+  c.ok = true;
+  return c;
+}
+
+// One launch of the fused chain for batch rows [0, b) of X (row offset *d_off when non-null).
+static int launch_rowchain(hb_worker* w, const RcCfg& c, const void* X, int64_t ldx, int64_t x_rows,
+                           const int32_t* y, const int* d_off, int b, cudaStream_t s) {
+  hb_model* m = w->m;
+  const int L = (int)m->layers.size();
+  const int n = m->dims[1];
+  RcParams P;
+  std::memset(&P, 0, sizeof(P));
+  int rc = make_map(&P.mX, X, m->dims[0], x_rows, ldx * 2, 64, 128);
+  for (int l = 0; l < L && !rc; ++l) {
+    const Layer& Ly = m->layers[l];
+    const __nv_bfloat16* W = m->shadow + Ly.w_off;
+    rc = make_map(&P.mW[l], W, Ly.n_in, Ly.n_out, (int64_t)Ly.ldw * 2, 64, l == L - 1 ? 16 : c.NH);
+    if (!rc && l >= 1) rc = make_map(&P.mWt[l], W, Ly.n_in, Ly.n_out, (int64_t)Ly.ldw * 2, 64, 64);
+    if (!rc && l <= L - 2) {
+      rc = make_map(&P.mH[l], w->H[l], n, b, (int64_t)Ly.ldo * 2, 64, 32);
+      if (!rc) rc = make_map(&P.mDZ[l], w->dZ[l], n, b, (int64_t)Ly.ldo * 2, 64, 32);
+      P.S[l] = static_cast<__nv_bfloat16*>(w->S[l]);
+    }
+    P.bias[l] = m->master + Ly.b_off;
+    P.bpart[l] = w->bpart[l];
+  }
+  if (rc) return rc;
+  P.d_off = d_off;
+  P.y = y;
+  P.dz_head = static_cast<__nv_bfloat16*>(w->dZ[L - 1]);
+  P.row_loss = w->row_loss;
+  P.ldo = m->layers[0].ldo;
+  P.ldo_head = m->layers[L - 1].ldo;
+  P.L = L;
+  P.n0 = m->dims[0];
+  P.n = n;
+  P.C = m->dims[L];
+  P.b = b;
+  P.CS = c.CS;
+  P.NH = c.NH;
+  P.nstages = c.NS;
+  P.abuf_chunks = c.NCA;
+  P.tmem_cols = c.tmem;
+  P.inv_b = 1.0f / (float)b;
+  int dev = 0;
+  cudaGetDevice(&dev);
+  {
+    std::lock_guard<std::mutex> g(g_attr_mu);
+    auto key = std::make_pair((const void*)rowchain_kernel, dev);
+    if (!g_attr_done.count(key)) {
+      HB_CUDA_TRY(cudaFuncSetAttribute(rowchain_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, RC_SMEM_CAP));
+      g_attr_done.insert(key);
+    }
+  }
+  cudaLaunchConfig_t cfg{};
+  cfg.gridDim = dim3(c.CS * ((b + 127) / 128), 1, 1);
+  cfg.blockDim = dim3(RC_THREADS);
+  cfg.dynamicSmemBytes = c.smem;
+  cfg.stream = s;
+  cudaLaunchAttribute attr[2];
+  int na = 0;
+  attr[na].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+  attr[na].val.programmaticStreamSerializationAllowed = 1;
+  ++na;
+  if (c.CS > 1) {
+    attr[na].id = cudaLaunchAttributeClusterDimension;
+    attr[na].val.clusterDim.x = c.CS;
+    attr[na].val.clusterDim.y = 1;
+    attr[na].val.clusterDim.z = 1;
+    ++na;
+  }
+  cfg.attrs = attr;
+  cfg.numAttrs = na;
+  HB_CUDA_TRY(cudaLaunchKernelEx(&cfg, rowchain_kernel, P));
+  HB_CUDA_TRY(cudaGetLastError());
+  return HB_OK;
+}
+
+// algorithmic FLOPs / bytes of one chain launch: forward + dX contractions; X, W (read by the
+// forward and the dX GEMMs), y, and the H/S/dZ/row-loss traffic the dW GEMMs need
+static void rowchain_cost(const hb_model* m, int b, double* flops, double* bytes) {
+  const int L = (int)m->layers.size();
+  double P = 0, hid = 0;
+  for (int l = 0; l < L; ++l) P += (double)m->layers[l].n_in * m->layers[l].n_out;
+  for (int l = 0; l + 1 < L; ++l) hid += m->layers[l].n_out;
+  const double p1 = (double)m->layers[0].n_in * m->layers[0].n_out;
+  *flops = 2.0 * b * P + 2.0 * b * (P - p1);
+  *bytes = 2.0 * b * m->dims[0] + 4.0 * P + 4.0 * b + 2.0 * b * hid * 4.0 + 2.0 * b * m->dims[L] + 4.0 * b;
+}
+
+// ----------------------------------------------------------------------------------------
 // model / worker
 // ----------------------------------------------------------------------------------------
 static int act_dt(const hb_model* m) { return m->prec == HB_PREC_BF16 ? HB_BF16 : HB_F32; }
@@ -388,6 +517,14 @@ static void free_worker_buffers(hb_worker* w) {
   w->ev_bwd.clear();
   if (w->ev_join2) cudaEventDestroy(w->ev_join2);
   w->ev_join2 = nullptr;
+  for (cudaStream_t x : w->sdw) cudaStreamDestroy(x);
+  w->sdw.clear();
+  for (cudaEvent_t e : w->ev_dw) cudaEventDestroy(e);
+  w->ev_dw.clear();
+  if (w->ev_chain) cudaEventDestroy(w->ev_chain);
+  w->ev_chain = nullptr;
+  for (float* p : w->ws_l) cudaFree(p);
+  w->ws_l.clear();
   if (w->s2) cudaStreamDestroy(w->s2);
   w->s2 = nullptr;
   cudaFree(w->logits);
@@ -400,7 +537,7 @@ static void free_worker_buffers(hb_worker* w) {
   w->h_dsum = nullptr;
 }
 
-static int alloc_worker(hb_model* m, int max_b, cudaStream_t stream, bool own, hb_worker** out) {
+static int alloc_worker(hb_model* m, int max_b, cudaStream_t stream, bool own, hb_worker** out, bool train = true) {
   hb_worker* w = new hb_worker();
   w->m = m;
   w->max_b = max_b;
@@ -449,6 +586,22 @@ static int alloc_worker(hb_model* m, int max_b, cudaStream_t stream, bool own, h
       w->ev_bwd.push_back(e);
     }
     cudaEventCreateWithFlags(&w->ev_join2, cudaEventDisableTiming);
+  }
+  if (train && rowchain_cfg(m).ok) {  // fused path: concurrent dW GEMMs, one stream + workspace per layer
+    for (int l = 0; l < L; ++l) {
+      cudaStream_t x;
+      cudaEvent_t e;
+      float* p = nullptr;
+      if (cudaStreamCreateWithFlags(&x, cudaStreamNonBlocking) != cudaSuccess)
+        return fail_free(fail(HB_ECUDA, "stream create"));
+      w->sdw.push_back(x);
+      cudaEventCreateWithFlags(&e, cudaEventDisableTiming);
+      w->ev_dw.push_back(e);
+      if (cudaMalloc(&p, (size_t)148 * TC_BM * 256 * 4) != cudaSuccess)
+        return fail_free(fail(HB_ENOMEM, "split-K workspace alloc"));
+      w->ws_l.push_back(p);
+    }
+    cudaEventCreateWithFlags(&w->ev_chain, cudaEventDisableTiming);
   }
   if (cudaMalloc(&w->logits, (size_t)max_b * w->ldc * 4) != cudaSuccess ||
       cudaMalloc(&w->row_loss, (size_t)max_b * 4) != cudaSuccess ||
@@ -646,16 +799,87 @@ static int forward_tc(hb_worker* w, const void* X, int64_t ldx, int64_t x_rows, 
   return HB_OK;
 }
 
+// dW_l = dZ_l^T A_{l-1} with the fused in-place SGD of W_l and b_l (b_l from the partials of the
+// dZ producer) on stream s, split-K workspace ws
+static int launch_wgrad(hb_worker* w, int l, const void* X, int64_t ldx, int64_t x_rows, const int* d_off, int b,
+                        float lr, bool grads_only, cudaStream_t s, float* ws) {
+  hb_model* m = w->m;
+  const Layer& Ly = m->layers[l];
+  TcOp dZl{w->dZ[l], Ly.ldo, b, nullptr};
+  TcOp Al = l == 0 ? TcOp{X, ldx, x_rows, d_off} : TcOp{w->H[l - 1], m->layers[l - 1].ldo, b, nullptr};
+  EpiArgs ep{};
+  const int epi = grads_only ? EPI_WGRAD_STORE : EPI_WGRAD_SGD;
+  ep.master = m->master + Ly.w_off;
+  ep.shadow = m->shadow + Ly.w_off;
+  ep.ldw = Ly.ldw;
+  ep.lr = lr;
+  if (grads_only) ep.out0 = w->grads + Ly.w_off;
+  ep.bpart_in = w->bpart[l];
+  ep.ldp = Ly.n_out;
+  ep.n_mtiles = (b + TC_BM - 1) / TC_BM;
+  ep.bias_upd = m->master + Ly.b_off;
+  ep.bias_grad = grads_only ? w->grads + Ly.b_off : nullptr;
+  ep.ws = ws;
+  const bool tr = Ly.n_out < 128 && Ly.n_out < Ly.n_in;  // small head: M = n_in instead of n_out
+  ep.transposed = tr ? 1 : 0;
+  if (!tr) {
+    ep.M = Ly.n_out;
+    ep.N = Ly.n_in;
+    return gemm_tc_p(epi, true, true, Ly.n_out, Ly.n_in, b, dZl, Al, ep, s);
+  }
+  ep.M = Ly.n_in;
+  ep.N = Ly.n_out;
+  return gemm_tc_p(epi, true, true, Ly.n_in, Ly.n_out, b, Al, dZl, ep, s);
+}
+
+// Fused path: one rowchain launch (forward, head, dX chain for every 128-row block), then the dW
+// GEMMs of all layers concurrently on the worker's per-layer streams (they only read H/dZ and each
+// updates a different W_l; every dX read of W happened inside the chain), joined on s.
+static int run_step_rowchain(hb_worker* w, const RcCfg& c, const void* X, int64_t ldx, int64_t x_rows,
+                             const int32_t* y, const int* d_off, int b, float lr, bool grads_only, cudaStream_t s) {
+  hb_model* m = w->m;
+  const int L = (int)m->layers.size();
+  {
+    Prof pr(HB_PROF_ROWCHAIN, s);
+    int rc = launch_rowchain(w, c, X, ldx, x_rows, y, d_off, b, s);
+    if (rc) return rc;
+    double fl, by;
+    rowchain_cost(m, b, &fl, &by);
+    pr.done(1, fl, by);
+  }
+  static const bool conc = env_int("HB_RC_DW_SERIAL", 0) == 0;
+  if (!conc) {
+    for (int l = L - 1; l >= 0; --l) {
+      int rc = launch_wgrad(w, l, X, ldx, x_rows, d_off, b, lr, grads_only, s, w->ws_l[l]);
+      if (rc) return rc;
+    }
+    return HB_OK;
+  }
+  HB_CUDA_TRY(cudaEventRecord(w->ev_chain, s));
+  for (int l = L - 1; l >= 0; --l) {
+    HB_CUDA_TRY(cudaStreamWaitEvent(w->sdw[l], w->ev_chain, 0));
+    int rc = launch_wgrad(w, l, X, ldx, x_rows, d_off, b, lr, grads_only, w->sdw[l], w->ws_l[l]);
+    if (rc) return rc;
+    HB_CUDA_TRY(cudaEventRecord(w->ev_dw[l], w->sdw[l]));
+  }
+  for (int l = L - 1; l >= 0; --l) HB_CUDA_TRY(cudaStreamWaitEvent(s, w->ev_dw[l], 0));
+  return HB_OK;
+}
+
 // One SGD step of the bf16 tensor-core path: forward + fused head, then for l = L..1
 // dgrad (reads W_l before it is updated) and wgrad with the fused in-place SGD of W_l and b_l.
-// 3L - 1 kernel launches for C <= 16 (L fwd incl. head, L-1 dgrad, L wgrad).
+// 3L - 1 kernel launches for C <= 16 (L fwd incl. head, L-1 dgrad, L wgrad).  Narrow nets take
+// the fused row-block path (L + 1 launches).
 static int run_step_tc(hb_worker* w, const void* X, int64_t ldx, int64_t x_rows, const int32_t* y, const int* d_off,
                        int b, float lr, bool grads_only, cudaStream_t s) {
   hb_model* m = w->m;
   const int L = (int)m->layers.size();
+  {
+    const RcCfg c = rowchain_cfg(m);
+    if (c.ok && !w->sdw.empty()) return run_step_rowchain(w, c, X, ldx, x_rows, y, d_off, b, lr, grads_only, s);
+  }
   int rc = forward_tc(w, X, ldx, x_rows, y, d_off, b, true, s);
   if (rc) return rc;
-  const int mt = (b + TC_BM - 1) / TC_BM;
   // dW_l only has to follow dX_l (the last reader of W_l): it runs on the worker's second stream,
   // overlapping dX_{l-1} (HB_NO_BWD_OVERLAP=1 keeps everything on one stream)
   static const bool overlap = env_int("HB_NO_BWD_OVERLAP", 0) == 0;
@@ -663,7 +887,6 @@ static int run_step_tc(hb_worker* w, const void* X, int64_t ldx, int64_t x_rows,
   for (int l = L - 1; l >= 0; --l) {
     const Layer& Ly = m->layers[l];
     TcOp dZl{w->dZ[l], Ly.ldo, b, nullptr};
-    TcOp Al = l == 0 ? TcOp{X, ldx, x_rows, d_off} : TcOp{w->H[l - 1], m->layers[l - 1].ldo, b, nullptr};
     TcOp Wl{m->shadow + Ly.w_off, Ly.ldw, 0, nullptr};
     if (l > 0 && !(l == L - 1 && head_dx_fused(m))) {  // dZ_{l-1} = (dZ_l W_l) * sigma'(Z_{l-1}) + bias partials
       const Layer& Lp = m->layers[l - 1];
@@ -683,31 +906,7 @@ static int run_step_tc(hb_worker* w, const void* X, int64_t ldx, int64_t x_rows,
       HB_CUDA_TRY(cudaEventRecord(w->ev_bwd[l], s));
       HB_CUDA_TRY(cudaStreamWaitEvent(s2, w->ev_bwd[l], 0));
     }
-    // W_l -= lr * dZ_l^T A_{l-1};  b_l -= lr * 1^T dZ_l  (from the partials)
-    EpiArgs ep{};
-    const int epi = grads_only ? EPI_WGRAD_STORE : EPI_WGRAD_SGD;
-    ep.master = m->master + Ly.w_off;
-    ep.shadow = m->shadow + Ly.w_off;
-    ep.ldw = Ly.ldw;
-    ep.lr = lr;
-    if (grads_only) ep.out0 = w->grads + Ly.w_off;
-    ep.bpart_in = w->bpart[l];
-    ep.ldp = Ly.n_out;
-    ep.n_mtiles = mt;
-    ep.bias_upd = m->master + Ly.b_off;
-    ep.bias_grad = grads_only ? w->grads + Ly.b_off : nullptr;
-    ep.ws = w->ws;
-    const bool tr = Ly.n_out < 128 && Ly.n_out < Ly.n_in;  // small head: M = n_in instead of n_out
-    ep.transposed = tr ? 1 : 0;
-    if (!tr) {
-      ep.M = Ly.n_out;
-      ep.N = Ly.n_in;
-      rc = gemm_tc_p(epi, true, true, Ly.n_out, Ly.n_in, b, dZl, Al, ep, s2);
-    } else {
-      ep.M = Ly.n_in;
-      ep.N = Ly.n_out;
-      rc = gemm_tc_p(epi, true, true, Ly.n_in, Ly.n_out, b, Al, dZl, ep, s2);
-    }
+    rc = launch_wgrad(w, l, X, ldx, x_rows, d_off, b, lr, grads_only, s2, w->ws);
     if (rc) return rc;
   }
   if (s2 != s) {  // join: the step completes on the worker's stream
@@ -984,6 +1183,13 @@ int mlp_num_params(const hb_model* m, int64_t* n_out) {
   return HB_OK;
 }
 
+int mlp_fused_path(const hb_model* m, int32_t* cluster_size) {
+  HB_CHECK_ARG(m && cluster_size, "null arg");
+  const RcCfg c = rowchain_cfg(m);
+  *cluster_size = c.ok ? c.CS : 0;
+  return c.ok ? 1 : 0;
+}
+
 int mlp_get_params(const hb_model* m, float* host_dst, int64_t n) {
   int64_t need;
   int rc = mlp_num_params(m, &need);
@@ -1255,7 +1461,7 @@ int mlp_loss(hb_model* m, const void* X, int64_t ldx, int32_t x_dtype, const int
   const int chunk = 8192;
   std::lock_guard<std::mutex> g(m->eval_mu);
   if (!m->eval) {
-    int rc = alloc_worker(m, chunk, m->stream, false, &m->eval);
+    int rc = alloc_worker(m, chunk, m->stream, false, &m->eval, false);
     if (rc) return rc;
   }
   hb_worker* w = m->eval;

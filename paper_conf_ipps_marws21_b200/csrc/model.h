@@ -81,6 +81,12 @@ struct hb_worker {
   cudaStream_t s2 = nullptr;    // dW GEMMs overlap the next dX GEMM on this stream
   std::vector<cudaEvent_t> ev_bwd;  // per layer: "dX_l issued" (W_l no longer read)
   cudaEvent_t ev_join2 = nullptr;
+  // fused row-block path (rowchain.cuh): the dW GEMMs of all layers run concurrently after the
+  // chain kernel, one stream and one split-K workspace per layer
+  std::vector<cudaStream_t> sdw;
+  std::vector<cudaEvent_t> ev_dw;
+  cudaEvent_t ev_chain = nullptr;
+  std::vector<float*> ws_l;
   // nested worker (Alg. 2 "CPU worker", L224-L235): t sub-workers run the sub-batches of one
   // ExecuteWork concurrently, each updating the shared model in place
   std::vector<hb_worker*> subs;

@@ -1,0 +1,455 @@
+// rowchain.cuh — fused per-row-block pass of one SGD step for narrow MLPs.
+//
+// For a net n_0 - n x (L-1) - C (uniform hidden width n <= 512, n_0 <= 512, C <= 16) one launch
+// computes, for every block of 128 batch rows, everything of the step that is row-local:
+//   forward   H_l = sigma(H_{l-1} W_l^T + b_l), S_l = sigma'(z)        l = 0..L-2  [Eq. (1), L43]
+//   head      dZ_{L-1} = (softmax(H_{L-2} W_{L-1}^T + b_{L-1}) - Y)/b, row losses  [L258]
+//   dX chain  dZ_{l-1} = (dZ_l W_l) * S_{l-1}                          l = L-1..1  [Eq. (2), L49]
+// plus the per-block column sums of every dZ (bias-gradient partials).  Only the dW GEMMs
+// (K = batch, a reduction over ALL row blocks) remain; they run afterwards with the in-place SGD
+// epilogue of tc_gemm.cuh, which also keeps Eq. (3)'s order: every dX read of W_l precedes the
+// W_l update.
+//
+// The activations of a row block never leave the SM between layers: the A operand of every
+// GEMM of the chain is a 128 x n bf16 tile resident in shared memory (`abuf`, SWIZZLE_128B K-major
+// chunks of 64 columns), rewritten in place by the epilogue of the previous GEMM; only W streams
+// in (TMA ring) and only what the dW GEMMs need (H_l, dZ_l, S_l) streams out (TMA stores).
+// A cluster of CS = 2 CTAs shares a row block when n > 128: CTA r computes output columns
+// [r*NH, (r+1)*NH) of every layer and ships its half of the new activation tile to the peer
+// (cp.async.bulk shared::cta -> shared::cluster), so 2 x 64 CTAs cover a b = 8192 batch.
+//
+// Roles (384 threads): warp 0 TMA producer (X once, W tiles of every step in MMA order), warp 1
+// MMA issuer (one thread, tcgen05.mma M=128 N=NH into one of two TMEM accumulators), warp 2 TMEM
+// allocator, warps 4..11 epilogue (quadrant q = warp % 4 = TMEM lanes / tile rows 32q..32q+31;
+// column group h = (warp-4)/4 takes the CTA's 64-column chunks c = h, h+2, ...).
+//
+// Synchronisation (mbarriers):
+//   w_full/w_empty[stage]   W ring (TMA complete_tx / tcgen05.commit)
+//   x_full                  X row block loaded (step 0 input)
+//   chunk_ready[g]          abuf chunk g holds the previous step's output: 4 arrivals (one per
+//                           32-row piece; a remote piece arrives with expect_tx + bulk copy)
+//   head_ready              dZ_{L-1} tile written (input of the output layer's dX)
+//   acc_full/acc_empty[2]   TMEM double buffer (MMA <-> epilogue)
+//   peer_free               the PEER's MMAs of the current step have completed (multicast commit):
+//                           only then may this CTA overwrite chunks in the peer's abuf (its input)
+//                           or in its own abuf whose previous bulk copy the peer had to consume.
+#pragma once
+
+#include "common.cuh"
+#include "tc_gemm.cuh"
+
+namespace hb {
+
+constexpr int RC_MAX_L = 12;     // weight layers supported by one launch
+constexpr int RC_THREADS = 384;  // 4 control warps + 8 epilogue warps
+constexpr int RC_EPI_THREADS = 256;
+constexpr int RC_CHUNK = 16384;  // 128 rows x 64 bf16 columns (SW128 K-major)
+constexpr int RC_PIECE = 4096;   // 32 rows of a chunk (one epilogue warp's share)
+
+enum { RC_FWD = 0, RC_HEAD = 1, RC_DX = 2 };
+
+__device__ __forceinline__ void epi_bar_sync_n(int) { asm volatile("bar.sync 1, 256;" ::: "memory"); }
+
+struct RcParams {
+  CUtensorMap mX;                // X [x_rows x n0], box {64, 128}
+  CUtensorMap mW[RC_MAX_L];      // W_l K-major, box {64, NH} (output layer {64, 16})
+  CUtensorMap mWt[RC_MAX_L];     // W_l as MN-major operand (l >= 1), box {64, 64}
+  CUtensorMap mH[RC_MAX_L];      // H_l store [b x n], box {64, 32}          (l <= L-2)
+  CUtensorMap mDZ[RC_MAX_L];     // dZ_l store [b x n], box {64, 32}         (l <= L-2)
+  const float* bias[RC_MAX_L];   // fp32 master b_l
+  __nv_bfloat16* S[RC_MAX_L];    // sigma' stash S_l [b x ldo]                (l <= L-2)
+  float* bpart[RC_MAX_L];        // bias-gradient partials of dZ_l [row blocks x n_out(l)]
+  const int* d_off;              // device row offset of the batch in X / y (nullable)
+  const int32_t* y;
+  __nv_bfloat16* dz_head;        // dZ_{L-1} [b x ldo_head]
+  float* row_loss;               // [b]
+  int64_t ldo, ldo_head;
+  int L, n0, n, C, b;
+  int CS, NH;                    // cluster size, output columns per CTA (multiple of 64)
+  int nstages, abuf_chunks, tmem_cols;
+  float inv_b;
+};
+
+struct RcStep {
+  int kind, layer, N, nkb, kkn;
+  bool bmn;
+};
+
+// Step s of the chain: s < L-1 forward layer s; s = L-1 output layer + softmax-xent;
+// s >= L dX of layer 2L-1-s (s = L: the output layer, K = C <= 16 -> one UMMA_K step).
+__device__ __forceinline__ RcStep rc_step(const RcParams& P, int s) {
+  RcStep st;
+  if (s < P.L - 1) {
+    st.kind = RC_FWD;
+    st.layer = s;
+    st.N = P.NH;
+    st.nkb = ((s == 0 ? P.n0 : P.n) + 63) / 64;
+    st.kkn = 4;
+    st.bmn = false;
+  } else if (s == P.L - 1) {
+    st.kind = RC_HEAD;
+    st.layer = P.L - 1;
+    st.N = 16;
+    st.nkb = (P.n + 63) / 64;
+    st.kkn = 4;
+    st.bmn = false;
+  } else {
+    st.kind = RC_DX;
+    st.layer = 2 * P.L - 1 - s;
+    st.N = P.NH;
+    const bool head = st.layer == P.L - 1;
+    st.nkb = head ? 1 : (P.n + 63) / 64;
+    st.kkn = head ? 1 : 4;
+    st.bmn = true;
+  }
+  return st;
+}
+
+// k-block i of step s reads abuf chunk rc_kchunk(...): this CTA's own chunks first (its epilogue
+// produced them, they are ready before the peer's arrive), then the peer's, in index order.
+__device__ __forceinline__ int rc_kchunk(const RcParams& P, int s, int nkb, int i, int rank) {
+  if (s == 0 || s == P.L) return i;
+  const int ncl = P.NH / 64;
+  const int lo = rank * ncl, hi = min(lo + ncl, nkb);
+  const int nown = max(0, hi - lo);
+  if (i < nown) return lo + i;
+  const int j = i - nown;
+  return j < lo ? j : j + nown;
+}
+
+__global__ void __launch_bounds__(RC_THREADS, 1) rowchain_kernel(const __grid_constant__ RcParams P) {
+  extern __shared__ uint8_t smem_raw[];
+  uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
+  const int NCA = P.abuf_chunks;
+  const int STB = P.NH * 128;  // W stage bytes: NH rows x 128 B (K-major) = NH/64 boxes of 8 KB (MN-major)
+  const int NS = P.nstages;
+  uint8_t* abuf = smem;
+  uint8_t* hbuf = smem + NCA * RC_CHUNK;  // dZ_{L-1} tile (output-layer dX operand)
+  uint8_t* ring = hbuf + RC_CHUNK;
+  uint64_t* w_full = reinterpret_cast<uint64_t*>(ring + NS * STB);
+  uint64_t* w_empty = w_full + NS;
+  uint64_t* chunk_ready = w_empty + NS;
+  uint64_t* head_ready = chunk_ready + NCA;
+  uint64_t* x_full = head_ready + 1;
+  uint64_t* acc_full = x_full + 1;
+  uint64_t* acc_empty = acc_full + 2;
+  uint64_t* peer_free = acc_empty + 2;
+  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(peer_free + 1);
+  __shared__ float red[4 * 256];  // per-quadrant column sums (bias-gradient partials)
+
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  const int CS = P.CS;
+  const int rank = CS > 1 ? (int)cluster_ctarank() : 0;
+  const int peer = rank ^ 1;
+  const int rb = blockIdx.x / CS;  // row block
+  const int NSTEPS = 2 * P.L - 1;
+
+  if (warp == 0 && lane == 0) {
+    tma_prefetch_desc(&P.mX);
+    for (int s = 0; s < NS; ++s) {
+      mbar_init(&w_full[s], 1);
+      mbar_init(&w_empty[s], 1);
+    }
+    for (int g = 0; g < NCA; ++g) mbar_init(&chunk_ready[g], 4);
+    mbar_init(head_ready, 4);
+    mbar_init(x_full, 1);
+    for (int a = 0; a < 2; ++a) {
+      mbar_init(&acc_full[a], 1);
+      mbar_init(&acc_empty[a], 8);
+    }
+    mbar_init(peer_free, 1);
+    fence_barrier_init();
+  }
+  if (warp == 2) {
+    switch (P.tmem_cols) {
+      case 64: tmem_alloc<64>(tmem_slot); break;
+      case 128: tmem_alloc<128>(tmem_slot); break;
+      case 256: tmem_alloc<256>(tmem_slot); break;
+      default: tmem_alloc<512>(tmem_slot); break;
+    }
+  }
+  tc_fence_before();
+  __syncthreads();
+  if (CS > 1) cluster_sync_all();  // the peer's barriers are initialised before any remote op
+  tc_fence_after();
+  const uint32_t tmem_base = *tmem_slot;
+  asm volatile("griddepcontrol.wait;" ::: "memory");
+  asm volatile("griddepcontrol.launch_dependents;" ::: "memory");
+
+  if (warp == 0 && lane == 0) {
+    // ===== TMA producer: X row block, then the W tiles of every step in MMA k-order =====
+    const int off = P.d_off ? __ldg(P.d_off) : 0;
+    const int nc0 = (P.n0 + 63) / 64;
+    mbar_arrive_expect_tx(x_full, nc0 * RC_CHUNK);
+    for (int j = 0; j < nc0; ++j) tma_load_2d(abuf + j * RC_CHUNK, &P.mX, x_full, j * 64, off + rb * 128);
+    int it = 0;
+    for (int s = 0; s < NSTEPS; ++s) {
+      const RcStep st = rc_step(P, s);
+      for (int i = 0; i < st.nkb; ++i, ++it) {
+        const int j = rc_kchunk(P, s, st.nkb, i, rank);
+        const int stg = it % NS;
+        mbar_wait(&w_empty[stg], ((it / NS) & 1) ^ 1);
+        uint8_t* dst = ring + stg * STB;
+        if (st.kind != RC_DX) {
+          const int rows = st.kind == RC_HEAD ? 16 : P.NH;
+          mbar_arrive_expect_tx(&w_full[stg], rows * 128);
+          tma_load_2d(dst, &P.mW[st.layer], &w_full[stg], j * 64, st.kind == RC_HEAD ? 0 : rank * P.NH);
+        } else {
+          const int nb = P.NH / 64;
+          mbar_arrive_expect_tx(&w_full[stg], nb * 8192);
+          for (int q = 0; q < nb; ++q)
+            tma_load_2d(dst + q * 8192, &P.mWt[st.layer], &w_full[stg], rank * P.NH + q * 64, j * 64);
+        }
+      }
+    }
+  } else if (warp == 1 && lane == 0) {
+    // ===== MMA issuer =====
+    int it = 0;
+    uint32_t cnt_bits = 0;  // parity of the next chunk_ready phase per chunk
+    for (int s = 0; s < NSTEPS; ++s) {
+      const RcStep st = rc_step(P, s);
+      const int buf = s & 1;
+      mbar_wait(&acc_empty[buf], ((s >> 1) & 1) ^ 1);
+      tc_fence_after();
+      const uint32_t tacc = tmem_base + (uint32_t)(buf * P.NH);
+      const uint32_t idesc = make_idesc_bf16(128, st.N, false, st.bmn);
+      for (int i = 0; i < st.nkb; ++i, ++it) {
+        const int j = rc_kchunk(P, s, st.nkb, i, rank);
+        uint8_t* a_ptr;
+        if (s == 0) {
+          if (i == 0) mbar_wait(x_full, 0);
+          a_ptr = abuf + j * RC_CHUNK;
+        } else if (s == P.L) {
+          mbar_wait(head_ready, 0);
+          a_ptr = hbuf;
+        } else {
+          mbar_wait_cluster(&chunk_ready[j], (cnt_bits >> j) & 1);
+          cnt_bits ^= 1u << j;
+          a_ptr = abuf + j * RC_CHUNK;
+        }
+        const int stg = it % NS;
+        mbar_wait(&w_full[stg], (it / NS) & 1);
+        tc_fence_after();
+        const uint32_t a_base = smem_u32(a_ptr);
+        const uint32_t b_base = smem_u32(ring + stg * STB);
+        for (int kk = 0; kk < st.kkn; ++kk) {
+          const uint64_t ad = make_sw128_desc(a_base + kk * 32, 16, 1024);
+          const uint64_t bd = st.bmn ? make_sw128_desc(b_base + kk * 2048, 8192, 1024)
+                                     : make_sw128_desc(b_base + kk * 32, 16, 1024);
+          umma_bf16(tacc, ad, bd, idesc, (i | kk) != 0);
+        }
+        umma_commit(&w_empty[stg]);
+      }
+      umma_commit(&acc_full[buf]);
+      if (CS > 1) umma_commit_multicast(peer_free, (uint16_t)(1u << peer));
+    }
+  } else if (warp >= 4) {
+    // ===== epilogue =====
+    const int q = warp & 3;
+    const int h = (warp - 4) >> 2;
+    const int et = threadIdx.x - 128;
+    const int rl = q * 32 + lane;
+    const int grow = rb * 128 + rl;  // batch row
+    const bool row_ok = grow < P.b;
+    const int ncl = P.NH / 64;
+    const int n = P.n;
+    for (int s = 0; s < NSTEPS; ++s) {
+      const RcStep st = rc_step(P, s);
+      const int buf = s & 1;
+      epi_bar_sync_n(RC_EPI_THREADS);  // red[] of the previous step consumed
+      mbar_wait(&acc_full[buf], (s >> 1) & 1);
+      tc_fence_after();
+      if (CS > 1 && st.kind != RC_HEAD) mbar_wait_cluster(peer_free, s & 1);
+      if (lane == 0) tma_store_wait_read();  // this warp's earlier bulk stores no longer read abuf
+      __syncwarp();
+      const uint32_t tq = tmem_base + (uint32_t)(buf * P.NH) + ((uint32_t)(q * 32) << 16);
+      if (st.kind == RC_HEAD) {
+        // ---- softmax cross-entropy on the thread's row of logits (C <= 16) ----
+        if (h == 0) {
+          uint32_t raw[16];
+          tmem_ld_32x32b_x16(tq, raw);
+          tmem_ld_wait();
+          const int C = P.C;
+          const float* bl = P.bias[P.L - 1];
+          float z[16], dz[16];
+          float mx = -INFINITY;
+#pragma unroll
+          for (int j = 0; j < 16; ++j) {
+            z[j] = j < C ? __uint_as_float(raw[j]) + __ldg(bl + j) : -INFINITY;
+            mx = fmaxf(mx, z[j]);
+          }
+          float se = 0.f;
+#pragma unroll
+          for (int j = 0; j < 16; ++j) se += j < C ? expf(z[j] - mx) : 0.f;
+          const float lse = mx + logf(se);
+          const int off = P.d_off ? __ldg(P.d_off) : 0;
+          const int yi = row_ok ? __ldg(P.y + off + grow) : -1;
+          float zy = 0.f;
+#pragma unroll
+          for (int j = 0; j < 16; ++j) {
+            dz[j] = (row_ok && j < C) ? (expf(z[j] - lse) - (j == yi ? 1.f : 0.f)) * P.inv_b : 0.f;
+            zy = j == yi ? z[j] : zy;
+          }
+          uint32_t pk[8];
+#pragma unroll
+          for (int j = 0; j < 8; ++j) pk[j] = pack_bf16x2(dz[2 * j], dz[2 * j + 1]);
+          uint8_t* row = hbuf + rl * 128;
+          *reinterpret_cast<uint4*>(row + ((0 ^ (rl & 7)) << 4)) = make_uint4(pk[0], pk[1], pk[2], pk[3]);
+          *reinterpret_cast<uint4*>(row + ((1 ^ (rl & 7)) << 4)) = make_uint4(pk[4], pk[5], pk[6], pk[7]);
+          if (rank == 0) {
+            if (row_ok) {
+              P.row_loss[grow] = lse - zy;
+              uint4* D = reinterpret_cast<uint4*>(P.dz_head + (int64_t)grow * P.ldo_head);
+              D[0] = make_uint4(pk[0], pk[1], pk[2], pk[3]);
+              if (P.ldo_head >= 16) D[1] = make_uint4(pk[4], pk[5], pk[6], pk[7]);
+            }
+            const float t = warp_colsum16(dz, lane);
+            if (!(lane & 1)) red[q * 256 + colsum16_col(lane)] = t;
+          }
+          fence_proxy_async();
+          __syncwarp();
+          if (lane == 0) mbar_arrive(head_ready);
+        }
+        if (rank == 0) {
+          epi_bar_sync_n(RC_EPI_THREADS);
+          if (et < P.C)
+            P.bpart[P.L - 1][(int64_t)rb * P.C + et] = (red[et] + red[256 + et]) + (red[512 + et] + red[768 + et]);
+        }
+      } else {
+        const bool fwd = st.kind == RC_FWD;
+        const int lo = fwd ? st.layer : st.layer - 1;  // layer whose activation / gradient is produced
+        const bool signal = fwd || st.layer >= 2;       // the output is the next step's A operand
+        const float* bias = fwd ? P.bias[lo] : nullptr;
+        __nv_bfloat16* Sg = P.S[lo];
+        for (int c = h; c < ncl; c += 2) {
+          const int g = rank * ncl + c;
+          const int n0 = g * 64;
+          if (n0 >= n) break;
+          uint8_t* piece = abuf + g * RC_CHUNK + q * RC_PIECE;
+          uint8_t* prow = piece + lane * 128;
+          // prefetch this row's sigma' stash for the chunk (dX)
+          const bool full_chunk = n0 + 64 <= n;
+          uint4 sv[8];
+#pragma unroll
+          for (int k = 0; k < 8; ++k) sv[k] = make_uint4(0, 0, 0, 0);
+          if (!fwd && row_ok && full_chunk) {
+            const uint4* srow = reinterpret_cast<const uint4*>(Sg + (int64_t)grow * P.ldo + n0);
+#pragma unroll
+            for (int k = 0; k < 8; ++k) sv[k] = __ldg(srow + k);
+          }
+#pragma unroll
+          for (int gc = 0; gc < 4; ++gc) {
+            uint32_t raw[16];
+            tmem_ld_32x32b_x16(tq + (uint32_t)(c * 64 + gc * 16), raw);
+            tmem_ld_wait();
+            const int nc = n0 + gc * 16;
+            uint32_t pk[8];
+            if (fwd) {
+              uint32_t sp[8];
+              float bb[16];
+              if (nc + 16 <= n) {
+                const float4* b4 = reinterpret_cast<const float4*>(bias + nc);
+#pragma unroll
+                for (int k = 0; k < 4; ++k) {
+                  const float4 t = __ldg(b4 + k);
+                  bb[4 * k] = t.x;
+                  bb[4 * k + 1] = t.y;
+                  bb[4 * k + 2] = t.z;
+                  bb[4 * k + 3] = t.w;
+                }
+              } else {
+#pragma unroll
+                for (int k = 0; k < 16; ++k) bb[k] = nc + k < n ? __ldg(bias + nc + k) : 0.f;
+              }
+#pragma unroll
+              for (int k = 0; k < 8; ++k) {
+                float h0, d0, h1, d1;
+                sigmoid_d(__uint_as_float(raw[2 * k]) + bb[2 * k], h0, d0);
+                sigmoid_d(__uint_as_float(raw[2 * k + 1]) + bb[2 * k + 1], h1, d1);
+                pk[k] = pack_bf16x2(h0, h1);
+                sp[k] = pack_bf16x2(d0, d1);
+              }
+              if (row_ok) {
+                __nv_bfloat16* srow = Sg + (int64_t)grow * P.ldo + nc;
+                if (nc + 16 <= n) {
+                  reinterpret_cast<uint4*>(srow)[0] = make_uint4(sp[0], sp[1], sp[2], sp[3]);
+                  reinterpret_cast<uint4*>(srow)[1] = make_uint4(sp[4], sp[5], sp[6], sp[7]);
+                } else {
+#pragma unroll
+                  for (int k = 0; k < 16; ++k)
+                    if (nc + k < n) srow[k] = __ushort_as_bfloat16((unsigned short)(sp[k >> 1] >> (16 * (k & 1))));
+                }
+              }
+            } else {
+              float v[16];
+              if (full_chunk) {
+                const uint32_t sw[8] = {sv[2 * gc].x, sv[2 * gc].y, sv[2 * gc].z, sv[2 * gc].w,
+                                        sv[2 * gc + 1].x, sv[2 * gc + 1].y, sv[2 * gc + 1].z, sv[2 * gc + 1].w};
+#pragma unroll
+                for (int k = 0; k < 8; ++k) {
+                  const float2 a = __bfloat1622float2(*reinterpret_cast<const __nv_bfloat162*>(&sw[k]));
+                  v[2 * k] = __uint_as_float(raw[2 * k]) * a.x;
+                  v[2 * k + 1] = __uint_as_float(raw[2 * k + 1]) * a.y;
+                }
+              } else {  // ragged last chunk: columns >= n are zero
+                const __nv_bfloat16* srow = Sg + (int64_t)grow * P.ldo + nc;
+#pragma unroll
+                for (int k = 0; k < 16; ++k)
+                  v[k] = (row_ok && nc + k < n) ? __uint_as_float(raw[k]) * __bfloat162float(srow[k]) : 0.f;
+              }
+#pragma unroll
+              for (int k = 0; k < 8; ++k) pk[k] = pack_bf16x2(v[2 * k], v[2 * k + 1]);
+              const float t = warp_colsum16(v, lane);
+              if (!(lane & 1)) red[q * 256 + c * 64 + gc * 16 + colsum16_col(lane)] = t;
+            }
+            const int j0 = gc * 2;
+            *reinterpret_cast<uint4*>(prow + ((j0 ^ (lane & 7)) << 4)) = make_uint4(pk[0], pk[1], pk[2], pk[3]);
+            *reinterpret_cast<uint4*>(prow + (((j0 + 1) ^ (lane & 7)) << 4)) = make_uint4(pk[4], pk[5], pk[6], pk[7]);
+          }
+          fence_proxy_async();
+          __syncwarp();
+          if (lane == 0) {
+            tma_store_2d(fwd ? &P.mH[lo] : &P.mDZ[lo], piece, n0, rb * 128 + q * 32);
+            if (signal) {
+              if (CS > 1) {
+                const uint32_t rbar = mapa_shared(smem_u32(&chunk_ready[g]), peer);
+                mbar_arrive_expect_tx_remote(rbar, RC_PIECE);
+                bulk_copy_s2cluster(mapa_shared(smem_u32(piece), peer), piece, RC_PIECE, rbar);
+              }
+              mbar_arrive(&chunk_ready[g]);
+            }
+          }
+        }
+        if (lane == 0) tma_store_commit();
+        if (!fwd) {  // bias-gradient partials of dZ_lo for this row block
+          epi_bar_sync_n(RC_EPI_THREADS);
+          for (int cc = et; cc < P.NH; cc += RC_EPI_THREADS) {
+            const int nn = rank * P.NH + cc;
+            if (nn < n)
+              P.bpart[lo][(int64_t)rb * n + nn] = (red[cc] + red[256 + cc]) + (red[512 + cc] + red[768 + cc]);
+          }
+        }
+      }
+      // release the accumulator (all TMEM reads of this warp have completed)
+      tc_fence_before();
+      __syncwarp();
+      if (lane == 0) mbar_arrive(&acc_empty[buf]);
+    }
+    if (lane == 0) tma_store_wait_all();
+  }
+
+  tc_fence_before();
+  __syncthreads();
+  if (CS > 1) cluster_sync_all();  // no remote access to this CTA's shared memory remains
+  if (warp == 2) {
+    tc_fence_after();
+    switch (P.tmem_cols) {
+      case 64: tmem_dealloc<64>(tmem_base); break;
+      case 128: tmem_dealloc<128>(tmem_base); break;
+      case 256: tmem_dealloc<256>(tmem_base); break;
+      default: tmem_dealloc<512>(tmem_base); break;
+    }
+  }
+}
+
+}  // namespace hb
