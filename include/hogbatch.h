@@ -147,12 +147,17 @@ int mlp_create(const int32_t* dims, int32_t n_dims, int32_t activation, int32_t 
 int mlp_destroy(hb_model* m);
 /* number of parameters P + sum n_l (weights + biases) */
 int mlp_num_params(const hb_model* m, int64_t* n_out);
-/* Which step implementation the model's workers use (introspection for tests / benches):
- * returns 1 and sets *cluster_size (1 or 2 CTAs per 128-row block) if SGD steps take the fused
+/* Which step implementation the model's workers use at `batch` rows (<= 0: 8192)
+ * (introspection for tests / benches):
+ * returns 1 and sets *cluster_size (1, 2, 4 or 8 CTAs per 128-row block) if SGD steps take the fused
  * row-block chain (one kernel for forward, softmax-xent head and the whole dX chain, then the dW
  * GEMMs; eligible: bf16 model, uniform hidden width n <= 512, n_0 <= 512, C <= 16, 2..12 layers,
  * not disabled with HB_ROWCHAIN=0), 0 if they take the per-layer GEMM chain, < 0 on error. */
-int mlp_fused_path(const hb_model* m, int32_t* cluster_size);
+int mlp_fused_path(const hb_model* m, int32_t batch, int32_t* cluster_size);
+/* Steps of at least min_batch rows take the fused row-block chain when the shape is eligible
+ * (0 = never; default 8192 = the measured crossover on B200, or HB_RC_MIN_B).  Workers created
+ * afterwards allocate what the fused path needs; set it before mlp_worker_create. */
+int mlp_set_fused_min_batch(hb_model* m, int32_t min_batch);
 /* host flat fp32 layout: [W_1 (n_1 x n_0 row-major, unpadded), b_1, W_2, b_2, ...]; n must equal
  * mlp_num_params.  Blocking.  set also refreshes the bf16 shadow. */
 int mlp_get_params(const hb_model* m, float* host_dst, int64_t n);
@@ -231,6 +236,13 @@ int hb_prof_read(hb_prof_entry* out, int32_t n, int32_t reset);
  * (0 forward+sigmoid, 1 dgrad+sigma', 2 wgrad+SGD) and shape on zero-filled scratch buffers */
 int hb_bench_gemm(int32_t kind, int32_t M, int32_t N, int32_t K, int32_t iters, float* us_out);
 /* tuning only: per-CTA phase timestamps (8 globaltimer ns values per CTA, cap entries) of one launch */
+/* tuning only: hb_rc_trace(NULL, cap) arms per-step globaltimer stamps (10 per CTA per step, 24 steps
+ * per CTA) in later fused row-block launches; hb_rc_trace(host, cap) reads the last launch's */
+int hb_rc_trace(unsigned long long* host, int64_t cap);
+/* tuning only: mean device microseconds of one SGD step (graph-replayed `iters` times, lr = 0) on
+ * rows [0, batch) of X/y; part 0 = whole step, 1 = fused chain only, 2 = dW GEMMs only */
+int hb_bench_step(hb_worker* w, const void* X, int64_t ldx, const int32_t* y, int32_t batch, int32_t iters,
+                  int32_t part, float* us_out);
 int hb_bench_gemm_phases(int32_t kind, int32_t M, int32_t N, int32_t K, unsigned long long* host_ts, int64_t cap);
 
 /* Merge points of one rank for one epoch of served batch sizes batches[0..n):

@@ -65,10 +65,16 @@ class MLP:
         _check(lib.mlp_num_params(self.h, C.byref(n)))
         return n.value
 
-    def fused_path(self) -> int:
-        """Cluster size (1 or 2) of the fused row-block step kernel, 0 if steps use the per-layer chain."""
+    def set_fused_min_batch(self, min_batch: int) -> None:
+        """Steps of >= min_batch rows take the fused row-block kernel when eligible (0 = never).
+        Call before creating workers."""
+        _check(lib.mlp_set_fused_min_batch(self.h, min_batch))
+
+    def fused_path(self, batch: int = 8192) -> int:
+        """Cluster size (1, 2, 4 or 8) of the fused row-block step kernel at `batch` rows, 0 if
+        steps use the per-layer GEMM chain."""
         cs = C.c_int32(0)
-        r = lib.mlp_fused_path(self.h, C.byref(cs))
+        r = lib.mlp_fused_path(self.h, batch, C.byref(cs))
         if r < 0:
             _check(r)
         return cs.value if r == 1 else 0

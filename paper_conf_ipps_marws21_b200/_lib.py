@@ -22,11 +22,11 @@ ACTIONS = ("none", "halve", "double", "clamp_lo", "clamp_hi")
 
 # every symbol include/hogbatch.h declares (checked by tests/test_abi.py)
 EXPORTS = ("hb_last_error", "hb_abi_version", "hb_device_ok", "mlp_create", "mlp_destroy",
-           "mlp_num_params", "mlp_fused_path", "mlp_get_params", "mlp_set_params", "mlp_worker_create",
+           "mlp_num_params", "mlp_fused_path", "mlp_set_fused_min_batch", "mlp_get_params", "mlp_set_params", "mlp_worker_create",
            "mlp_worker_destroy", "mlp_worker_stream", "mlp_step", "mlp_step_grads", "mlp_loss",
            "hb_schedule_trace", "hogbatch_run", "hb_nccl_unique_id", "hb_comm_create",
            "hb_comm_destroy", "hb_merge_begin", "hb_merge", "hb_kernel_launches", "hb_prof_enable",
-           "hb_prof_read", "hb_bench_gemm", "hb_bench_gemm_phases", "hb_merge_schedule",
+           "hb_prof_read", "hb_bench_gemm", "hb_bench_gemm_phases", "hb_rc_trace", "hb_bench_step", "hb_merge_schedule",
            "mlp_worker_create_nested")
 PROF_CLASSES = ("fwd_gemm", "head_gemm", "softmax_xent", "dgrad_gemm", "wgrad_sgd_gemm", "bias_sgd", "other",
                 "rowchain")
@@ -85,7 +85,8 @@ def load():
         "mlp_create": ([P(I32), I32, I32, I32, C.c_uint64, I32, P(VP)], C.c_int),
         "mlp_destroy": ([VP], C.c_int),
         "mlp_num_params": ([VP, P(I64)], C.c_int),
-        "mlp_fused_path": ([VP, P(I32)], C.c_int),
+        "mlp_fused_path": ([VP, I32, P(I32)], C.c_int),
+        "mlp_set_fused_min_batch": ([VP, I32], C.c_int),
         "mlp_get_params": ([VP, P(F), I64], C.c_int),
         "mlp_set_params": ([VP, P(F), I64], C.c_int),
         "mlp_worker_create": ([VP, I32, I32, VP, P(VP)], C.c_int),
@@ -104,6 +105,8 @@ def load():
         "hb_merge": ([VP, VP, F, VP], C.c_int),
         "hb_kernel_launches": ([], I64),
         "hb_prof_enable": ([I32], C.c_int),
+        "hb_rc_trace": ([VP, I64], C.c_int),
+        "hb_bench_step": ([VP, VP, I64, VP, I32, I32, I32, P(F)], C.c_int),
         "hb_prof_read": ([P(ProfEntry), I32, I32], C.c_int),
         "hb_bench_gemm": ([I32, I32, I32, I32, I32, P(F)], C.c_int),
         "hb_bench_gemm_phases": ([I32, I32, I32, I32, P(C.c_uint64), I64], C.c_int),

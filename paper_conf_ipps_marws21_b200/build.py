@@ -35,6 +35,33 @@ def _newer(target, deps):
     return any(os.path.getmtime(d) > t for d in deps)
 
 
+def build_variant(name: str, defines: list[str]) -> str:
+    """Tuning only: a copy of the library compiled with extra -D flags, loaded with HB_LIB=<path>."""
+    nccl_inc, nccl_lib = _nccl_dirs()
+    out_dir = os.path.join(HERE, "variants")
+    os.makedirs(out_dir, exist_ok=True)
+    objdir = os.path.join(ROOT, "build", "obj_" + name)
+    os.makedirs(objdir, exist_ok=True)
+    common = ["-O3", "-lineinfo", "-std=c++17", "-Xcompiler", "-fPIC", "-I", nccl_inc,
+              "-I", os.path.join(ROOT, "include")] + ARCH + ["-D" + d for d in defines]
+    objs = []
+    for src in SOURCES:
+        o = os.path.join(objdir, src + ".o")
+        objs.append(o)
+        cmd = [os.environ.get("NVCC", "nvcc")] + common + (["-x", "cu"] if src.endswith(".cpp") else []) + [
+            "-c", os.path.join(CSRC, src), "-o", o]
+        res = subprocess.run(cmd, capture_output=True, text=True)
+        if res.returncode != 0:
+            raise RuntimeError("nvcc failed:\n" + res.stdout + res.stderr)
+    lib = os.path.join(out_dir, f"libhogbatch_{name}.so")
+    cmd = [os.environ.get("NVCC", "nvcc")] + ARCH + ["-shared", "-o", lib] + objs + [
+        "-L", nccl_lib, "-l:libnccl.so.2", "-Xlinker", "-rpath," + nccl_lib]
+    res = subprocess.run(cmd, capture_output=True, text=True)
+    if res.returncode != 0:
+        raise RuntimeError("link failed:\n" + res.stdout + res.stderr)
+    return lib
+
+
 def build(force: bool = False, verbose: bool = False) -> str:
     nccl_inc, nccl_lib = _nccl_dirs()
     nvcc = os.environ.get("NVCC", "nvcc")
@@ -68,4 +95,7 @@ def build(force: bool = False, verbose: bool = False) -> str:
 
 
 if __name__ == "__main__":
-    print(build(force="--force" in sys.argv, verbose=True))
+    if len(sys.argv) > 2 and sys.argv[1] == "--variant":  # --variant NAME DEF1 DEF2 ...
+        print(build_variant(sys.argv[2], sys.argv[3:]))
+    else:
+        print(build(force="--force" in sys.argv, verbose=True))

@@ -264,7 +264,7 @@ struct TcOp {
 static int gemm_tc(int epi, bool a_mn, bool b_mn, int M, int N, int K, TcOp A, TcOp B, const EpiArgs& ep,
                    cudaStream_t s) {
   const int bn = epi == EPI_HEAD_XENT                          ? 16
-                 : (epi == EPI_WGRAD_SGD || epi == EPI_WGRAD_STORE) ? choose_bn_wgrad(M, N, K)
+                 : (epi == EPI_WGRAD_SGD || epi == EPI_WGRAD_STORE) ? (ep.force_bn ? ep.force_bn : choose_bn_wgrad(M, N, K))
                                                                     : choose_bn(M, N);
   CUtensorMap ma, mb;
   const int64_t ar = A.rows ? A.rows : (a_mn ? K : M);
@@ -281,7 +281,7 @@ static int gemm_tc(int epi, bool a_mn, bool b_mn, int M, int N, int K, TcOp A, T
   } else if (!a_mn && b_mn) {
     if (epi == EPI_DGRAD_SIG) return launch_tc_bn<false, true, EPI_DGRAD_SIG>(bn, ma, mb, M, N, K, A.off, B.off, ep, s);
   } else if (a_mn && b_mn) {
-    const int S = ep.ws ? choose_splits(M, N, K, bn) : 1;
+    const int S = !ep.ws ? 1 : ep.force_splits ? ep.force_splits : choose_splits(M, N, K, bn);
     if (epi == EPI_WGRAD_SGD)
       return launch_tc_bn<true, true, EPI_WGRAD_SGD>(bn, ma, mb, M, N, K, A.off, B.off, ep, s, S);
     if (epi == EPI_WGRAD_STORE)
@@ -371,11 +371,16 @@ struct RcCfg {
   int CS = 1, NH = 64, NCA = 1, NS = 2, tmem = 128, smem = 0;
 };
 
-static constexpr int RC_SMEM_CAP = 232448 - 4096 /*static red[]*/ - 512 /*margin*/;
+static unsigned long long* g_rc_trace = nullptr;  // tuning only: hb_rc_trace
+static int g_bench_part = 0;                      // tuning only: hb_bench_step part
+static int64_t g_rc_trace_cap = 0;
+static constexpr int RC_SMEM_CAP = 232448;  // 227 KB opt-in dynamic shared memory per CTA
 
 // n_0 - n x (L-1) - C with uniform hidden width n <= 512, n_0 <= 512, C <= 16, 2 <= L <= 12
-// (HB_ROWCHAIN=0 disables; HB_RC_CS=1|2 forces the cluster size)
-static RcCfg rowchain_cfg(const hb_model* m) {
+// (HB_ROWCHAIN=0 disables).  Cluster size for a batch of b rows: the widest CS in {1,2,4,8} with
+// at least 64 output columns per CTA whose CS x ceil(b/128) CTAs still fit the SMs in one wave
+// (every doubling halves the W bytes each SM streams per layer); HB_RC_CS forces it.
+static RcCfg rowchain_cfg(const hb_model* m, int b = 8192) {
   RcCfg c;
   static const int on = env_int("HB_ROWCHAIN", 1);
   if (!on || m->prec != HB_PREC_BF16) return c;
@@ -385,20 +390,38 @@ static RcCfg rowchain_cfg(const hb_model* m) {
   for (int l = 1; l < L; ++l)
     if (m->dims[l] != n) return c;
   if (n0 > 512 || n > 512 || C > 16) return c;
+  // measured on B200 (scripts/rc_probe.py, C2 shape): the fused chain is latency-bound at
+  // ~65-90 us whatever the batch, the per-layer chain is cheaper below b = 8192
+  if (m->rc_min_b <= 0 || b < m->rc_min_b) return c;
   static const int cs_env = env_int("HB_RC_CS", 0);
-  c.CS = cs_env == 1 || cs_env == 2 ? cs_env : (n > 128 ? 2 : 1);
-  c.NH = (int)round_up((n + c.CS - 1) / c.CS, 64);
-  if (c.NH > 256) {
-    c.CS = 2;
-    c.NH = (int)round_up((n + 1) / 2, 64);
+  static int nsm = 0;
+  if (!nsm) {
+    int dev = 0;
+    cudaGetDevice(&dev);
+    cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, dev);
+    if (nsm <= 0) nsm = 148;
   }
+  const int rbs = std::max(1, (b + 127) / 128);
+  auto nh_of = [&](int cs) { return (int)round_up((n + cs - 1) / cs, 64); };
+  int cs = 1;
+  if (cs_env == 1 || cs_env == 2 || cs_env == 4 || cs_env == 8) {
+    cs = cs_env;
+  } else {
+    while (cs < RC_MAX_CS && nh_of(cs * 2) >= 64 && (n + cs * 2 * 64 - 1) / (cs * 2 * 64) >= 1 &&
+           nh_of(cs * 2) * (cs * 2 - 1) < n && (long)cs * 2 * rbs <= nsm)
+      cs *= 2;
+  }
+  while (nh_of(cs) > 256 && cs < RC_MAX_CS) cs *= 2;  // TMEM: two NH-column accumulators
+  c.CS = cs;
+  c.NH = nh_of(cs);
   if (c.NH > 256) return c;
   c.NCA = std::max((n0 + 63) / 64, c.CS * c.NH / 64);
   const int stb = c.NH * 128;
-  const int fixed = 1024 + (c.NCA + 1) * RC_CHUNK + 8 * (2 * 8 + c.NCA + 8) + 64;
-  c.NS = std::min(8, (RC_SMEM_CAP - fixed) / stb);
+  // 1 KB alignment slack + abuf + W ring + staged bias (1 KB) + mbarriers
+  const int fixed = 1024 + c.NCA * RC_CHUNK + 1024 + 8 * (2 * RC_MAX_STAGES + c.NCA + 8) + 16;
+  c.NS = std::min(RC_MAX_STAGES, (RC_SMEM_CAP - fixed) / stb);
   if (c.NS < 2) return c;
-  c.smem = 1024 + (c.NCA + 1) * RC_CHUNK + c.NS * stb + 8 * (2 * c.NS + c.NCA + 8) + 16;
+  c.smem = 1024 + c.NCA * RC_CHUNK + c.NS * stb + 1024 + 8 * (2 * c.NS + c.NCA + 8) + 16;
   c.tmem = 64;
   while (c.tmem < 2 * c.NH) c.tmem *= 2;
   c.ok = true;
@@ -445,6 +468,7 @@ static int launch_rowchain(hb_worker* w, const RcCfg& c, const void* X, int64_t 
   P.abuf_chunks = c.NCA;
   P.tmem_cols = c.tmem;
   P.inv_b = 1.0f / (float)b;
+  P.dbg = g_rc_trace;
   int dev = 0;
   cudaGetDevice(&dev);
   {
@@ -571,7 +595,7 @@ static int alloc_worker(hb_model* m, int max_b, cudaStream_t stream, bool own, h
   const int mt = (max_b + 127) / 128;
   for (int l = 0; l < L; ++l) {
     float* p = nullptr;
-    if (cudaMalloc(&p, (size_t)mt * m->layers[l].n_out * 4) != cudaSuccess)
+    if (cudaMalloc(&p, (size_t)4 * mt * m->layers[l].n_out * 4) != cudaSuccess)  // x4: per-quadrant (fused path)
       return fail_free(fail(HB_ENOMEM, "bias partial alloc"));
     w->bpart.push_back(p);
   }
@@ -587,7 +611,7 @@ static int alloc_worker(hb_model* m, int max_b, cudaStream_t stream, bool own, h
     }
     cudaEventCreateWithFlags(&w->ev_join2, cudaEventDisableTiming);
   }
-  if (train && rowchain_cfg(m).ok) {  // fused path: concurrent dW GEMMs, one stream + workspace per layer
+  if (train && rowchain_cfg(m, max_b).ok) {  // fused path possible: per-layer dW streams + workspaces
     for (int l = 0; l < L; ++l) {
       cudaStream_t x;
       cudaEvent_t e;
@@ -605,7 +629,7 @@ static int alloc_worker(hb_model* m, int max_b, cudaStream_t stream, bool own, h
   }
   if (cudaMalloc(&w->logits, (size_t)max_b * w->ldc * 4) != cudaSuccess ||
       cudaMalloc(&w->row_loss, (size_t)max_b * 4) != cudaSuccess ||
-      cudaMalloc(&w->d_off, sizeof(int)) != cudaSuccess || cudaMallocHost(&w->h_off, sizeof(int)) != cudaSuccess ||
+      cudaMalloc(&w->d_off, sizeof(int)) != cudaSuccess || cudaMallocHost(&w->h_off, HB_MAX_INFLIGHT * sizeof(int)) != cudaSuccess ||
       cudaMalloc(&w->dsum, 64 * sizeof(double)) != cudaSuccess ||
       cudaMallocHost(&w->h_dsum, 64 * sizeof(double)) != cudaSuccess)
     return fail_free(fail(HB_ENOMEM, "worker scratch alloc"));
@@ -802,7 +826,8 @@ static int forward_tc(hb_worker* w, const void* X, int64_t ldx, int64_t x_rows, 
 // dW_l = dZ_l^T A_{l-1} with the fused in-place SGD of W_l and b_l (b_l from the partials of the
 // dZ producer) on stream s, split-K workspace ws
 static int launch_wgrad(hb_worker* w, int l, const void* X, int64_t ldx, int64_t x_rows, const int* d_off, int b,
-                        float lr, bool grads_only, cudaStream_t s, float* ws) {
+                        float lr, bool grads_only, cudaStream_t s, float* ws, int part_rows, int force_bn = 0,
+                        int force_splits = 0) {
   hb_model* m = w->m;
   const Layer& Ly = m->layers[l];
   TcOp dZl{w->dZ[l], Ly.ldo, b, nullptr};
@@ -816,7 +841,9 @@ static int launch_wgrad(hb_worker* w, int l, const void* X, int64_t ldx, int64_t
   if (grads_only) ep.out0 = w->grads + Ly.w_off;
   ep.bpart_in = w->bpart[l];
   ep.ldp = Ly.n_out;
-  ep.n_mtiles = (b + TC_BM - 1) / TC_BM;
+  ep.n_mtiles = part_rows;
+  ep.force_bn = force_bn;
+  ep.force_splits = force_splits;
   ep.bias_upd = m->master + Ly.b_off;
   ep.bias_grad = grads_only ? w->grads + Ly.b_off : nullptr;
   ep.ws = ws;
@@ -839,7 +866,7 @@ static int run_step_rowchain(hb_worker* w, const RcCfg& c, const void* X, int64_
                              const int32_t* y, const int* d_off, int b, float lr, bool grads_only, cudaStream_t s) {
   hb_model* m = w->m;
   const int L = (int)m->layers.size();
-  {
+  if (g_bench_part != 2) {
     Prof pr(HB_PROF_ROWCHAIN, s);
     int rc = launch_rowchain(w, c, X, ldx, x_rows, y, d_off, b, s);
     if (rc) return rc;
@@ -847,10 +874,11 @@ static int run_step_rowchain(hb_worker* w, const RcCfg& c, const void* X, int64_
     rowchain_cost(m, b, &fl, &by);
     pr.done(1, fl, by);
   }
+  if (g_bench_part == 1) return HB_OK;
   static const bool conc = env_int("HB_RC_DW_SERIAL", 0) == 0;
   if (!conc) {
     for (int l = L - 1; l >= 0; --l) {
-      int rc = launch_wgrad(w, l, X, ldx, x_rows, d_off, b, lr, grads_only, s, w->ws_l[l]);
+      int rc = launch_wgrad(w, l, X, ldx, x_rows, d_off, b, lr, grads_only, s, w->ws_l[l], 4 * ((b + 127) / 128));
       if (rc) return rc;
     }
     return HB_OK;
@@ -858,7 +886,12 @@ static int run_step_rowchain(hb_worker* w, const RcCfg& c, const void* X, int64_
   HB_CUDA_TRY(cudaEventRecord(w->ev_chain, s));
   for (int l = L - 1; l >= 0; --l) {
     HB_CUDA_TRY(cudaStreamWaitEvent(w->sdw[l], w->ev_chain, 0));
-    int rc = launch_wgrad(w, l, X, ldx, x_rows, d_off, b, lr, grads_only, w->sdw[l], w->ws_l[l]);
+    static const int fbn = env_int("HB_RC_WGRAD_BN", 0), fs = env_int("HB_RC_WGRAD_S", 0);
+    const Layer& Ly = m->layers[l];
+    const bool wide = Ly.n_out >= 128 || Ly.n_out >= Ly.n_in;  // not the transposed small head
+    int rc = launch_wgrad(w, l, X, ldx, x_rows, d_off, b, lr, grads_only, w->sdw[l], w->ws_l[l],
+                          4 * ((b + 127) / 128),  // per-quadrant bias partials of the chain
+                          wide ? fbn : 0, wide ? fs : 0);
     if (rc) return rc;
     HB_CUDA_TRY(cudaEventRecord(w->ev_dw[l], w->sdw[l]));
   }
@@ -875,7 +908,7 @@ static int run_step_tc(hb_worker* w, const void* X, int64_t ldx, int64_t x_rows,
   hb_model* m = w->m;
   const int L = (int)m->layers.size();
   {
-    const RcCfg c = rowchain_cfg(m);
+    const RcCfg c = rowchain_cfg(m, b);
     if (c.ok && !w->sdw.empty()) return run_step_rowchain(w, c, X, ldx, x_rows, y, d_off, b, lr, grads_only, s);
   }
   int rc = forward_tc(w, X, ldx, x_rows, y, d_off, b, true, s);
@@ -906,7 +939,7 @@ static int run_step_tc(hb_worker* w, const void* X, int64_t ldx, int64_t x_rows,
       HB_CUDA_TRY(cudaEventRecord(w->ev_bwd[l], s));
       HB_CUDA_TRY(cudaStreamWaitEvent(s2, w->ev_bwd[l], 0));
     }
-    rc = launch_wgrad(w, l, X, ldx, x_rows, d_off, b, lr, grads_only, s2, w->ws);
+    rc = launch_wgrad(w, l, X, ldx, x_rows, d_off, b, lr, grads_only, s2, w->ws, (b + TC_BM - 1) / TC_BM);
     if (rc) return rc;
   }
   if (s2 != s) {  // join: the step completes on the worker's stream
@@ -940,13 +973,17 @@ int step_graph(hb_worker* w, const void* X, int64_t ldx, int64_t x_rows, const i
   }
   uint32_t lrbits;
   std::memcpy(&lrbits, &lr, 4);
-  auto key = std::make_pair(b, lrbits);
+  // one graph per in-flight slot: a queued replay reads its batch offset from its own pinned
+  // word when it starts, so up to HB_MAX_INFLIGHT replays of this worker may be enqueued
+  const int slot = w->slot;
+  w->slot = (w->slot + 1) % HB_MAX_INFLIGHT;
+  auto key = std::make_tuple(b, lrbits, slot);
   auto it = w->graphs.find(key);
   if (it == w->graphs.end()) {
     cudaStream_t s = w->stream;
     const int64_t l0 = g_launches.load();
     HB_CUDA_TRY(cudaStreamBeginCapture(s, cudaStreamCaptureModeThreadLocal));
-    cudaMemcpyAsync(w->d_off, w->h_off, sizeof(int), cudaMemcpyHostToDevice, s);
+    cudaMemcpyAsync(w->d_off, w->h_off + slot, sizeof(int), cudaMemcpyHostToDevice, s);
     int rc = run_step(w, X, ldx, HB_BF16, x_rows, y, w->d_off, b, lr, false, s);
     cudaGraph_t graph = nullptr;
     cudaError_t ce = cudaStreamEndCapture(s, &graph);
@@ -963,7 +1000,7 @@ int step_graph(hb_worker* w, const void* X, int64_t ldx, int64_t x_rows, const i
     g_launches.fetch_sub(gr.launches);  // counted when replayed
     it = w->graphs.emplace(key, gr).first;
   }
-  *w->h_off = (int)off;  // the previous replay of this worker has completed (caller synchronises)
+  w->h_off[slot] = (int)off;  // the replay that last used this slot has completed (caller's in-flight bound)
   HB_CUDA_TRY(cudaGraphLaunch(it->second.exec, w->stream));
   g_launches.fetch_add(it->second.launches);
   return HB_OK;
@@ -1107,6 +1144,8 @@ int mlp_create(const int32_t* dims, int32_t n_dims, int32_t activation, int32_t 
   m->device = device;
   m->prec = precision;
   m->dims.assign(dims, dims + n_dims);
+  // fused row-block path from this batch size up (measured crossover on B200)
+  m->rc_min_b = env_int("HB_RC_MIN_B", 8192);
   size_t off = 0;
   for (int l = 1; l < n_dims; ++l) {
     Layer Ly;
@@ -1183,9 +1222,80 @@ int mlp_num_params(const hb_model* m, int64_t* n_out) {
   return HB_OK;
 }
 
-int mlp_fused_path(const hb_model* m, int32_t* cluster_size) {
+// Tuning only: cap > 0 arms per-step phase stamps in every later rowchain launch (the buffer is
+// overwritten by each launch); cap == 0 copies the last launch's stamps to host and disarms.
+int hb_rc_trace(unsigned long long* host, int64_t cap) {
+  if (cap > 0 && !host) {
+    cudaFree(g_rc_trace);
+    g_rc_trace = nullptr;
+    HB_CUDA_TRY(cudaMalloc(&g_rc_trace, cap * sizeof(unsigned long long)));
+    HB_CUDA_TRY(cudaMemset(g_rc_trace, 0, cap * sizeof(unsigned long long)));
+    g_rc_trace_cap = cap;
+    return HB_OK;
+  }
+  HB_CHECK_ARG(host && cap > 0, "bad args");
+  HB_CUDA_TRY(cudaDeviceSynchronize());
+  HB_CUDA_TRY(cudaMemcpy(host, g_rc_trace, std::min(cap, g_rc_trace_cap) * sizeof(unsigned long long),
+                         cudaMemcpyDeviceToHost));
+  HB_CUDA_TRY(cudaMemset(g_rc_trace, 0, g_rc_trace_cap * sizeof(unsigned long long)));
+  return HB_OK;
+}
+
+// Tuning only: mean device microseconds of one SGD step of worker w on rows [0, batch) of (X, y),
+// captured once into a CUDA graph and replayed `iters` times back to back (lr = 0: the model
+// is unchanged).  part = 0 whole step, 1 fused chain only (dW GEMMs skipped), 2 dW GEMMs only.
+int hb_bench_step(hb_worker* w, const void* X, int64_t ldx, const int32_t* y, int32_t batch, int32_t iters,
+                  int32_t part, float* us_out) {
+  int rc = check_step_args(w, X, ldx, HB_BF16, y, batch);
+  if (rc) return rc;
+  HB_CHECK_ARG(us_out && iters > 0 && part >= 0 && part <= 2, "bad args");
+  HB_CHECK_ARG(w->m->prec == HB_PREC_BF16 && w->subs.empty(), "bf16 plain worker only");
+  HB_CUDA_TRY(cudaSetDevice(w->m->device));
+  cudaStream_t s = w->stream;
+  g_bench_part = part;
+  rc = run_step(w, X, ldx, HB_BF16, batch, y, nullptr, batch, 0.f, false, s);  // warm-up, attributes
+  cudaGraph_t g = nullptr;
+  cudaGraphExec_t ge = nullptr;
+  if (!rc) {
+    HB_CUDA_TRY(cudaStreamBeginCapture(s, cudaStreamCaptureModeThreadLocal));
+    for (int i = 0; i < iters && !rc; ++i) rc = run_step(w, X, ldx, HB_BF16, batch, y, nullptr, batch, 0.f, false, s);
+    cudaError_t ce = cudaStreamEndCapture(s, &g);
+    if (!rc && ce != cudaSuccess) rc = fail(HB_ECUDA, std::string("capture: ") + cudaGetErrorString(ce));
+  }
+  g_bench_part = 0;
+  if (rc) {
+    if (g) cudaGraphDestroy(g);
+    return rc;
+  }
+  HB_CUDA_TRY(cudaGraphInstantiate(&ge, g, 0));
+  cudaGraphDestroy(g);
+  cudaEvent_t e0, e1;
+  cudaEventCreate(&e0);
+  cudaEventCreate(&e1);
+  cudaGraphLaunch(ge, s);  // warm
+  cudaEventRecord(e0, s);
+  cudaGraphLaunch(ge, s);
+  cudaEventRecord(e1, s);
+  cudaError_t ce = cudaStreamSynchronize(s);
+  float ms = 0.f;
+  cudaEventElapsedTime(&ms, e0, e1);
+  *us_out = ms * 1000.f / iters;
+  cudaEventDestroy(e0);
+  cudaEventDestroy(e1);
+  cudaGraphExecDestroy(ge);
+  if (ce != cudaSuccess) return fail(HB_ECUDA, std::string("bench step: ") + cudaGetErrorString(ce));
+  return HB_OK;
+}
+
+int mlp_set_fused_min_batch(hb_model* m, int32_t min_batch) {
+  HB_CHECK_ARG(m && min_batch >= 0, "bad args");
+  m->rc_min_b = min_batch;
+  return HB_OK;
+}
+
+int mlp_fused_path(const hb_model* m, int32_t batch, int32_t* cluster_size) {
   HB_CHECK_ARG(m && cluster_size, "null arg");
-  const RcCfg c = rowchain_cfg(m);
+  const RcCfg c = rowchain_cfg(m, batch > 0 ? batch : 8192);
   *cluster_size = c.ok ? c.CS : 0;
   return c.ok ? 1 : 0;
 }

@@ -5,12 +5,16 @@
 #include <cuda_runtime.h>
 
 #include <map>
+#include <tuple>
 #include <mutex>
 #include <vector>
 
 #include "../../include/hogbatch.h"
 
 namespace hb {
+
+// graph replays of one worker that may be enqueued before the oldest completes (hogbatch_run)
+constexpr int HB_MAX_INFLIGHT = 4;
 
 // One fully-connected layer W_l [n_out x n_in] (row stride ldw, padded to 8 elements so every
 // bf16 row is 16-byte aligned for TMA) and bias b_l [n_out]; offsets index the flat parameter
@@ -40,6 +44,7 @@ struct hb_model {
   int device = 0;
   int prec = HB_PREC_BF16;
   std::vector<int> dims;
+  int rc_min_b = 8192;              // fused row-block step from this batch size up (0 = never)
   std::vector<hb::Layer> layers;
   size_t total = 0;                 // floats in the flat parameter buffer (incl. padding)
   float* master = nullptr;          // fp32 master weights + biases (the shared global model)
@@ -64,13 +69,14 @@ struct hb_worker {
   float* row_loss = nullptr;    // [max_b]
   std::vector<float*> bpart;    // per layer [ceil(max_b/128) x n_out] bias-gradient partial sums
   int* d_off = nullptr;         // device row offset of the current batch (graph replay)
-  int* h_off = nullptr;         // pinned host source of d_off
+  int* h_off = nullptr;         // pinned host sources of d_off, one per in-flight slot
+  int slot = 0;                 // next slot (graph replays of a worker may be queued HB_MAX_INFLIGHT deep)
   // CUDA graphs of one SGD step, per (batch size, lr), for the dataset they were captured on
   struct Graph {
     cudaGraphExec_t exec = nullptr;
     int launches = 0;
   };
-  std::map<std::pair<int, uint32_t>, Graph> graphs;
+  std::map<std::tuple<int, uint32_t, int>, Graph> graphs;  // (b, lr bits, slot)
   const void* g_X = nullptr;
   const void* g_y = nullptr;
   int64_t g_ldx = 0, g_rows = 0;

@@ -5,23 +5,27 @@
 //   forward   H_l = sigma(H_{l-1} W_l^T + b_l), S_l = sigma'(z)        l = 0..L-2  [Eq. (1), L43]
 //   head      dZ_{L-1} = (softmax(H_{L-2} W_{L-1}^T + b_{L-1}) - Y)/b, row losses  [L258]
 //   dX chain  dZ_{l-1} = (dZ_l W_l) * S_{l-1}                          l = L-1..1  [Eq. (2), L49]
-// plus the per-block column sums of every dZ (bias-gradient partials).  Only the dW GEMMs
-// (K = batch, a reduction over ALL row blocks) remain; they run afterwards with the in-place SGD
+// plus per-32-row column sums of every dZ (bias-gradient partials).  Only the dW GEMMs (K =
+// batch, a reduction over ALL row blocks) remain; they run afterwards with the in-place SGD
 // epilogue of tc_gemm.cuh, which also keeps Eq. (3)'s order: every dX read of W_l precedes the
 // W_l update.
 //
-// The activations of a row block never leave the SM between layers: the A operand of every
-// GEMM of the chain is a 128 x n bf16 tile resident in shared memory (`abuf`, SWIZZLE_128B K-major
+// The activations of a row block never leave the SM between layers: the A operand of every GEMM
+// of the chain is a 128 x n bf16 tile resident in shared memory (`abuf`, SWIZZLE_128B K-major
 // chunks of 64 columns), rewritten in place by the epilogue of the previous GEMM; only W streams
 // in (TMA ring) and only what the dW GEMMs need (H_l, dZ_l, S_l) streams out (TMA stores).
-// A cluster of CS = 2 CTAs shares a row block when n > 128: CTA r computes output columns
-// [r*NH, (r+1)*NH) of every layer and ships its half of the new activation tile to the peer
-// (cp.async.bulk shared::cta -> shared::cluster), so 2 x 64 CTAs cover a b = 8192 batch.
+// A cluster of CS = 1, 2, 4 or 8 CTAs shares a row block: CTA r computes output columns
+// [r*NH, (r+1)*NH) of every layer and ships its 64-column chunks of the new activation tile to
+// every other CTA of the cluster (cp.async.bulk shared::cta -> shared::cluster).  Splitting the
+// columns divides the W bytes each SM must stream per layer by CS — the chain is bound by the
+// W bytes in flight per SM (the shared memory left next to abuf) — so small batches use wide
+// clusters and b = 8192 uses CS = 2 (64 row blocks x 2 CTAs fill the 148 SMs once).
 //
 // Roles (384 threads): warp 0 TMA producer (X once, W tiles of every step in MMA order), warp 1
 // MMA issuer (one thread, tcgen05.mma M=128 N=NH into one of two TMEM accumulators), warp 2 TMEM
-// allocator, warps 4..11 epilogue (quadrant q = warp % 4 = TMEM lanes / tile rows 32q..32q+31;
-// column group h = (warp-4)/4 takes the CTA's 64-column chunks c = h, h+2, ...).
+// allocator, warps 4..11 epilogue: quadrant q = warp % 4 (TMEM lanes = tile rows 32q..32q+31),
+// half h = (warp-4)/4 (columns 32h..32h+31 of every 64-column chunk; the two warps of a quadrant
+// meet on a named barrier before the chunk's 32-row piece is shipped).
 //
 // Synchronisation (mbarriers):
 //   w_full/w_empty[stage]   W ring (TMA complete_tx / tcgen05.commit)
@@ -30,9 +34,10 @@
 //                           32-row piece; a remote piece arrives with expect_tx + bulk copy)
 //   head_ready              dZ_{L-1} tile written (input of the output layer's dX)
 //   acc_full/acc_empty[2]   TMEM double buffer (MMA <-> epilogue)
-//   peer_free               the PEER's MMAs of the current step have completed (multicast commit):
-//                           only then may this CTA overwrite chunks in the peer's abuf (its input)
-//                           or in its own abuf whose previous bulk copy the peer had to consume.
+//   peer_free               the OTHER CTAs' MMAs of the current step have completed (multicast
+//                           commits, CS-1 arrivals per step): only then may this CTA overwrite
+//                           chunks in their abufs (their input) or chunks of its own abuf whose
+//                           previous bulk copies they had to consume.
 #pragma once
 
 #include "common.cuh"
@@ -41,14 +46,18 @@
 namespace hb {
 
 constexpr int RC_MAX_L = 12;     // weight layers supported by one launch
+constexpr int RC_MAX_CS = 8;     // CTAs per row block (portable cluster size)
 constexpr int RC_THREADS = 384;  // 4 control warps + 8 epilogue warps
 constexpr int RC_EPI_THREADS = 256;
 constexpr int RC_CHUNK = 16384;  // 128 rows x 64 bf16 columns (SW128 K-major)
-constexpr int RC_PIECE = 4096;   // 32 rows of a chunk (one epilogue warp's share)
+constexpr int RC_PIECE = 4096;   // 32 rows of a chunk (one quadrant's share)
+constexpr int RC_MAX_STAGES = 12;
 
 enum { RC_FWD = 0, RC_HEAD = 1, RC_DX = 2 };
 
 __device__ __forceinline__ void epi_bar_sync_n(int) { asm volatile("bar.sync 1, 256;" ::: "memory"); }
+// the two epilogue warps of quadrant q (named barriers 2..5)
+__device__ __forceinline__ void quad_bar_sync(int q) { asm volatile("bar.sync %0, 64;" ::"r"(2 + q) : "memory"); }
 
 struct RcParams {
   CUtensorMap mX;                // X [x_rows x n0], box {64, 128}
@@ -58,7 +67,7 @@ struct RcParams {
   CUtensorMap mDZ[RC_MAX_L];     // dZ_l store [b x n], box {64, 32}         (l <= L-2)
   const float* bias[RC_MAX_L];   // fp32 master b_l
   __nv_bfloat16* S[RC_MAX_L];    // sigma' stash S_l [b x ldo]                (l <= L-2)
-  float* bpart[RC_MAX_L];        // bias-gradient partials of dZ_l [row blocks x n_out(l)]
+  float* bpart[RC_MAX_L];        // bias-gradient partials of dZ_l [4 x row blocks x n_out(l)] (per quadrant)
   const int* d_off;              // device row offset of the batch in X / y (nullable)
   const int32_t* y;
   __nv_bfloat16* dz_head;        // dZ_{L-1} [b x ldo_head]
@@ -68,7 +77,10 @@ struct RcParams {
   int CS, NH;                    // cluster size, output columns per CTA (multiple of 64)
   int nstages, abuf_chunks, tmem_cols;
   float inv_b;
+  unsigned long long* dbg;       // tuning only: per CTA, per step RC_DBG_W globaltimer stamps (nullable)
 };
+constexpr int RC_DBG_STEPS = 24;
+constexpr int RC_DBG_W = 10;  // stamps per step
 
 struct RcStep {
   int kind, layer, N, nkb, kkn;
@@ -106,7 +118,7 @@ __device__ __forceinline__ RcStep rc_step(const RcParams& P, int s) {
 }
 
 // k-block i of step s reads abuf chunk rc_kchunk(...): this CTA's own chunks first (its epilogue
-// produced them, they are ready before the peer's arrive), then the peer's, in index order.
+// produced them, they are ready before the others arrive), then the others in index order.
 __device__ __forceinline__ int rc_kchunk(const RcParams& P, int s, int nkb, int i, int rank) {
   if (s == 0 || s == P.L) return i;
   const int ncl = P.NH / 64;
@@ -117,16 +129,24 @@ __device__ __forceinline__ int rc_kchunk(const RcParams& P, int s, int nkb, int 
   return j < lo ? j : j + nown;
 }
 
+// abuf chunk that receives the dZ_{L-1} tile (the output layer's dX operand): with a cluster, the
+// first chunk OWNED BY THE NEXT CTA — only its bulk copies ever write that chunk here, so after
+// this CTA's output-layer MMAs it is free (no outgoing copy or TMA store reads it), and the
+// owner's next write into it waits for this CTA's output-layer dX MMAs (peer_free)
+__device__ __forceinline__ int rc_head_chunk(const RcParams& P, int rank) {
+  return P.CS > 1 ? ((rank + 1) % P.CS) * (P.NH / 64) : 0;
+}
+
 __global__ void __launch_bounds__(RC_THREADS, 1) rowchain_kernel(const __grid_constant__ RcParams P) {
-  extern __shared__ uint8_t smem_raw[];
+  extern __shared__ __align__(1024) uint8_t smem_raw[];
   uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
   const int NCA = P.abuf_chunks;
   const int STB = P.NH * 128;  // W stage bytes: NH rows x 128 B (K-major) = NH/64 boxes of 8 KB (MN-major)
   const int NS = P.nstages;
   uint8_t* abuf = smem;
-  uint8_t* hbuf = smem + NCA * RC_CHUNK;  // dZ_{L-1} tile (output-layer dX operand)
-  uint8_t* ring = hbuf + RC_CHUNK;
-  uint64_t* w_full = reinterpret_cast<uint64_t*>(ring + NS * STB);
+  uint8_t* ring = abuf + NCA * RC_CHUNK;
+  float* sbias = reinterpret_cast<float*>(ring + NS * STB);  // [NH] bias of the current forward step
+  uint64_t* w_full = reinterpret_cast<uint64_t*>(sbias + 256);
   uint64_t* w_empty = w_full + NS;
   uint64_t* chunk_ready = w_empty + NS;
   uint64_t* head_ready = chunk_ready + NCA;
@@ -135,14 +155,13 @@ __global__ void __launch_bounds__(RC_THREADS, 1) rowchain_kernel(const __grid_co
   uint64_t* acc_empty = acc_full + 2;
   uint64_t* peer_free = acc_empty + 2;
   uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(peer_free + 1);
-  __shared__ float red[4 * 256];  // per-quadrant column sums (bias-gradient partials)
 
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const int CS = P.CS;
   const int rank = CS > 1 ? (int)cluster_ctarank() : 0;
-  const int peer = rank ^ 1;
   const int rb = blockIdx.x / CS;  // row block
   const int NSTEPS = 2 * P.L - 1;
+  const int hc = rc_head_chunk(P, rank);
 
   if (warp == 0 && lane == 0) {
     tma_prefetch_desc(&P.mX);
@@ -150,15 +169,21 @@ __global__ void __launch_bounds__(RC_THREADS, 1) rowchain_kernel(const __grid_co
       mbar_init(&w_full[s], 1);
       mbar_init(&w_empty[s], 1);
     }
-    for (int g = 0; g < NCA; ++g) mbar_init(&chunk_ready[g], 4);
+    // chunk g: 4 local arrivals (one per 32-row piece) if this CTA produces it, else one
+    // pre-arming arrival with expect_tx(16 KB) completed by the owner's four bulk copies
+    const int ncl0 = P.NH / 64;
+    for (int g = 0; g < NCA; ++g) mbar_init(&chunk_ready[g], g / ncl0 == rank ? 4 : 1);
     mbar_init(head_ready, 4);
     mbar_init(x_full, 1);
     for (int a = 0; a < 2; ++a) {
       mbar_init(&acc_full[a], 1);
       mbar_init(&acc_empty[a], 8);
     }
-    mbar_init(peer_free, 1);
+    mbar_init(peer_free, CS > 1 ? CS - 1 : 1);
     fence_barrier_init();
+    // pre-arm phase 0 of every valid chunk another CTA produces (step 0's output)
+    for (int g = 0; g < NCA && g * 64 < P.n; ++g)
+      if (g / ncl0 != rank) mbar_arrive_expect_tx(&chunk_ready[g], RC_CHUNK);
   }
   if (warp == 2) {
     switch (P.tmem_cols) {
@@ -170,7 +195,7 @@ __global__ void __launch_bounds__(RC_THREADS, 1) rowchain_kernel(const __grid_co
   }
   tc_fence_before();
   __syncthreads();
-  if (CS > 1) cluster_sync_all();  // the peer's barriers are initialised before any remote op
+  if (CS > 1) cluster_sync_all();  // the other CTAs' barriers are initialised before any remote op
   tc_fence_after();
   const uint32_t tmem_base = *tmem_slot;
   asm volatile("griddepcontrol.wait;" ::: "memory");
@@ -206,11 +231,15 @@ __global__ void __launch_bounds__(RC_THREADS, 1) rowchain_kernel(const __grid_co
     // ===== MMA issuer =====
     int it = 0;
     uint32_t cnt_bits = 0;  // parity of the next chunk_ready phase per chunk
+    const uint16_t others = (uint16_t)(((1u << CS) - 1) & ~(1u << rank));
     for (int s = 0; s < NSTEPS; ++s) {
       const RcStep st = rc_step(P, s);
       const int buf = s & 1;
       mbar_wait(&acc_empty[buf], ((s >> 1) & 1) ^ 1);
       tc_fence_after();
+      unsigned long long* dbg =
+          P.dbg && s < RC_DBG_STEPS ? P.dbg + ((size_t)blockIdx.x * RC_DBG_STEPS + s) * RC_DBG_W : nullptr;
+      if (dbg) dbg[0] = gtimer();
       const uint32_t tacc = tmem_base + (uint32_t)(buf * P.NH);
       const uint32_t idesc = make_idesc_bf16(128, st.N, false, st.bmn);
       for (int i = 0; i < st.nkb; ++i, ++it) {
@@ -221,15 +250,21 @@ __global__ void __launch_bounds__(RC_THREADS, 1) rowchain_kernel(const __grid_co
           a_ptr = abuf + j * RC_CHUNK;
         } else if (s == P.L) {
           mbar_wait(head_ready, 0);
-          a_ptr = hbuf;
+          a_ptr = abuf + hc * RC_CHUNK;
         } else {
-          mbar_wait_cluster(&chunk_ready[j], (cnt_bits >> j) & 1);
+          // local pieces: release.cta arrivals after fence.proxy.async; remote pieces: bulk copies
+          // (async proxy, complete_tx) — both are ordered for the tensor core by the wait itself
+          mbar_wait(&chunk_ready[j], (cnt_bits >> j) & 1);
           cnt_bits ^= 1u << j;
+          // remote chunk: pre-arm its next phase (its owner writes it again after this step's
+          // MMAs have completed, i.e. strictly after this arrive)
+          if (j / (P.NH / 64) != rank && s < NSTEPS - 1) mbar_arrive_expect_tx(&chunk_ready[j], RC_CHUNK);
           a_ptr = abuf + j * RC_CHUNK;
         }
         const int stg = it % NS;
         mbar_wait(&w_full[stg], (it / NS) & 1);
         tc_fence_after();
+        if (dbg && i == 0) dbg[1] = gtimer();
         const uint32_t a_base = smem_u32(a_ptr);
         const uint32_t b_base = smem_u32(ring + stg * STB);
         for (int kk = 0; kk < st.kkn; ++kk) {
@@ -241,27 +276,50 @@ __global__ void __launch_bounds__(RC_THREADS, 1) rowchain_kernel(const __grid_co
         umma_commit(&w_empty[stg]);
       }
       umma_commit(&acc_full[buf]);
-      if (CS > 1) umma_commit_multicast(peer_free, (uint16_t)(1u << peer));
+      if (CS > 1) umma_commit_multicast(peer_free, others);
+      if (dbg) dbg[2] = gtimer();
     }
   } else if (warp >= 4) {
     // ===== epilogue =====
     const int q = warp & 3;
-    const int h = (warp - 4) >> 2;
+    const int h = (warp - 4) >> 2;  // 32-column half of every chunk
     const int et = threadIdx.x - 128;
     const int rl = q * 32 + lane;
     const int grow = rb * 128 + rl;  // batch row
     const bool row_ok = grow < P.b;
     const int ncl = P.NH / 64;
     const int n = P.n;
+    const int64_t prow = (int64_t)rb * 4 + q;  // bias-gradient partial row of this quadrant
+    int nmy = 0;                               // this CTA's chunks that start below n
+    while (nmy < ncl && (rank * ncl + nmy) * 64 < n) ++nmy;
     for (int s = 0; s < NSTEPS; ++s) {
       const RcStep st = rc_step(P, s);
       const int buf = s & 1;
-      epi_bar_sync_n(RC_EPI_THREADS);  // red[] of the previous step consumed
+      const bool fwd = st.kind == RC_FWD;
+      const int lo = fwd ? st.layer : st.layer - 1;  // layer whose activation / gradient is produced
+      __nv_bfloat16* Sg = st.kind == RC_HEAD ? nullptr : P.S[lo];
+      if (fwd) {  // stage this CTA's bias columns of the layer (previous step's readers are done)
+        epi_bar_sync_n(RC_EPI_THREADS);
+        const int nn = rank * P.NH + et;
+        if (et < P.NH) sbias[et] = nn < n ? __ldg(P.bias[lo] + nn) : 0.f;
+        epi_bar_sync_n(RC_EPI_THREADS);
+      }
+      // dX: prefetch this row's sigma' (this warp's 32 columns of the first chunk) while the MMAs run
+      uint4 sv[4];
+#pragma unroll
+      for (int k = 0; k < 4; ++k) sv[k] = make_uint4(0, 0, 0, 0);
+      if (st.kind == RC_DX && row_ok && nmy > 0 && (rank * ncl + 1) * 64 <= n) {
+        const uint4* srow = reinterpret_cast<const uint4*>(Sg + (int64_t)grow * P.ldo + rank * ncl * 64 + h * 32);
+#pragma unroll
+        for (int k = 0; k < 4; ++k) sv[k] = __ldg(srow + k);
+      }
       mbar_wait(&acc_full[buf], (s >> 1) & 1);
       tc_fence_after();
-      if (CS > 1 && st.kind != RC_HEAD) mbar_wait_cluster(peer_free, s & 1);
-      if (lane == 0) tma_store_wait_read();  // this warp's earlier bulk stores no longer read abuf
-      __syncwarp();
+      unsigned long long* dbg =
+          P.dbg && s < RC_DBG_STEPS && et == 0 ? P.dbg + ((size_t)blockIdx.x * RC_DBG_STEPS + s) * RC_DBG_W : nullptr;
+      if (dbg) dbg[3] = gtimer();
+      if (CS > 1 && st.kind != RC_HEAD) mbar_wait(peer_free, s & 1);
+      if (dbg) dbg[4] = gtimer();
       const uint32_t tq = tmem_base + (uint32_t)(buf * P.NH) + ((uint32_t)(q * 32) << 16);
       if (st.kind == RC_HEAD) {
         // ---- softmax cross-entropy on the thread's row of logits (C <= 16) ----
@@ -293,9 +351,18 @@ __global__ void __launch_bounds__(RC_THREADS, 1) rowchain_kernel(const __grid_co
           uint32_t pk[8];
 #pragma unroll
           for (int j = 0; j < 8; ++j) pk[j] = pack_bf16x2(dz[2 * j], dz[2 * j + 1]);
-          uint8_t* row = hbuf + rl * 128;
-          *reinterpret_cast<uint4*>(row + ((0 ^ (rl & 7)) << 4)) = make_uint4(pk[0], pk[1], pk[2], pk[3]);
-          *reinterpret_cast<uint4*>(row + ((1 ^ (rl & 7)) << 4)) = make_uint4(pk[4], pk[5], pk[6], pk[7]);
+          // with a cluster the head chunk is never a TMA-store or bulk-copy source of this CTA
+          // (rc_head_chunk); alone, it is chunk 0, last stored by this warp
+          if (CS == 1) {
+            if (lane == 0) tma_store_wait_read();
+            __syncwarp();
+          }
+          const uint32_t row = smem_u32(abuf + hc * RC_CHUNK) + rl * 128;
+          sts128(row + ((0 ^ (rl & 7)) << 4), pk[0], pk[1], pk[2], pk[3]);
+          sts128(row + ((1 ^ (rl & 7)) << 4), pk[4], pk[5], pk[6], pk[7]);
+          fence_proxy_async();
+          __syncwarp();
+          if (lane == 0) mbar_arrive(head_ready);
           if (rank == 0) {
             if (row_ok) {
               P.row_loss[grow] = lse - zy;
@@ -304,68 +371,53 @@ __global__ void __launch_bounds__(RC_THREADS, 1) rowchain_kernel(const __grid_co
               if (P.ldo_head >= 16) D[1] = make_uint4(pk[4], pk[5], pk[6], pk[7]);
             }
             const float t = warp_colsum16(dz, lane);
-            if (!(lane & 1)) red[q * 256 + colsum16_col(lane)] = t;
+            const int col = colsum16_col(lane);
+            if (!(lane & 1) && col < C) P.bpart[P.L - 1][prow * C + col] = t;
           }
-          fence_proxy_async();
-          __syncwarp();
-          if (lane == 0) mbar_arrive(head_ready);
-        }
-        if (rank == 0) {
-          epi_bar_sync_n(RC_EPI_THREADS);
-          if (et < P.C)
-            P.bpart[P.L - 1][(int64_t)rb * P.C + et] = (red[et] + red[256 + et]) + (red[512 + et] + red[768 + et]);
         }
       } else {
-        const bool fwd = st.kind == RC_FWD;
-        const int lo = fwd ? st.layer : st.layer - 1;  // layer whose activation / gradient is produced
-        const bool signal = fwd || st.layer >= 2;       // the output is the next step's A operand
-        const float* bias = fwd ? P.bias[lo] : nullptr;
-        __nv_bfloat16* Sg = P.S[lo];
-        for (int c = h; c < ncl; c += 2) {
+        // this quadrant's TMA stores of the previous step (issued by its h = 0 warp) have read
+        // abuf before either half writes the pieces again
+        if (h == 0 && lane == 0) tma_store_wait_read();
+        quad_bar_sync(q);
+        const bool signal = fwd || st.layer >= 2;  // the output is the next step's A operand
+        for (int c = 0; c < nmy; ++c) {
           const int g = rank * ncl + c;
           const int n0 = g * 64;
-          if (n0 >= n) break;
-          uint8_t* piece = abuf + g * RC_CHUNK + q * RC_PIECE;
-          uint8_t* prow = piece + lane * 128;
-          // prefetch this row's sigma' stash for the chunk (dX)
+          const int nh = n0 + h * 32;  // first column of this warp's half
           const bool full_chunk = n0 + 64 <= n;
-          uint4 sv[8];
+          uint32_t raw[32];
+          tmem_ld_32x32b_x32(tq + (uint32_t)(c * 64 + h * 32), raw);
+          if (!fwd && c > 0 && row_ok && full_chunk) {  // sigma' of later chunks
+            const uint4* srow = reinterpret_cast<const uint4*>(Sg + (int64_t)grow * P.ldo + nh);
 #pragma unroll
-          for (int k = 0; k < 8; ++k) sv[k] = make_uint4(0, 0, 0, 0);
-          if (!fwd && row_ok && full_chunk) {
-            const uint4* srow = reinterpret_cast<const uint4*>(Sg + (int64_t)grow * P.ldo + n0);
-#pragma unroll
-            for (int k = 0; k < 8; ++k) sv[k] = __ldg(srow + k);
+            for (int k = 0; k < 4; ++k) sv[k] = __ldg(srow + k);
           }
+          tmem_ld_wait();
+          if (dbg && c == 0) dbg[6] = gtimer();
+          uint8_t* piece = abuf + g * RC_CHUNK + q * RC_PIECE;
+          const uint32_t prow_s = smem_u32(piece) + lane * 128;
+          const uint32_t sb_s = smem_u32(sbias) + (uint32_t)(c * 64 + h * 32) * 4;
 #pragma unroll
-          for (int gc = 0; gc < 4; ++gc) {
-            uint32_t raw[16];
-            tmem_ld_32x32b_x16(tq + (uint32_t)(c * 64 + gc * 16), raw);
-            tmem_ld_wait();
-            const int nc = n0 + gc * 16;
+          for (int g2 = 0; g2 < 2; ++g2) {
+            const int nc = nh + g2 * 16;
             uint32_t pk[8];
             if (fwd) {
               uint32_t sp[8];
               float bb[16];
-              if (nc + 16 <= n) {
-                const float4* b4 = reinterpret_cast<const float4*>(bias + nc);
 #pragma unroll
-                for (int k = 0; k < 4; ++k) {
-                  const float4 t = __ldg(b4 + k);
-                  bb[4 * k] = t.x;
-                  bb[4 * k + 1] = t.y;
-                  bb[4 * k + 2] = t.z;
-                  bb[4 * k + 3] = t.w;
-                }
-              } else {
-#pragma unroll
-                for (int k = 0; k < 16; ++k) bb[k] = nc + k < n ? __ldg(bias + nc + k) : 0.f;
+              for (int k = 0; k < 4; ++k) {
+                const float4 t = lds128f(sb_s + (uint32_t)(g2 * 16 + 4 * k) * 4);
+                bb[4 * k] = t.x;
+                bb[4 * k + 1] = t.y;
+                bb[4 * k + 2] = t.z;
+                bb[4 * k + 3] = t.w;
               }
 #pragma unroll
               for (int k = 0; k < 8; ++k) {
                 float h0, d0, h1, d1;
-                sigmoid_d(__uint_as_float(raw[2 * k]) + bb[2 * k], h0, d0);
-                sigmoid_d(__uint_as_float(raw[2 * k + 1]) + bb[2 * k + 1], h1, d1);
+                sigmoid_d(__uint_as_float(raw[g2 * 16 + 2 * k]) + bb[2 * k], h0, d0);
+                sigmoid_d(__uint_as_float(raw[g2 * 16 + 2 * k + 1]) + bb[2 * k + 1], h1, d1);
                 pk[k] = pack_bf16x2(h0, h1);
                 sp[k] = pack_bf16x2(d0, d1);
               }
@@ -383,57 +435,60 @@ __global__ void __launch_bounds__(RC_THREADS, 1) rowchain_kernel(const __grid_co
             } else {
               float v[16];
               if (full_chunk) {
-                const uint32_t sw[8] = {sv[2 * gc].x, sv[2 * gc].y, sv[2 * gc].z, sv[2 * gc].w,
-                                        sv[2 * gc + 1].x, sv[2 * gc + 1].y, sv[2 * gc + 1].z, sv[2 * gc + 1].w};
+                const uint32_t sw[8] = {sv[2 * g2].x,     sv[2 * g2].y,     sv[2 * g2].z,     sv[2 * g2].w,
+                                        sv[2 * g2 + 1].x, sv[2 * g2 + 1].y, sv[2 * g2 + 1].z, sv[2 * g2 + 1].w};
 #pragma unroll
                 for (int k = 0; k < 8; ++k) {
                   const float2 a = __bfloat1622float2(*reinterpret_cast<const __nv_bfloat162*>(&sw[k]));
-                  v[2 * k] = __uint_as_float(raw[2 * k]) * a.x;
-                  v[2 * k + 1] = __uint_as_float(raw[2 * k + 1]) * a.y;
+                  v[2 * k] = __uint_as_float(raw[g2 * 16 + 2 * k]) * a.x;
+                  v[2 * k + 1] = __uint_as_float(raw[g2 * 16 + 2 * k + 1]) * a.y;
                 }
               } else {  // ragged last chunk: columns >= n are zero
                 const __nv_bfloat16* srow = Sg + (int64_t)grow * P.ldo + nc;
 #pragma unroll
                 for (int k = 0; k < 16; ++k)
-                  v[k] = (row_ok && nc + k < n) ? __uint_as_float(raw[k]) * __bfloat162float(srow[k]) : 0.f;
+                  v[k] = (row_ok && nc + k < n) ? __uint_as_float(raw[g2 * 16 + k]) * __bfloat162float(srow[k]) : 0.f;
               }
 #pragma unroll
               for (int k = 0; k < 8; ++k) pk[k] = pack_bf16x2(v[2 * k], v[2 * k + 1]);
+              // bias-gradient partial of this quadrant's 32 rows (deterministic, reduced by the dW GEMM)
               const float t = warp_colsum16(v, lane);
-              if (!(lane & 1)) red[q * 256 + c * 64 + gc * 16 + colsum16_col(lane)] = t;
+              const int col = nc + colsum16_col(lane);
+              if (!(lane & 1) && col < n) P.bpart[lo][prow * n + col] = t;
             }
-            const int j0 = gc * 2;
-            *reinterpret_cast<uint4*>(prow + ((j0 ^ (lane & 7)) << 4)) = make_uint4(pk[0], pk[1], pk[2], pk[3]);
-            *reinterpret_cast<uint4*>(prow + (((j0 + 1) ^ (lane & 7)) << 4)) = make_uint4(pk[4], pk[5], pk[6], pk[7]);
+            const int j0 = h * 4 + g2 * 2;  // 16-byte column chunk of the 128-byte row
+            sts128(prow_s + ((j0 ^ (lane & 7)) << 4), pk[0], pk[1], pk[2], pk[3]);
+            sts128(prow_s + (((j0 + 1) ^ (lane & 7)) << 4), pk[4], pk[5], pk[6], pk[7]);
           }
+          if (dbg && c == 0) dbg[7] = gtimer();
           fence_proxy_async();
-          __syncwarp();
-          if (lane == 0) {
-            tma_store_2d(fwd ? &P.mH[lo] : &P.mDZ[lo], piece, n0, rb * 128 + q * 32);
-            if (signal) {
-              if (CS > 1) {
-                const uint32_t rbar = mapa_shared(smem_u32(&chunk_ready[g]), peer);
-                mbar_arrive_expect_tx_remote(rbar, RC_PIECE);
-                bulk_copy_s2cluster(mapa_shared(smem_u32(piece), peer), piece, RC_PIECE, rbar);
+          quad_bar_sync(q);  // both halves of the piece are written
+          if (h == 0) {
+            // lane p ships the piece to CTA p (remote ops issued in parallel); lane `rank` stores
+            // the piece to global and arrives locally
+            if (lane == 0) {
+              tma_store_2d(fwd ? &P.mH[lo] : &P.mDZ[lo], piece, n0, rb * 128 + q * 32);
+              if (signal) {
+                // the receivers pre-armed their chunk_ready[g] with expect_tx (MMA thread), so a
+                // remote piece needs nothing but the bulk copy and its complete_tx
+                for (int p = 1; p < CS; ++p) {
+                  const int dst = (rank + p) % CS;
+                  bulk_copy_s2cluster(mapa_shared(smem_u32(piece), dst), piece, RC_PIECE,
+                                      mapa_shared(smem_u32(&chunk_ready[g]), dst));
+                }
+                mbar_arrive(&chunk_ready[g]);
               }
-              mbar_arrive(&chunk_ready[g]);
             }
           }
+          if (dbg) dbg[c == 0 ? 8 : 9] = gtimer();
         }
-        if (lane == 0) tma_store_commit();
-        if (!fwd) {  // bias-gradient partials of dZ_lo for this row block
-          epi_bar_sync_n(RC_EPI_THREADS);
-          for (int cc = et; cc < P.NH; cc += RC_EPI_THREADS) {
-            const int nn = rank * P.NH + cc;
-            if (nn < n)
-              P.bpart[lo][(int64_t)rb * n + nn] = (red[cc] + red[256 + cc]) + (red[512 + cc] + red[768 + cc]);
-          }
-        }
+        if (h == 0 && lane == 0) tma_store_commit();
       }
       // release the accumulator (all TMEM reads of this warp have completed)
       tc_fence_before();
       __syncwarp();
       if (lane == 0) mbar_arrive(&acc_empty[buf]);
+      if (dbg) dbg[5] = gtimer();
     }
     if (lane == 0) tma_store_wait_all();
   }

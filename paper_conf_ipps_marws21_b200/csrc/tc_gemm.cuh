@@ -96,6 +96,43 @@ __device__ __forceinline__ int colsum16_col(int lane) {
   return ((lane >> 4) & 1) * 8 + ((lane >> 3) & 1) * 4 + ((lane >> 2) & 1) * 2 + ((lane >> 1) & 1);
 }
 
+// Bias gradient of rows [lo, hi): db[bi] = sum_t part[t * ldp + bi] over the n_mtiles partial rows
+// written by the dZ producer, then b -= lr * db (SGD) or db stored (grads).  The 256 epilogue
+// threads split the work: tpr adjacent lanes per bias entry, each summing every tpr-th partial
+// row with 8 independent accumulators (loads in flight), combined in a fixed butterfly order —
+// deterministic, and no long chain of dependent L2 loads on the tail of the dW GEMM.
+template <int EPI>
+__device__ __forceinline__ void bias_reduce_update(const EpiArgs& ep, int lo, int hi, int tid) {
+  const int R = hi - lo;
+  if (R <= 0) return;  // CTA-uniform
+  int tpr = 1;
+  while (tpr < 32 && tpr * 2 * R <= TC_EPI_THREADS) tpr *= 2;
+  const int r = tid / tpr, k = tid % tpr;
+  const int nt = ep.n_mtiles;
+  float acc = 0.f;
+  if (r < R) {
+    const float* col = ep.bpart_in + lo + r;
+    float a[8];
+#pragma unroll
+    for (int u = 0; u < 8; ++u) a[u] = 0.f;
+    int t = k;
+    for (; t + 7 * tpr < nt; t += 8 * tpr) {
+#pragma unroll
+      for (int u = 0; u < 8; ++u) a[u] += __ldcg(col + (int64_t)(t + u * tpr) * ep.ldp);
+    }
+    for (; t < nt; t += tpr) a[0] += __ldcg(col + (int64_t)t * ep.ldp);
+    acc = ((a[0] + a[1]) + (a[2] + a[3])) + ((a[4] + a[5]) + (a[6] + a[7]));
+  }
+  for (int o = 1; o < tpr; o <<= 1) acc += __shfl_xor_sync(0xffffffffu, acc, o);
+  if (r < R && k == 0) {
+    const int bi = lo + r;
+    if (EPI == EPI_WGRAD_SGD)
+      ep.bias_upd[bi] -= ep.lr * acc;
+    else
+      ep.bias_grad[bi] = acc;
+  }
+}
+
 // Grouped tile rasterisation: consecutive tile indices walk down GROUP_M row tiles before moving
 // to the next column tile, so the ~148 tiles resident at once cover a compact block of the
 // output and share both their A row panels and their B column panels through L2.
@@ -569,17 +606,9 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
         // non-transposed: the n-tile-0 CTA owns bias rows m0..m0+127;
         // transposed (small head): the m-tile-0 CTA owns bias entries n0..n0+BN-1
         const bool own = !ep.transposed ? (n_tile == 0) : (m_tile == 0);
-        const int lo = !ep.transposed ? m0 + et : n0 + et;
+        const int lo = !ep.transposed ? m0 : n0;
         const int hi = !ep.transposed ? min(ep.M, m0 + TC_BM) : min(ep.N, n0 + BN);
-        if (own)
-          for (int bi = lo; bi < hi; bi += TC_EPI_THREADS) {
-            float sdb = 0.f;
-            for (int t = 0; t < ep.n_mtiles; ++t) sdb += ep.bpart_in[(int64_t)t * ep.ldp + bi];
-            if (EPI == EPI_WGRAD_SGD)
-              ep.bias_upd[bi] -= ep.lr * sdb;
-            else
-              ep.bias_grad[bi] = sdb;
-          }
+        if (own) bias_reduce_update<EPI>(ep, lo, hi, et);
       }
     }
     // release this accumulator to the MMA warp (all TMEM reads of the tile have completed)
@@ -636,22 +665,14 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
         bool own;
         if (!ep.transposed) {
           own = n_tile == 0;
-          lo = m0 + kz * rps + tid;
+          lo = m0 + kz * rps;
           hi = min(ep.M, m0 + (kz + 1) * rps);
         } else {
           own = m_tile == 0 && kz == 0;
-          lo = n0 + tid;
+          lo = n0;
           hi = min(ep.N, n0 + BN);
         }
-        if (own)
-          for (int bi = lo; bi < hi; bi += TC_EPI_THREADS) {
-            float sdb = 0.f;
-            for (int t = 0; t < ep.n_mtiles; ++t) sdb += ep.bpart_in[(int64_t)t * ep.ldp + bi];
-            if (EPI == EPI_WGRAD_SGD)
-              ep.bias_upd[bi] -= ep.lr * sdb;
-            else
-              ep.bias_grad[bi] = sdb;
-          }
+        if (own) bias_reduce_update<EPI>(ep, lo, hi, tid);
       }
     }
   }

@@ -1,0 +1,5 @@
+#!/bin/bash
+mkdir -p gpurun_out
+timeout -s KILL 300 ncu --set full --import-source on --clock-control none -k regex:rowchain -s 2 -c 1 \
+  -o gpurun_out/rc_full_8192 -f python scripts/rc_one.py 8192 > gpurun_out/ncu_rc.log 2>&1
+echo "ncu rc=$?"; tail -3 gpurun_out/ncu_rc.log

@@ -27,17 +27,19 @@ def _need_gpu():
 
 
 CASES = [
-    # dims, dataset kind, batch, expected CTAs per row block
+    # dims, dataset kind, batch, expected CTAs per row block (widest of 1/2/4/8 with >= 64
+    # columns per CTA whose clusters still fill the 148 SMs in one wave)
     ([54, 64, 64, 7], "covtype", 32, 1),
     ([54, 64, 64, 7], "covtype", 1, 1),
     ([24, 40, 3], "gauss", 77, 1),
-    ([54, 128, 128, 7], "covtype", 4096, 1),
-    ([54, 512, 512, 7], "covtype", 1000, 2),
-    ([54, 200, 200, 200, 7], "covtype", 129, 2),
+    ([54, 128, 128, 7], "covtype", 4096, 2),
+    ([54, 512, 512, 7], "covtype", 1000, 8),
+    ([54, 200, 200, 200, 7], "covtype", 129, 4),
     ([300, 300, 300, 2], "w8a", 333, 2),
-    ([54, 512, 7], "covtype", 256, 2),
-    ([300] + [512] * 8 + [2], "w8a", 200, 2),
-    ([64, 256, 256, 16], "gauss", 500, 2),
+    ([54, 512, 7], "covtype", 256, 8),
+    ([300] + [512] * 8 + [2], "w8a", 200, 8),
+    ([64, 256, 256, 16], "gauss", 500, 4),
+    ([54, 512, 512, 512, 512, 7], "covtype", 4096, 4),
     ([54, 512, 512, 512, 512, 7], "covtype", 8192, 2),
 ]
 
@@ -50,7 +52,8 @@ def test_fused_gradients_match_oracle(dims, kind, b, cs):
     if dims[-1] > 2:
         y = np.random.default_rng(5).integers(0, dims[-1], b).astype(np.int32)
     m = hb.MLP(dims, precision="bf16", seed=0)
-    assert m.fused_path() == cs
+    m.set_fused_min_batch(1)  # exercise the fused kernel at every batch size
+    assert m.fused_path(b) == cs
     params = init_params(dims, seed=2)
     m.set_params(params_to_flat(params))
     w = hb.Worker(m, b)
@@ -70,7 +73,8 @@ def test_fused_steps_track_oracle_trajectory():
     dims, b, steps, lr = [54, 512, 512, 7], 512, 30, 0.5
     X, y = dataset("covtype", b * steps, seed=4)
     m = hb.MLP(dims, precision="bf16", seed=0)
-    assert m.fused_path() == 2
+    m.set_fused_min_batch(1)
+    assert m.fused_path(b) == 8
     params = init_params(dims, seed=2)
     m.set_params(params_to_flat(params))
     w = hb.Worker(m, b)
@@ -93,6 +97,8 @@ def test_fused_saturated_init():
     dims, b = [54, 512, 512, 512, 512, 7], 384
     X, y = dataset("covtype", b, seed=8)
     m = hb.MLP(dims, precision="bf16", seed=0)
+    m.set_fused_min_batch(1)
+    assert m.fused_path(b) > 0
     params = init_params(dims, seed=2, scale=4.0)
     m.set_params(params_to_flat(params))
     w = hb.Worker(m, b)
@@ -105,8 +111,51 @@ def test_fused_saturated_init():
         assert rel_err(got[l][1], db[l]) <= TOL, l
 
 
+_FORCED_CS_SCRIPT = r"""
+import os, sys, json
+sys.path.insert(0, os.getcwd())
+import numpy as np
+import paper_conf_ipps_marws21_b200 as hb
+from oracle import mlp64
+from tests.helpers import dataset, init_params, params_to_flat, rel_err, split_flat, to_device
+dims, b = [54, 256, 256, 7], 300
+X, y = dataset("covtype", b, seed=13)
+m = hb.MLP(dims, precision="bf16", seed=0)
+m.set_fused_min_batch(1)
+params = init_params(dims, seed=2)
+m.set_params(params_to_flat(params))
+w = hb.Worker(m, b)
+tX, ty = to_device(X, y)
+g, loss = w.step_grads(tX, ty, b)
+dW, db, l_ref = mlp64.grads(params, X.astype(np.float64), y)
+got = split_flat(g, dims)
+err = max(max(rel_err(got[l][0], dW[l]), rel_err(got[l][1], db[l])) for l in range(len(dims) - 1))
+print(json.dumps({"cs": m.fused_path(b), "err": err, "lerr": abs(loss - l_ref) / l_ref}))
+"""
+
+
+@pytest.mark.parametrize("cs", [1, 2, 4, 8])
+def test_every_cluster_size_matches_oracle(cs):
+    # the same 256-wide net at every cluster size (HB_RC_CS), each in a fresh process; at CS = 8
+    # the last four CTAs of every cluster own no valid column (n = 256 < 8 x 64 chunks)
+    import json, os, subprocess, sys
+    _need_gpu()
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    env = dict(os.environ, HB_RC_CS=str(cs))
+    out = subprocess.run([sys.executable, "-c", _FORCED_CS_SCRIPT], cwd=root, env=env, capture_output=True,
+                         text=True, timeout=300)
+    assert out.returncode == 0, out.stderr[-2000:]
+    r = json.loads(out.stdout.strip().splitlines()[-1])
+    assert r["cs"] == cs
+    assert r["err"] <= TOL and r["lerr"] <= TOL, r
+
+
 def test_unfused_shapes_report_layer_chain():
     _need_gpu()
+    m = hb.MLP([54, 512, 512, 7])
+    assert m.fused_path(8192) == 2 and m.fused_path(4096) == 0   # default crossover b = 8192
+    m.set_fused_min_batch(0)
+    assert m.fused_path(8192) == 0
     assert hb.MLP([54, 1024, 1024, 7]).fused_path() == 0     # n > 512
     assert hb.MLP([54, 128, 64, 7]).fused_path() == 0        # non-uniform hidden widths
     assert hb.MLP([64, 96, 40]).fused_path() == 0            # C > 16
