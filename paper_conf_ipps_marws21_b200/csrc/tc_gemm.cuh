@@ -502,15 +502,17 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
               spre[i][1] = spre[i + 1][1];
             }
           } else if ((EPI == EPI_WGRAD_SGD || EPI == EPI_WGRAD_STORE) && splits > 1) {
-            // split-K: park the fp32 partial tile; reduced after the cluster barrier below
-            float4* wsp = reinterpret_cast<float4*>(
-                ep.ws + ((((size_t)t) * splits + kz) * TC_BM + rl) * BN + c);
+            // split-K: park the fp32 partial tile in this CTA's (now idle) stage ring, row stride
+            // BN + 4 floats (conflict-free row-per-lane writes); the cluster reduces it over DSMEM
             if (num_kb == 0) {
 #pragma unroll
               for (int j = 0; j < 16; ++j) v[j] = 0.f;
             }
+            const uint32_t pa = smem_u32(smem) + (uint32_t)((rl * (BN + 4) + c) * 4);
 #pragma unroll
-            for (int qq = 0; qq < 4; ++qq) wsp[qq] = make_float4(v[4 * qq], v[4 * qq + 1], v[4 * qq + 2], v[4 * qq + 3]);
+            for (int qq = 0; qq < 4; ++qq)
+              sts128(pa + qq * 16, __float_as_uint(v[4 * qq]), __float_as_uint(v[4 * qq + 1]),
+                     __float_as_uint(v[4 * qq + 2]), __float_as_uint(v[4 * qq + 3]));
           } else if (TO::on && EPI == EPI_FWD_SIG) {
             // all rows / columns staged; rows >= M and columns >= N are clipped by the TMA store
             uint32_t hp[8], sp[8];
@@ -620,9 +622,10 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
 
   if ((EPI == EPI_WGRAD_SGD || EPI == EPI_WGRAD_STORE) && splits > 1) {
     // ---- split-K reduce-scatter: CTA kz of the cluster reduces rows [kz*rps, (kz+1)*rps) of the
-    //      tile over the `splits` partials in fixed order and applies the fused SGD update ----
-    __threadfence();
-    cluster_sync_all();
+    //      tile over the `splits` partials (read from every CTA's shared memory, fixed order) and
+    //      applies the fused SGD update ----
+    static_assert(TC_BM * (BN + 4) * 4 <= Cfg::STAGES * Cfg::STAGE_BYTES, "split-K tile must fit the ring");
+    cluster_sync_all();  // every partial tile is in shared memory (release/acquire, cluster scope)
     if (warp >= 4) {
       const int t = t_first;
       int m_tile, n_tile;
@@ -630,12 +633,13 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
       const int m0 = m_tile * TC_BM, n0 = n_tile * BN;
       const int tid = threadIdx.x - 128;  // 0..255
       const int rps = TC_BM / splits;
-      const size_t tile_base = (size_t)t * splits * TC_BM * BN;
+      const uint32_t tile_s = smem_u32(smem);
       for (int e = tid * 4; e < rps * BN; e += TC_EPI_THREADS * 4) {
         const int rloc = kz * rps + e / BN, col = e % BN;
+        const uint32_t off = (uint32_t)((rloc * (BN + 4) + col) * 4);
         float4 acc = make_float4(0.f, 0.f, 0.f, 0.f);
         for (int sp = 0; sp < splits; ++sp) {
-          const float4 t = *reinterpret_cast<const float4*>(ep.ws + tile_base + ((size_t)sp * TC_BM + rloc) * BN + col);
+          const float4 t = ld_dsmem_f4(mapa_shared(tile_s + off, (uint32_t)sp));
           acc.x += t.x;
           acc.y += t.y;
           acc.z += t.z;
@@ -675,6 +679,7 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
         if (own) bias_reduce_update<EPI>(ep, lo, hi, tid);
       }
     }
+    cluster_sync_all();  // no CTA leaves while another still reads its partial tile
   }
 
   if (TO::on && threadIdx.x == 128) tma_store_wait_all();  // bulk stores complete before exit
