@@ -467,6 +467,8 @@ static int launch_rowchain(hb_worker* w, const RcCfg& c, const void* X, int64_t 
   P.nstages = c.NS;
   P.abuf_chunks = c.NCA;
   P.tmem_cols = c.tmem;
+  static const int korder = env_int("HB_RC_KORDER", 0);  // 1 measured slower (B200, C2 b = 8192: 103 vs 88 us)
+  P.korder = korder;
   P.inv_b = 1.0f / (float)b;
   P.dbg = g_rc_trace;
   int dev = 0;
@@ -889,9 +891,15 @@ static int run_step_rowchain(hb_worker* w, const RcCfg& c, const void* X, int64_
     static const int fbn = env_int("HB_RC_WGRAD_BN", 0), fs = env_int("HB_RC_WGRAD_S", 0);
     const Layer& Ly = m->layers[l];
     const bool wide = Ly.n_out >= 128 || Ly.n_out >= Ly.n_in;  // not the transposed small head
+    // the L GEMMs share the SMs, so each takes wide tiles (fewer L2 re-reads of dZ / H) and a
+    // short split: measured on B200 (scripts/gpu_dw_sweep.sh, C2 b = 8192) BN 256 x 4 splits
+    // 32 us vs 59 us for the standalone choice (BN 64 x 4)
+    const int bn = fbn ? fbn : Ly.n_in <= 64 ? 64 : Ly.n_in <= 128 ? 128 : 256;
+    int sp = fs ? fs : b >= 1024 ? 4 : 2;
+    while (sp > 1 && sp > (b + TC_BK - 1) / TC_BK) sp /= 2;  // at least one k-block per split
     int rc = launch_wgrad(w, l, X, ldx, x_rows, d_off, b, lr, grads_only, w->sdw[l], w->ws_l[l],
                           4 * ((b + 127) / 128),  // per-quadrant bias partials of the chain
-                          wide ? fbn : 0, wide ? fs : 0);
+                          wide ? bn : 0, wide ? sp : 0);
     if (rc) return rc;
     HB_CUDA_TRY(cudaEventRecord(w->ev_dw[l], w->sdw[l]));
   }

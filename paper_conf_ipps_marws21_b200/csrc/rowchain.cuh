@@ -76,6 +76,7 @@ struct RcParams {
   int L, n0, n, C, b;
   int CS, NH;                    // cluster size, output columns per CTA (multiple of 64)
   int nstages, abuf_chunks, tmem_cols;
+  int korder;                    // k-block order of chunked steps (rc_kchunk)
   float inv_b;
   unsigned long long* dbg;       // tuning only: per CTA, per step RC_DBG_W globaltimer stamps (nullable)
 };
@@ -117,11 +118,22 @@ __device__ __forceinline__ RcStep rc_step(const RcParams& P, int s) {
   return st;
 }
 
-// k-block i of step s reads abuf chunk rc_kchunk(...): this CTA's own chunks first (its epilogue
-// produced them, they are ready before the others arrive), then the others in index order.
+// k-block i of step s reads abuf chunk rc_kchunk(...).  korder 0: this CTA's own chunks first
+// (its epilogue produced them, they are ready before the others arrive), then the others in index
+// order.  korder 1: round robin over the cluster starting with this CTA (own c0, next CTA's c0, ...,
+// own c1, ...): every CTA's epilogue emits its chunks in the same order at about the same time, so
+// the MMAs (and the W ring behind them) keep pace with the epilogues instead of leaving all remote
+// k-blocks — more W stages than the ring holds — for after the last chunk.
 __device__ __forceinline__ int rc_kchunk(const RcParams& P, int s, int nkb, int i, int rank) {
   if (s == 0 || s == P.L) return i;
   const int ncl = P.NH / 64;
+  if (P.korder == 1) {
+    for (int t = 0, v = 0; t < P.CS * ncl; ++t) {
+      const int g = ((rank + t % P.CS) % P.CS) * ncl + t / P.CS;
+      if (g < nkb && v++ == i) return g;
+    }
+    return i;  // unreachable for i < nkb
+  }
   const int lo = rank * ncl, hi = min(lo + ncl, nkb);
   const int nown = max(0, hi - lo);
   if (i < nown) return lo + i;
@@ -242,8 +254,11 @@ __global__ void __launch_bounds__(RC_THREADS, 1) rowchain_kernel(const __grid_co
       if (dbg) dbg[0] = gtimer();
       const uint32_t tacc = tmem_base + (uint32_t)(buf * P.NH);
       const uint32_t idesc = make_idesc_bf16(128, st.N, false, st.bmn);
+      // tuning only: per-k-block stamps of step 2 (issue, chunk ready, W ready) after the step table
+      unsigned long long* kdbg = P.dbg && s == 2 ? P.dbg + (size_t)gridDim.x * RC_DBG_STEPS * RC_DBG_W : nullptr;
       for (int i = 0; i < st.nkb; ++i, ++it) {
         const int j = rc_kchunk(P, s, st.nkb, i, rank);
+        if (kdbg && i < 16) kdbg[blockIdx.x * 16 + i] = gtimer();
         uint8_t* a_ptr;
         if (s == 0) {
           if (i == 0) mbar_wait(x_full, 0);
@@ -261,9 +276,11 @@ __global__ void __launch_bounds__(RC_THREADS, 1) rowchain_kernel(const __grid_co
           if (j / (P.NH / 64) != rank && s < NSTEPS - 1) mbar_arrive_expect_tx(&chunk_ready[j], RC_CHUNK);
           a_ptr = abuf + j * RC_CHUNK;
         }
+        if (kdbg && i < 16) kdbg[(gridDim.x + blockIdx.x) * 16 + i] = gtimer();
         const int stg = it % NS;
         mbar_wait(&w_full[stg], (it / NS) & 1);
         tc_fence_after();
+        if (kdbg && i < 16) kdbg[(2 * gridDim.x + blockIdx.x) * 16 + i] = gtimer();
         if (dbg && i == 0) dbg[1] = gtimer();
         const uint32_t a_base = smem_u32(a_ptr);
         const uint32_t b_base = smem_u32(ring + stg * STB);
@@ -388,10 +405,15 @@ __global__ void __launch_bounds__(RC_THREADS, 1) rowchain_kernel(const __grid_co
           const bool full_chunk = n0 + 64 <= n;
           uint32_t raw[32];
           tmem_ld_32x32b_x32(tq + (uint32_t)(c * 64 + h * 32), raw);
-          if (!fwd && c > 0 && row_ok && full_chunk) {  // sigma' of later chunks
-            const uint4* srow = reinterpret_cast<const uint4*>(Sg + (int64_t)grow * P.ldo + nh);
+          // sigma' of the NEXT chunk: its global load overlaps this chunk's work (chunk 0's was
+          // issued before the accumulator wait)
+          uint4 svn[4];
 #pragma unroll
-            for (int k = 0; k < 4; ++k) sv[k] = __ldg(srow + k);
+          for (int k = 0; k < 4; ++k) svn[k] = make_uint4(0, 0, 0, 0);
+          if (!fwd && c + 1 < nmy && row_ok && n0 + 128 <= n) {
+            const uint4* srow = reinterpret_cast<const uint4*>(Sg + (int64_t)grow * P.ldo + nh + 64);
+#pragma unroll
+            for (int k = 0; k < 4; ++k) svn[k] = __ldg(srow + k);
           }
           tmem_ld_wait();
           if (dbg && c == 0) dbg[6] = gtimer();
@@ -416,12 +438,23 @@ __global__ void __launch_bounds__(RC_THREADS, 1) rowchain_kernel(const __grid_co
 #pragma unroll
               for (int k = 0; k < 8; ++k) {
                 float h0, d0, h1, d1;
+#ifdef HB_RC_FAKE_SIG  // tuning only (wrong numerics): epilogue cost without the MUFU work
+                h0 = __uint_as_float(raw[g2 * 16 + 2 * k]) + bb[2 * k];
+                h1 = __uint_as_float(raw[g2 * 16 + 2 * k + 1]) + bb[2 * k + 1];
+                d0 = h0 * 0.25f;
+                d1 = h1 * 0.25f;
+#else
                 sigmoid_d(__uint_as_float(raw[g2 * 16 + 2 * k]) + bb[2 * k], h0, d0);
                 sigmoid_d(__uint_as_float(raw[g2 * 16 + 2 * k + 1]) + bb[2 * k + 1], h1, d1);
+#endif
                 pk[k] = pack_bf16x2(h0, h1);
                 sp[k] = pack_bf16x2(d0, d1);
               }
+#ifdef HB_RC_NO_S_STORE  // tuning only (wrong numerics): epilogue cost without the sigma' stash stores
+              if (false) {
+#else
               if (row_ok) {
+#endif
                 __nv_bfloat16* srow = Sg + (int64_t)grow * P.ldo + nc;
                 if (nc + 16 <= n) {
                   reinterpret_cast<uint4*>(srow)[0] = make_uint4(sp[0], sp[1], sp[2], sp[3]);
@@ -481,6 +514,8 @@ __global__ void __launch_bounds__(RC_THREADS, 1) rowchain_kernel(const __grid_co
             }
           }
           if (dbg) dbg[c == 0 ? 8 : 9] = gtimer();
+#pragma unroll
+          for (int k = 0; k < 4; ++k) sv[k] = svn[k];
         }
         if (h == 0 && lane == 0) tma_store_commit();
       }

@@ -54,9 +54,9 @@ if m.fused_path():
         tail = raw[nct * 24 * 10: nct * 24 * 10 + 3 * nct * 16].reshape(3, nct, 16)
         for ci in range(min(2, nct)):
             iss, crdy, wrdy = tail[0, ci, :8], tail[1, ci, :8], tail[2, ci, :8]
-            print(f"   cta{ci} step2 k-blocks: issue->W-ready us", [round(float(w_ - i_) / 1000, 2) for i_, w_ in zip(iss, wrdy)],
-                  " chunk-ready->W-ready us", [round(float(w_ - c_) / 1000, 2) for c_, w_ in zip(crdy, wrdy)],
-                  " issue times", [round(float(i_ - t0) / 1000, 2) for i_ in iss])
+            rel = lambda v: [round(float(x - t0) / 1000, 2) for x in v]
+            print(f"   cta{ci} step2 k-blocks (us from kernel start): issue {rel(iss)}\n"
+                  f"        chunk ready {rel(crdy)}\n        W ready     {rel(wrdy)}")
         print(f"--- b={b}: {len(ctas)} CTAs, span {(a[a > 0].max() - t0) / 1000:.2f} us; per step (median over CTAs, us from kernel start):")
         print("   step  mma_start  first_w  mma_issued  epi_acc  epi_peer  epi_end  ld0  c0comp  c0sig  c1sig")
         for s in range(2 * L - 1):
