@@ -284,4 +284,19 @@ __device__ __forceinline__ void sigmoid_d(float z, float& h, float& d) {
   d = es * s;
 }
 
+// Tensor-core epilogues: the same formulas with ONE MUFU op per element (ex2).  1/(1+e), 1+e in
+// (1, 2], starts from the minimax line 24/17 - 8/17 y (relative error <= 1/17) and takes two
+// Newton steps s <- s (2 - y s) on the FMA pipe (error 1/17 -> 3.5e-3 -> 1.2e-5, far below the
+// bf16 rounding of H and S).  The fp32 check mode keeps sigmoid_d.
+__device__ __forceinline__ void sigmoid_d_fast(float z, float& h, float& d) {
+  const float e = __expf(-fabsf(z));
+  const float y = 1.0f + e;
+  float s = fmaf(-8.0f / 17.0f, y, 24.0f / 17.0f);
+  s = s * fmaf(-y, s, 2.0f);
+  s = s * fmaf(-y, s, 2.0f);
+  const float es = e * s;
+  h = z >= 0.f ? s : es;
+  d = es * s;
+}
+
 }  // namespace hb

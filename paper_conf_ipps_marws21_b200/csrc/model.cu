@@ -419,7 +419,9 @@ static RcCfg rowchain_cfg(const hb_model* m, int b = 8192) {
   const int stb = c.NH * 128;
   // 1 KB alignment slack + abuf + W ring + staged bias (1 KB) + mbarriers
   const int fixed = 1024 + c.NCA * RC_CHUNK + 1024 + 8 * (2 * RC_MAX_STAGES + c.NCA + 8) + 16;
+  static const int ns_env = env_int("HB_RC_NS", 0);  // tuning only: force the W ring depth
   c.NS = std::min(RC_MAX_STAGES, (RC_SMEM_CAP - fixed) / stb);
+  if (ns_env >= 2 && ns_env < c.NS) c.NS = ns_env;
   if (c.NS < 2) return c;
   c.smem = 1024 + c.NCA * RC_CHUNK + c.NS * stb + 1024 + 8 * (2 * c.NS + c.NCA + 8) + 16;
   c.tmem = 64;
@@ -893,13 +895,14 @@ static int run_step_rowchain(hb_worker* w, const RcCfg& c, const void* X, int64_
     const bool wide = Ly.n_out >= 128 || Ly.n_out >= Ly.n_in;  // not the transposed small head
     // the L GEMMs share the SMs, so each takes wide tiles (fewer L2 re-reads of dZ / H) and a
     // short split: measured on B200 (scripts/gpu_dw_sweep.sh, C2 b = 8192) BN 256 x 4 splits
-    // 32 us vs 59 us for the standalone choice (BN 64 x 4)
+    // 32 us vs 59 us for the standalone choice (BN 64 x 4).  Every GEMM uses clusters of <= 4 so
+    // that all of them are co-resident (B200: 33 clusters of 4 x 200 KB CTAs at once)
     const int bn = fbn ? fbn : Ly.n_in <= 64 ? 64 : Ly.n_in <= 128 ? 128 : 256;
     int sp = fs ? fs : b >= 1024 ? 4 : 2;
     while (sp > 1 && sp > (b + TC_BK - 1) / TC_BK) sp /= 2;  // at least one k-block per split
     int rc = launch_wgrad(w, l, X, ldx, x_rows, d_off, b, lr, grads_only, w->sdw[l], w->ws_l[l],
                           4 * ((b + 127) / 128),  // per-quadrant bias partials of the chain
-                          wide ? bn : 0, wide ? sp : 0);
+                          wide ? bn : 0, sp);  // the small head keeps its BN 16 tiles, 4 splits
     if (rc) return rc;
     HB_CUDA_TRY(cudaEventRecord(w->ev_dw[l], w->sdw[l]));
   }

@@ -118,7 +118,8 @@ __device__ __forceinline__ RcStep rc_step(const RcParams& P, int s) {
   return st;
 }
 
-// k-block i of step s reads abuf chunk rc_kchunk(...).  korder 0: this CTA's own chunks first
+// k-block i of step s reads abuf chunk rc_kchunk(...).  korder 2: own chunk t, then the other
+// CTAs' chunks t-1 (a remote chunk arrives about one epilogue chunk after the local one).  korder 0: this CTA's own chunks first
 // (its epilogue produced them, they are ready before the others arrive), then the others in index
 // order.  korder 1: round robin over the cluster starting with this CTA (own c0, next CTA's c0, ...,
 // own c1, ...): every CTA's epilogue emits its chunks in the same order at about the same time, so
@@ -127,6 +128,21 @@ __device__ __forceinline__ RcStep rc_step(const RcParams& P, int s) {
 __device__ __forceinline__ int rc_kchunk(const RcParams& P, int s, int nkb, int i, int rank) {
   if (s == 0 || s == P.L) return i;
   const int ncl = P.NH / 64;
+  if (P.korder == 2) {  // own chunks first, the other CTAs' chunks one position behind
+    int v = 0;
+    for (int t = 0; t <= ncl; ++t) {
+      if (t < ncl) {
+        const int g = rank * ncl + t;
+        if (g < nkb && v++ == i) return g;
+      }
+      if (t >= 1)
+        for (int p = 1; p < P.CS; ++p) {
+          const int g = ((rank + p) % P.CS) * ncl + t - 1;
+          if (g < nkb && v++ == i) return g;
+        }
+    }
+    return i;
+  }
   if (P.korder == 1) {
     for (int t = 0, v = 0; t < P.CS * ncl; ++t) {
       const int g = ((rank + t % P.CS) % P.CS) * ncl + t / P.CS;
@@ -444,8 +460,8 @@ __global__ void __launch_bounds__(RC_THREADS, 1) rowchain_kernel(const __grid_co
                 d0 = h0 * 0.25f;
                 d1 = h1 * 0.25f;
 #else
-                sigmoid_d(__uint_as_float(raw[g2 * 16 + 2 * k]) + bb[2 * k], h0, d0);
-                sigmoid_d(__uint_as_float(raw[g2 * 16 + 2 * k + 1]) + bb[2 * k + 1], h1, d1);
+                sigmoid_d_fast(__uint_as_float(raw[g2 * 16 + 2 * k]) + bb[2 * k], h0, d0);
+                sigmoid_d_fast(__uint_as_float(raw[g2 * 16 + 2 * k + 1]) + bb[2 * k + 1], h1, d1);
 #endif
                 pk[k] = pack_bf16x2(h0, h1);
                 sp[k] = pack_bf16x2(d0, d1);
@@ -500,10 +516,10 @@ __global__ void __launch_bounds__(RC_THREADS, 1) rowchain_kernel(const __grid_co
             // lane p ships the piece to CTA p (remote ops issued in parallel); lane `rank` stores
             // the piece to global and arrives locally
             if (lane == 0) {
-              tma_store_2d(fwd ? &P.mH[lo] : &P.mDZ[lo], piece, n0, rb * 128 + q * 32);
               if (signal) {
                 // the receivers pre-armed their chunk_ready[g] with expect_tx (MMA thread), so a
-                // remote piece needs nothing but the bulk copy and its complete_tx
+                // remote piece needs nothing but the bulk copy and its complete_tx; the copies go
+                // first (the peers' MMAs wait on them; the global store is off the critical path)
                 for (int p = 1; p < CS; ++p) {
                   const int dst = (rank + p) % CS;
                   bulk_copy_s2cluster(mapa_shared(smem_u32(piece), dst), piece, RC_PIECE,
@@ -511,6 +527,7 @@ __global__ void __launch_bounds__(RC_THREADS, 1) rowchain_kernel(const __grid_co
                 }
                 mbar_arrive(&chunk_ready[g]);
               }
+              tma_store_2d(fwd ? &P.mH[lo] : &P.mDZ[lo], piece, n0, rb * 128 + q * 32);
             }
           }
           if (dbg) dbg[c == 0 ? 8 : 9] = gtimer();

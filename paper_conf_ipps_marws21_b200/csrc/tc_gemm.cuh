@@ -180,7 +180,7 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
 
   const int warp = threadIdx.x >> 5;
   const int lane = threadIdx.x & 31;
-  unsigned long long* dbg = ep.dbg ? ep.dbg + 8 * ((size_t)(blockIdx.z * gridDim.y + blockIdx.y) * gridDim.x + blockIdx.x) : nullptr;
+  unsigned long long* dbg = ep.dbg ? ep.dbg + 12 * ((size_t)(blockIdx.z * gridDim.y + blockIdx.y) * gridDim.x + blockIdx.x) : nullptr;
   if (dbg && threadIdx.x == 0) dbg[0] = gtimer();
   // Tiles: persistent CTAs walk tiles t = blockIdx.x, +gridDim.x, ... (n fastest, so CTAs running
   // together share the A row panel in L2).  Split-K launches (gridDim.z > 1) are one tile per CTA.
@@ -519,8 +519,8 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
 #pragma unroll
             for (int qq = 0; qq < 8; ++qq) {
               float h0, d0, h1, d1;
-              sigmoid_d(v[2 * qq] + sb[c + 2 * qq], h0, d0);
-              sigmoid_d(v[2 * qq + 1] + sb[c + 2 * qq + 1], h1, d1);
+              sigmoid_d_fast(v[2 * qq] + sb[c + 2 * qq], h0, d0);
+              sigmoid_d_fast(v[2 * qq + 1] + sb[c + 2 * qq + 1], h1, d1);
               hp[qq] = pack_bf16x2(h0, h1);
               sp[qq] = pack_bf16x2(d0, d1);
             }
@@ -532,7 +532,7 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
 #pragma unroll
               for (int qq = 0; qq < 16; ++qq) {
                 float hv, dv;
-                sigmoid_d(v[qq] + sb[c + qq], hv, dv);
+                sigmoid_d_fast(v[qq] + sb[c + qq], hv, dv);
                 acc += hv + dv;
               }
               if (acc == 12345.f) static_cast<float*>(ep.bias_upd)[0] = acc;
@@ -541,8 +541,8 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
 #pragma unroll
               for (int qq = 0; qq < 8; ++qq) {
                 float h0, d0, h1, d1;
-                sigmoid_d(v[2 * qq] + sb[c + 2 * qq], h0, d0);
-                sigmoid_d(v[2 * qq + 1] + sb[c + 2 * qq + 1], h1, d1);
+                sigmoid_d_fast(v[2 * qq] + sb[c + 2 * qq], h0, d0);
+                sigmoid_d_fast(v[2 * qq + 1] + sb[c + 2 * qq + 1], h1, d1);
                 hp[qq] = pack_bf16x2(h0, h1);
                 sp[qq] = pack_bf16x2(d0, d1);
               }
@@ -563,7 +563,7 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
                     static_cast<float*>(ep.out0)[(int64_t)r * ep.ld0 + nc + j] = z;
                   } else {
                     float hv, dv;
-                    sigmoid_d(z, hv, dv);
+                    sigmoid_d_fast(z, hv, dv);
                     static_cast<__nv_bfloat16*>(ep.out0)[(int64_t)r * ep.ld0 + nc + j] = __float2bfloat16_rn(hv);
                     if (ep.out1)
                       static_cast<__nv_bfloat16*>(ep.out1)[(int64_t)r * ep.ld1 + nc + j] = __float2bfloat16_rn(dv);
@@ -625,7 +625,29 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
     //      tile over the `splits` partials (read from every CTA's shared memory, fixed order) and
     //      applies the fused SGD update ----
     static_assert(TC_BM * (BN + 4) * 4 <= Cfg::STAGES * Cfg::STAGE_BYTES, "split-K tile must fit the ring");
+    // the fp32 master rows of this CTA's slice do not depend on the partials: fetch them (up to 8
+    // float4 per thread) before the cluster barrier so their latency hides behind it
+    constexpr int RED_MAXIT = 8;
+    float4 wpre[RED_MAXIT];
+    {
+      const int t = t_first;
+      int m_tile, n_tile;
+      tile_coords(t, tiles_m, tiles_n, m_tile, n_tile);
+      const int tid = threadIdx.x - 128;
+      const int rps = TC_BM / splits;
+#pragma unroll
+      for (int u = 0; u < RED_MAXIT; ++u) {
+        wpre[u] = make_float4(0.f, 0.f, 0.f, 0.f);
+        const int e = (tid + u * TC_EPI_THREADS) * 4;
+        if (EPI == EPI_WGRAD_SGD && warp >= 4 && !ep.transposed && e < rps * BN) {
+          const int gm = m_tile * TC_BM + kz * rps + e / BN, gn = n_tile * BN + e % BN;
+          if (gm < ep.M && gn + 4 <= ep.N) wpre[u] = __ldcg(reinterpret_cast<const float4*>(ep.master + (int64_t)gm * ep.ldw + gn));
+        }
+      }
+    }
+    if (dbg && threadIdx.x == 128) dbg[8] = gtimer();
     cluster_sync_all();  // every partial tile is in shared memory (release/acquire, cluster scope)
+    if (dbg && threadIdx.x == 128) dbg[9] = gtimer();
     if (warp >= 4) {
       const int t = t_first;
       int m_tile, n_tile;
@@ -634,23 +656,43 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
       const int tid = threadIdx.x - 128;  // 0..255
       const int rps = TC_BM / splits;
       const uint32_t tile_s = smem_u32(smem);
-      for (int e = tid * 4; e < rps * BN; e += TC_EPI_THREADS * 4) {
+      // every load of an element group is issued before the first add (the adds keep the fixed
+      // split order, so the result is bitwise the same as a sequential sum): one DSMEM round trip
+      // per group instead of `splits` dependent ones; the master row is fetched up front too
+#pragma unroll 1
+      for (int e = tid * 4, u = 0; e < rps * BN; e += TC_EPI_THREADS * 4, ++u) {
         const int rloc = kz * rps + e / BN, col = e % BN;
         const uint32_t off = (uint32_t)((rloc * (BN + 4) + col) * 4);
-        float4 acc = make_float4(0.f, 0.f, 0.f, 0.f);
-        for (int sp = 0; sp < splits; ++sp) {
-          const float4 t = ld_dsmem_f4(mapa_shared(tile_s + off, (uint32_t)sp));
-          acc.x += t.x;
-          acc.y += t.y;
-          acc.z += t.z;
-          acc.w += t.w;
-        }
         const int gm = m0 + rloc, gn = n0 + col;
-        if (gm >= ep.M || gn >= ep.N) continue;
+        const bool in = gm < ep.M && gn < ep.N;
+        const bool vec = in && !ep.transposed && gn + 4 <= ep.N && EPI == EPI_WGRAD_SGD;
+        float4* W = vec ? reinterpret_cast<float4*>(ep.master + (int64_t)gm * ep.ldw + gn) : nullptr;
+        float4 w = make_float4(0.f, 0.f, 0.f, 0.f);
+        if (vec) {
+          if (u < RED_MAXIT) {  // prefetched (static register index via the unrolled select)
+#pragma unroll
+            for (int k = 0; k < RED_MAXIT; ++k)
+              if (k == u) w = wpre[k];
+          } else {
+            w = *W;
+          }
+        }
+        float4 part[8];
+#pragma unroll
+        for (int sp = 0; sp < 8; ++sp)
+          if (sp < splits) part[sp] = ld_dsmem_f4(mapa_shared(tile_s + off, (uint32_t)sp));
+        float4 acc = make_float4(0.f, 0.f, 0.f, 0.f);
+#pragma unroll
+        for (int sp = 0; sp < 8; ++sp)
+          if (sp < splits) {
+            acc.x += part[sp].x;
+            acc.y += part[sp].y;
+            acc.z += part[sp].z;
+            acc.w += part[sp].w;
+          }
+        if (!in) continue;
         const float a4[4] = {acc.x, acc.y, acc.z, acc.w};
-        if (!ep.transposed && gn + 4 <= ep.N && EPI == EPI_WGRAD_SGD) {
-          float4* W = reinterpret_cast<float4*>(ep.master + (int64_t)gm * ep.ldw + gn);
-          float4 w = *W;
+        if (vec) {
           w.x -= ep.lr * acc.x;
           w.y -= ep.lr * acc.y;
           w.z -= ep.lr * acc.z;
@@ -664,6 +706,7 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
             if (gn + j < ep.N) epi_elem<EPI, __nv_bfloat16, false>(ep, gm, gn + j, a4[j]);
         }
       }
+      if (dbg && threadIdx.x == 128) dbg[10] = gtimer();
       if (ep.bpart_in) {  // bias: rows of this CTA's slice (or, transposed, the tile's columns)
         int lo, hi;
         bool own;
@@ -679,6 +722,7 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
         if (own) bias_reduce_update<EPI>(ep, lo, hi, tid);
       }
     }
+    if (dbg && threadIdx.x == 128) dbg[11] = gtimer();
     cluster_sync_all();  // no CTA leaves while another still reads its partial tile
   }
 

@@ -1,0 +1,6 @@
+#!/bin/bash
+for sp in 4 8; do HB_WGRAD_BN=256 HB_MAX_SPLITS=$sp timeout -s KILL 60 python scripts/gemm_phases.py 2,512,512,8192 2>&1 | tail -13; done
+HB_WGRAD_BN=256 HB_MAX_SPLITS=4 timeout -s KILL 60 python scripts/gemm_bench.py 2,512,512,8192 2,4096,4096,8192 2,4096,20958,8192 2>&1 | tail -3
+timeout -s KILL 60 python scripts/gemm_bench.py 2,512,512,8192 2,4096,4096,8192 2,4096,20958,8192 2>&1 | tail -3
+timeout -s KILL 100 python scripts/rc_probe.py 54,512,512,512,512,7 8192 2>&1 | grep graph
+timeout -s KILL 400 python -m pytest tests -m gpu -q -x --timeout 300 2>&1 | tail -2

