@@ -368,7 +368,7 @@ static int gemm_simt_p(int epi, bool a_mn, bool b_mn, int M, int N, int K, const
 // ----------------------------------------------------------------------------------------
 struct RcCfg {
   bool ok = false;
-  int CS = 1, NH = 64, NCA = 1, NS = 2, tmem = 128, smem = 0;
+  int CS = 1, NH = 64, NCA = 1, NS = 2, tmem = 128, smem = 0, s_tma = 0;
 };
 
 static unsigned long long* g_rc_trace = nullptr;  // tuning only: hb_rc_trace
@@ -418,12 +418,18 @@ static RcCfg rowchain_cfg(const hb_model* m, int b = 8192) {
   c.NCA = std::max((n0 + 63) / 64, c.CS * c.NH / 64);
   const int stb = c.NH * 128;
   // 1 KB alignment slack + abuf + W ring + staged bias (1 KB) + mbarriers
-  const int fixed = 1024 + c.NCA * RC_CHUNK + 1024 + 8 * (2 * RC_MAX_STAGES + c.NCA + 8) + 16;
+  // sigma' staging for TMA stores (2 chunk buffers) when the W ring keeps >= 2 stages: the
+  // per-thread-row global stores it replaces cost ~0.45 us per chunk (B200, C2 b = 8192) and a
+  // 2-stage ring measured as fast as 3 (scripts/gpu_refresh.sh)
+  static const int s_tma_env = env_int("HB_RC_S_TMA", 1);
+  c.s_tma = s_tma_env && (RC_SMEM_CAP - (1024 + c.NCA * RC_CHUNK + 2 * RC_CHUNK + 1024 + 8 * (2 * 2 + c.NCA + 8) + 16)) /
+                             (c.NH * 128) >= 2;
+  const int fixed = 1024 + c.NCA * RC_CHUNK + (c.s_tma ? 2 * RC_CHUNK : 0) + 1024 + 8 * (2 * RC_MAX_STAGES + c.NCA + 8) + 16;
   static const int ns_env = env_int("HB_RC_NS", 0);  // tuning only: force the W ring depth
   c.NS = std::min(RC_MAX_STAGES, (RC_SMEM_CAP - fixed) / stb);
   if (ns_env >= 2 && ns_env < c.NS) c.NS = ns_env;
   if (c.NS < 2) return c;
-  c.smem = 1024 + c.NCA * RC_CHUNK + c.NS * stb + 1024 + 8 * (2 * c.NS + c.NCA + 8) + 16;
+  c.smem = 1024 + c.NCA * RC_CHUNK + c.NS * stb + (c.s_tma ? 2 * RC_CHUNK : 0) + 1024 + 8 * (2 * c.NS + c.NCA + 8) + 16;
   c.tmem = 64;
   while (c.tmem < 2 * c.NH) c.tmem *= 2;
   c.ok = true;
@@ -447,6 +453,7 @@ static int launch_rowchain(hb_worker* w, const RcCfg& c, const void* X, int64_t 
     if (!rc && l <= L - 2) {
       rc = make_map(&P.mH[l], w->H[l], n, b, (int64_t)Ly.ldo * 2, 64, 32);
       if (!rc) rc = make_map(&P.mDZ[l], w->dZ[l], n, b, (int64_t)Ly.ldo * 2, 64, 32);
+      if (!rc) rc = make_map(&P.mS[l], w->S[l], n, b, (int64_t)Ly.ldo * 2, 64, 32);
       P.S[l] = static_cast<__nv_bfloat16*>(w->S[l]);
     }
     P.bias[l] = m->master + Ly.b_off;
@@ -471,6 +478,7 @@ static int launch_rowchain(hb_worker* w, const RcCfg& c, const void* X, int64_t 
   P.tmem_cols = c.tmem;
   static const int korder = env_int("HB_RC_KORDER", 0);  // 1 measured slower (B200, C2 b = 8192: 103 vs 88 us)
   P.korder = korder;
+  P.s_tma = c.s_tma;
   P.inv_b = 1.0f / (float)b;
   P.dbg = g_rc_trace;
   int dev = 0;

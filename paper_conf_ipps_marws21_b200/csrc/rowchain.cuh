@@ -65,6 +65,7 @@ struct RcParams {
   CUtensorMap mWt[RC_MAX_L];     // W_l as MN-major operand (l >= 1), box {64, 64}
   CUtensorMap mH[RC_MAX_L];      // H_l store [b x n], box {64, 32}          (l <= L-2)
   CUtensorMap mDZ[RC_MAX_L];     // dZ_l store [b x n], box {64, 32}         (l <= L-2)
+  CUtensorMap mS[RC_MAX_L];      // S_l store [b x n], box {64, 32}          (l <= L-2)
   const float* bias[RC_MAX_L];   // fp32 master b_l
   __nv_bfloat16* S[RC_MAX_L];    // sigma' stash S_l [b x ldo]                (l <= L-2)
   float* bpart[RC_MAX_L];        // bias-gradient partials of dZ_l [4 x row blocks x n_out(l)] (per quadrant)
@@ -77,6 +78,7 @@ struct RcParams {
   int CS, NH;                    // cluster size, output columns per CTA (multiple of 64)
   int nstages, abuf_chunks, tmem_cols;
   int korder;                    // k-block order of chunked steps (rc_kchunk)
+  int s_tma;                     // 1: sigma' stash staged in smem (2 chunk buffers) and TMA-stored
   float inv_b;
   unsigned long long* dbg;       // tuning only: per CTA, per step RC_DBG_W globaltimer stamps (nullable)
 };
@@ -173,7 +175,8 @@ __global__ void __launch_bounds__(RC_THREADS, 1) rowchain_kernel(const __grid_co
   const int NS = P.nstages;
   uint8_t* abuf = smem;
   uint8_t* ring = abuf + NCA * RC_CHUNK;
-  float* sbias = reinterpret_cast<float*>(ring + NS * STB);  // [NH] bias of the current forward step
+  uint8_t* sstage = ring + NS * STB;  // [2][RC_CHUNK] sigma' staging (s_tma), else empty
+  float* sbias = reinterpret_cast<float*>(sstage + (P.s_tma ? 2 * RC_CHUNK : 0));  // [NH] bias of the current forward step
   uint64_t* w_full = reinterpret_cast<uint64_t*>(sbias + 256);
   uint64_t* w_empty = w_full + NS;
   uint64_t* chunk_ready = w_empty + NS;
@@ -417,6 +420,11 @@ __global__ void __launch_bounds__(RC_THREADS, 1) rowchain_kernel(const __grid_co
         for (int c = 0; c < nmy; ++c) {
           const int g = rank * ncl + c;
           const int n0 = g * 64;
+          if (fwd && P.s_tma && c >= 2) {  // staging buffer c % 2: chunk c-2's S store has read it
+            if (h == 0 && lane == 0) tma_store_wait_read_1();
+            quad_bar_sync(q);
+          }
+          const uint32_t srow_s = smem_u32(sstage + (c & 1) * RC_CHUNK + q * RC_PIECE) + lane * 128;
           const int nh = n0 + h * 32;  // first column of this warp's half
           const bool full_chunk = n0 + 64 <= n;
           uint32_t raw[32];
@@ -466,11 +474,11 @@ __global__ void __launch_bounds__(RC_THREADS, 1) rowchain_kernel(const __grid_co
                 pk[k] = pack_bf16x2(h0, h1);
                 sp[k] = pack_bf16x2(d0, d1);
               }
-#ifdef HB_RC_NO_S_STORE  // tuning only (wrong numerics): epilogue cost without the sigma' stash stores
-              if (false) {
-#else
-              if (row_ok) {
-#endif
+              if (P.s_tma) {  // swizzled like the H piece; rows >= b / columns >= n clipped by the store
+                const int js = h * 4 + g2 * 2;
+                sts128(srow_s + ((js ^ (lane & 7)) << 4), sp[0], sp[1], sp[2], sp[3]);
+                sts128(srow_s + (((js + 1) ^ (lane & 7)) << 4), sp[4], sp[5], sp[6], sp[7]);
+              } else if (row_ok) {
                 __nv_bfloat16* srow = Sg + (int64_t)grow * P.ldo + nc;
                 if (nc + 16 <= n) {
                   reinterpret_cast<uint4*>(srow)[0] = make_uint4(sp[0], sp[1], sp[2], sp[3]);
@@ -528,6 +536,10 @@ __global__ void __launch_bounds__(RC_THREADS, 1) rowchain_kernel(const __grid_co
                 mbar_arrive(&chunk_ready[g]);
               }
               tma_store_2d(fwd ? &P.mH[lo] : &P.mDZ[lo], piece, n0, rb * 128 + q * 32);
+              if (fwd && P.s_tma) {
+                tma_store_2d(&P.mS[lo], sstage + (c & 1) * RC_CHUNK + q * RC_PIECE, n0, rb * 128 + q * 32);
+                tma_store_commit();  // one group per chunk (the staging reuse waits on chunk c-2's)
+              }
             }
           }
           if (dbg) dbg[c == 0 ? 8 : 9] = gtimer();
