@@ -1,0 +1,149 @@
+"""Paper-shaped experiment reproduction on synthetic data.
+
+    python scripts/experiments.py [--nets covtype,w8a,realsim,delicious] [--epochs 10]
+                                  [--eta-grid 0.001,0.01,0.1,1] [--out profiles/r01_experiments.json]
+
+For each of the paper's network shapes (§VII.A: 512-unit sigmoid hidden layers,
+covtype 6 hidden layers, w8a 8, real-sim 4, delicious 8) on a synthetic dataset of the paper's
+shape (synth/), three algorithms run the same epoch budget from the same initial
+model on one B200 (Figs. 5, 6 and 8 analogues):
+
+* ``minibatch``  — one GPU worker, batch 8192 (the paper's GPU-only mini-batch baseline);
+* ``static``     — heterogeneous Hogbatch with fixed batches: a large-batch worker (8192) and a
+                   small-batch worker (32) on the same shared model (the paper's "CPU+GPU" static
+                   configuration, L177);
+* ``adaptive``   — Adaptive Hogbatch (Alg. 2): large worker [2048, 8192] from 8192, small worker
+                   [32, 2048] from 32, batch sizes re-assigned from the update counts.
+
+The learning rate follows the paper's protocol (L258): the best eta0 of a powers-of-10 grid (by the
+lowest loss any algorithm reaches), eta = eta0 * b / b0 with b0 = 32.  Reported per algorithm:
+full-data loss after every epoch, cumulative training time (loss evaluation excluded, L258), the
+normalised loss (loss / minimum over algorithms), time and epochs to reach 1.1x the minimum,
+and the share of model updates per worker (Fig. 8).  The delicious-shaped net is
+single-label with C = 983 classes (multi-label is out of scope) and exercises the warp-per-row
+softmax-xent kernel.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import sys
+import time
+
+import numpy as np
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+sys.path.insert(0, ROOT)
+
+NETS = {  # name: (dataset, hidden layers of 512 units)
+    "covtype": ("covtype", 6),
+    "w8a": ("w8a", 8),
+    "realsim": ("realsim", 4),
+    "delicious": ("delicious", 8),
+}
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--nets", default="covtype,w8a,realsim,delicious")
+    ap.add_argument("--epochs", type=int, default=10)
+    ap.add_argument("--eta-grid", default="0.001,0.01,0.1,1")
+    ap.add_argument("--b0", type=int, default=32)
+    ap.add_argument("--out", default=os.path.join(ROOT, "profiles", "r01_experiments.json"))
+    args = ap.parse_args()
+
+    import torch
+    import paper_conf_ipps_marws21_b200 as hb
+    from synth import init_params, make_dataset, params_to_flat, DATASETS
+
+    results = {}
+    for net in args.nets.split(","):
+        ds, nh = NETS[net]
+        spec = DATASETS[ds]
+        d, C, N = spec["d"], spec["C"], spec["N"]
+        dims = [d] + [512] * nh + [C]
+        t0 = time.time()
+        ld = (d + 7) // 8 * 8
+        if ds == "covtype":
+            X, y, _, _ = make_dataset(ds, N=N, seed=0)
+            Xp = np.zeros((N, ld), dtype=np.float32)
+            Xp[:, :d] = X
+            Xd = torch.from_numpy(Xp).to(torch.bfloat16).cuda()
+            del X, Xp
+        else:  # sparse-shaped: densified on the device ("processed in dense format", L255)
+            (indptr, indices, vals), y, _, _ = make_dataset(ds, N=N, seed=0, dense=False)
+            rows = torch.from_numpy(np.repeat(np.arange(N), np.diff(indptr))).cuda()
+            Xd = torch.zeros(N, ld, dtype=torch.bfloat16, device="cuda")
+            Xd[rows, torch.from_numpy(indices.astype(np.int64)).cuda()] = torch.from_numpy(vals).cuda().to(torch.bfloat16)
+        yd = torch.from_numpy(y.astype(np.int32)).cuda()
+        gen_s = time.time() - t0
+        model = hb.MLP(dims, precision="bf16", seed=0)
+        p0 = params_to_flat(init_params(dims, seed=2))
+        big = hb.Worker(model, 8192)
+        small = hb.Worker(model, 2048)
+        algos = {
+            "minibatch": (hb.HB_MINIBATCH, [big], [hb.WorkerSpec(8192, 8192, 8192)]),
+            "static": (hb.HB_STATIC, [big, small], [hb.WorkerSpec(8192, 8192, 8192), hb.WorkerSpec(32, 32, 32)]),
+            "adaptive": (hb.HB_ADAPTIVE, [big, small], [hb.WorkerSpec(2048, 8192, 8192), hb.WorkerSpec(32, 2048, 32)]),
+        }
+        runs = {}
+        for eta in [float(e) for e in args.eta_grid.split(",")]:
+            for name, (kind, ws, sp) in algos.items():
+                model.set_params(p0)
+                pol = hb.Policy(kind=kind, workers=sp, eta0=eta, b0=args.b0, eval_loss=True)
+                st = hb.hogbatch_run(ws, pol, Xd, yd, epochs=args.epochs)
+                upd = st["updates"].sum(axis=0)
+                runs[(eta, name)] = dict(
+                    loss=[float(v) for v in st["epoch_loss"]],
+                    t=np.cumsum(st["epoch_train_s"]).tolist(),
+                    updates=upd.tolist(),
+                    samples=st["samples"].sum(axis=0).tolist(),
+                    steps=int(st["n_steps"]))
+
+        def best(eta):
+            return min(min([v for v in runs[(eta, a)]["loss"] if v == v] or [np.inf]) for a in algos)
+        etas = sorted({e for e, _ in runs})
+        eta_star = min(etas, key=best)
+        lmin = best(eta_star)
+        target = 1.1 * lmin
+        out = {"dims": dims, "N": N, "classes": C, "eta0": eta_star, "b0": args.b0, "epochs": args.epochs,
+               "min_loss": lmin, "target_loss": target, "data_gen_s": round(gen_s, 1),
+               "grid_best_loss": {str(e): best(e) for e in etas}, "algorithms": {}}
+        for a in algos:
+            r = runs[(eta_star, a)]
+            hit = next((i for i, v in enumerate(r["loss"]) if v <= target), None)
+            tot_upd = sum(r["updates"]) or 1
+            samples = sum(r["samples"])
+            out["algorithms"][a] = {
+                "epoch_loss": [round(v, 5) for v in r["loss"]],
+                "normalised_loss": [round(v / lmin, 4) for v in r["loss"]],
+                "epoch_end_s": [round(v, 5) for v in r["t"]],
+                "epochs_to_target": None if hit is None else hit + 1,
+                "time_to_target_s": None if hit is None else r["t"][hit],
+                "update_share": [round(u / tot_upd, 4) for u in r["updates"]],
+                "samples_per_s": samples / r["t"][-1] if r["t"] and r["t"][-1] > 0 else None,
+                "steps": r["steps"],
+            }
+        results[net] = out
+        print(f"{net:9s} dims {dims[0]}-512x{nh}-{C}  eta0 {eta_star:g}  min loss {lmin:.4f}", flush=True)
+        for a, r in out["algorithms"].items():
+            print(f"   {a:9s} final {r['epoch_loss'][-1]:.4f}  to 1.1x min: "
+                  f"{r['epochs_to_target']} epochs / {r['time_to_target_s']} s  "
+                  f"samples/s {r['samples_per_s'] or 0:.3g}  update share {r['update_share']}", flush=True)
+        del algos, big, small
+        del model, Xd, yd
+        torch.cuda.empty_cache()
+    results["_meta"] = {"method": "same epoch budget per algorithm from the same initial model; eta0 from the "
+                                  "powers-of-10 grid by the lowest loss reached (PAPER.md L258); target = 1.1 x "
+                                  "minimum loss across algorithms (L264); training time only (L258)",
+                        "data": "synthetic, seeded (synth/), shapes of PAPER.md L255-L256",
+                        "device": torch.cuda.get_device_name(0)}
+    os.makedirs(os.path.dirname(args.out), exist_ok=True)
+    with open(args.out, "w") as f:
+        json.dump(results, f, indent=1)
+    print("wrote", args.out)
+
+
+if __name__ == "__main__":
+    main()

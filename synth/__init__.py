@@ -10,6 +10,7 @@ from .data import (  # noqa: F401
     DATASETS,
     bf16_round,
     covtype_like,
+    delicious_like,
     init_params,
     make_dataset,
     pad_cols,

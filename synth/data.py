@@ -138,6 +138,30 @@ def sparse_like(N: int, d: int, nnz_mean: float, pos_frac: float, binary: bool,
     return (indptr, indices.astype(np.int32), vals), y
 
 
+def delicious_like(N: int, seed: int = 0, teacher_seed: int = 1, C: int = 983, d: int = 500,
+                   nnz_mean: float = 18.2):
+    """delicious-shaped CSR (500 binary features, ~18 nonzeros/row) with ONE label per row out
+    of C = 983 classes (the paper's multi-label task is out of scope; a
+    single-label head of this width exercises the warp-per-row softmax kernel).  Class priors
+    are Zipf-like (p_c ~ 1/(c + 5)); labels from a C-class tanh teacher with Gumbel-max sampling
+    and calibrated offsets, as for the other shapes."""
+    csr, _ = sparse_like(N, d, nnz_mean, 0.5, True, seed=seed, teacher_seed=teacher_seed)
+    indptr, indices, vals = csr
+    rng = _rng(seed + 1000)
+    t = _rng(teacher_seed + 1000)
+    A = t.standard_normal((d, 32)) * (3.0 / np.sqrt(nnz_mean))
+    Cm = t.standard_normal((32, C)) * 2.0
+    lens = np.diff(indptr)
+    XA = np.zeros((N, 32))
+    rows = np.repeat(np.arange(N), lens)
+    np.add.at(XA, rows, vals.astype(np.float64)[:, None] * A[indices])
+    scores = np.tanh(XA) @ Cm / 0.5
+    g = -np.log(-np.log(rng.uniform(1e-12, 1.0, size=(N, C))))
+    pri = 1.0 / (np.arange(C) + 5.0)
+    y = _gumbel_labels(scores, pri / pri.sum(), g)
+    return csr, y
+
+
 def csr_to_dense(csr, d: int, ld: int | None = None) -> np.ndarray:
     indptr, indices, vals = csr
     N = len(indptr) - 1
@@ -154,6 +178,7 @@ DATASETS = {
     "w8a": dict(d=300, C=2, N=64700, hidden=[1024] * 3),
     "realsim": dict(d=20958, C=2, N=72309, hidden=[4096] * 4),
     "tiny": dict(d=54, C=7, N=10000, hidden=[64, 64]),
+    "delicious": dict(d=500, C=983, N=16105, hidden=[512] * 8),
 }
 
 
@@ -166,6 +191,8 @@ def make_dataset(name: str, N: int | None = None, seed: int = 0, dense: bool = T
         return X, y, spec["d"], spec["C"]
     if name == "w8a":
         csr, y = sparse_like(N, 300, 11.6, 0.03, True, seed=seed)
+    elif name == "delicious":
+        csr, y = delicious_like(N, seed=seed)
     else:
         csr, y = sparse_like(N, 20958, 51.5, 0.31, False, seed=seed)
     X = csr_to_dense(csr, spec["d"]) if dense else csr
