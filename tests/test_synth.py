@@ -41,3 +41,16 @@ def test_param_flat_roundtrip():
     q = flat_to_params(params_to_flat(p), dims)
     for (a, b), (c, d) in zip(p, q):
         assert np.array_equal(a, c) and np.array_equal(b, d)
+
+
+def test_delicious_like_single_label_zipf_priors():
+    from synth import delicious_like
+    csr, y = delicious_like(3000)
+    csr2, y2 = delicious_like(3000)
+    assert np.array_equal(y, y2) and np.array_equal(csr[1], csr2[1])
+    X = csr_to_dense(csr, 500)
+    assert X.shape == (3000, 500) and set(np.unique(X)) <= {0.0, 1.0}
+    assert y.dtype == np.int32 and y.min() >= 0 and y.max() < 983
+    # Zipf-like priors: the head classes dominate, frequencies decrease on average
+    f = np.bincount(y, minlength=983) / len(y)
+    assert f[:10].sum() > f[500:510].sum() * 5
