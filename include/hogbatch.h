@@ -155,7 +155,7 @@ int mlp_num_params(const hb_model* m, int64_t* n_out);
  * not disabled with HB_ROWCHAIN=0), 0 if they take the per-layer GEMM chain, < 0 on error. */
 int mlp_fused_path(const hb_model* m, int32_t batch, int32_t* cluster_size);
 /* Steps of at least min_batch rows take the fused row-block chain when the shape is eligible
- * (0 = never; default 8192 = the measured crossover on B200, or HB_RC_MIN_B).  Workers created
+ * (0 = never; default 4096 = the measured crossover on B200, or HB_RC_MIN_B).  Workers created
  * afterwards allocate what the fused path needs; set it before mlp_worker_create. */
 int mlp_set_fused_min_batch(hb_model* m, int32_t min_batch);
 /* host flat fp32 layout: [W_1 (n_1 x n_0 row-major, unpadded), b_1, W_2, b_2, ...]; n must equal

@@ -44,7 +44,7 @@ struct hb_model {
   int device = 0;
   int prec = HB_PREC_BF16;
   std::vector<int> dims;
-  int rc_min_b = 8192;              // fused row-block step from this batch size up (0 = never)
+  int rc_min_b = 4096;              // fused row-block step from this batch size up (0 = never)
   std::vector<hb::Layer> layers;
   size_t total = 0;                 // floats in the flat parameter buffer (incl. padding)
   float* master = nullptr;          // fp32 master weights + biases (the shared global model)

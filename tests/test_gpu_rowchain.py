@@ -153,7 +153,8 @@ def test_every_cluster_size_matches_oracle(cs):
 def test_unfused_shapes_report_layer_chain():
     _need_gpu()
     m = hb.MLP([54, 512, 512, 7])
-    assert m.fused_path(8192) == 2 and m.fused_path(4096) == 0   # default crossover b = 8192
+    assert m.fused_path(8192) == 2 and m.fused_path(4096) == 4   # default crossover b = 4096
+    assert m.fused_path(2048) == 0
     m.set_fused_min_batch(0)
     assert m.fused_path(8192) == 0
     assert hb.MLP([54, 1024, 1024, 7]).fused_path() == 0     # n > 512
