@@ -94,7 +94,12 @@ typedef struct hb_policy {
   const hb_worker_policy* workers;
 } hb_policy;
 
-/* Training data resident in device memory (borrowed; caller-owned). */
+/* Training data (borrowed; caller-owned).  X and y are both device pointers (used in place) or
+ * both host pointers (pinned for overlap; pageable works but copies synchronously): host data
+ * is staged by hogbatch_run into a device copy owned by the model, in chunks of
+ * HB_STAGE_ROWS (default 32768) rows on a copy stream, and a batch waits only for the chunk
+ * holding its last row — the host->device transfer of the data set overlaps training on its
+ * first rows ("the coordinator owns the data" [L123]; batches are row ranges [L141]). */
 typedef struct hb_dataset {
   const void* X;  /* [n x ldx] row-major, dtype x_dtype; ldx*elemsize must be a multiple of 16 */
   int64_t ldx;    /* row stride in elements (>= n_0)                                           */
@@ -203,7 +208,8 @@ int mlp_loss(hb_model* m, const void* X, int64_t ldx, int32_t x_dtype, const int
 int hb_schedule_trace(const hb_policy* p, int64_t N, int32_t epochs, hb_trace_rec* out,
                       int64_t cap, int64_t* n_out);
 /* Trains with n_workers workers (one host thread each, concurrent Hogbatch updates of the
- * shared model, L170) under policy p for `epochs` epochs over data.  Blocking.
+ * shared model, L170) under policy p for `epochs` epochs over data (device or host, see
+ * hb_dataset).  Blocking.
  * p->deterministic = 1 executes the virtual-clock trace serially (SERIAL policy, L125). */
 int hogbatch_run(hb_worker** workers, int32_t n_workers, const hb_policy* p,
                  const hb_dataset* data, int32_t epochs, hb_stats* stats_out);

@@ -1228,6 +1228,10 @@ int mlp_destroy(hb_model* m) {
   cudaFree(m->base);
   cudaFree(m->delta);
   cudaFree(m->chunk_sums);
+  cudaFree(m->stage_x);
+  cudaFree(m->stage_y);
+  for (cudaEvent_t e : m->stage_ev) cudaEventDestroy(e);
+  if (m->copy_stream) cudaStreamDestroy(m->copy_stream);
   if (m->stream) cudaStreamDestroy(m->stream);
   delete m;
   return HB_OK;

@@ -56,6 +56,14 @@ struct hb_model {
   std::mutex eval_mu;
   double* chunk_sums = nullptr;
   int64_t chunk_cap = 0;
+  // hogbatch_run over a HOST dataset: device staging copy (reused across calls), the copy
+  // stream and one event per staged chunk of rows
+  void* stage_x = nullptr;
+  size_t stage_x_cap = 0;
+  int32_t* stage_y = nullptr;
+  size_t stage_y_cap = 0;
+  cudaStream_t copy_stream = nullptr;
+  std::vector<cudaEvent_t> stage_ev;
 };
 
 struct hb_worker {
