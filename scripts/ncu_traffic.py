@@ -10,8 +10,7 @@ def col(name):
     return h.index(name) if name in h else None
 ci = {k: col(k) for k in ["Kernel Name", "Grid Size", "gpu__time_duration.sum", "dram__bytes_read.sum",
                           "dram__bytes_write.sum", "sm__pipe_tensor_cycles_active.avg.pct_of_peak_sustained_elapsed",
-                          "lts__t_bytes.sum", "sm__pipe_tensor_subpipe_hmma_cycles_active_realtime.avg",
-                          "sm__cycles_active.avg"]}
+                          "lts__t_sectors.sum", "sm__pipe_tensor_cycles_active.avg.pct_of_peak_sustained_active"]}
 units = rows[1]
 def val(r, k):
     i = ci[k]
@@ -30,14 +29,13 @@ for r in rows[2:]:
     rd, wr = val(r, "dram__bytes_read.sum") or 0, val(r, "dram__bytes_write.sum") or 0
     d = dict(kernel=name[:70], grid=r[ci["Grid Size"]], cls=cls, us=val(r, "gpu__time_duration.sum") * 1e6,
              dram_read=rd, dram_write=wr, tensor_pct=val(r, "sm__pipe_tensor_cycles_active.avg.pct_of_peak_sustained_elapsed"),
-             l2_bytes=val(r, "lts__t_bytes.sum"),
-             hmma_active=(val(r, "sm__pipe_tensor_subpipe_hmma_cycles_active_realtime.avg") or 0) /
-                         max(1.0, val(r, "sm__cycles_active.avg") or 1.0))
+             l2_bytes=(val(r, "lts__t_sectors.sum") or 0) * 32,
+             tensor_active=val(r, "sm__pipe_tensor_cycles_active.avg.pct_of_peak_sustained_active") or 0)
     summary.append(d)
     traffic.setdefault(cls, []).append(rd + wr)
 for d in summary:
     print(f"{d['cls']:15s} {d['grid']:14s} {d['us']:9.2f} us  dram {(d['dram_read']+d['dram_write'])/1e6:9.2f} MB  "
-          f"tensor {d['tensor_pct'] or 0:5.1f}%  hmma-active {100 * d['hmma_active']:5.1f}%  "
+          f"tensor {d['tensor_pct'] or 0:5.1f}% of elapsed ({d['tensor_active']:5.1f}% of active)  "
           f"L2 {(d['l2_bytes'] or 0) / 1e6:8.1f} MB  {d['kernel']}")
 path = os.path.join(os.path.dirname(os.path.dirname(os.path.abspath(__file__))), "profiles", "ncu_traffic.json")
 allt = json.load(open(path)) if os.path.exists(path) else {}
