@@ -47,17 +47,34 @@ namespace hb {
 
 constexpr int RC_MAX_L = 12;     // weight layers supported by one launch
 constexpr int RC_MAX_CS = 8;     // CTAs per row block (portable cluster size)
-constexpr int RC_THREADS = 384;  // 4 control warps + 8 epilogue warps
-constexpr int RC_EPI_THREADS = 256;
+// Epilogue warps: 4 TMEM quadrants x RC_PARTS column parts of every 64-column chunk (RC_PARTS = 4:
+// 16 warps of 16 columns — twice the latency hiding of 2 x 32 columns; the per-chunk work is
+// latency-bound, not issue-bound, on B200)
+#ifndef RC_EPI_PARTS
+#define RC_EPI_PARTS 4
+#endif
+constexpr int RC_PARTS = RC_EPI_PARTS;
+constexpr int RC_EPI_WARPS = 4 * RC_PARTS;
+constexpr int RC_THREADS = 128 + 32 * RC_EPI_WARPS;  // 4 control warps + the epilogue warps
+constexpr int RC_EPI_THREADS = 32 * RC_EPI_WARPS;
+constexpr int RC_CPW = 64 / RC_PARTS;  // columns of a chunk per epilogue warp
+constexpr int RC_NG = RC_CPW / 16;     // 16-column groups per warp and chunk
+constexpr int RC_NSV = RC_CPW / 8;     // uint4 of sigma' per warp row and chunk
 constexpr int RC_CHUNK = 16384;  // 128 rows x 64 bf16 columns (SW128 K-major)
 constexpr int RC_PIECE = 4096;   // 32 rows of a chunk (one quadrant's share)
 constexpr int RC_MAX_STAGES = 12;
 
 enum { RC_FWD = 0, RC_HEAD = 1, RC_DX = 2 };
 
-__device__ __forceinline__ void epi_bar_sync_n(int) { asm volatile("bar.sync 1, 256;" ::: "memory"); }
-// the two epilogue warps of quadrant q (named barriers 2..5)
-__device__ __forceinline__ void quad_bar_sync(int q) { asm volatile("bar.sync %0, 64;" ::"r"(2 + q) : "memory"); }
+// one warp's columns of a chunk from TMEM (32 lanes x RC_CPW columns)
+__device__ __forceinline__ void rc_tmem_ld(uint32_t t, uint32_t (&r)[32]) { tmem_ld_32x32b_x32(t, r); }
+__device__ __forceinline__ void rc_tmem_ld(uint32_t t, uint32_t (&r)[16]) { tmem_ld_32x32b_x16(t, r); }
+
+__device__ __forceinline__ void epi_bar_sync_n(int) { asm volatile("bar.sync 1, %0;" ::"n"(RC_EPI_THREADS) : "memory"); }
+// the RC_PARTS epilogue warps of quadrant q (named barriers 2..5)
+__device__ __forceinline__ void quad_bar_sync(int q) {
+  asm volatile("bar.sync %0, %1;" ::"r"(2 + q), "n"(32 * RC_PARTS) : "memory");
+}
 
 struct RcParams {
   CUtensorMap mX;                // X [x_rows x n0], box {64, 128}
@@ -208,7 +225,7 @@ __global__ void __launch_bounds__(RC_THREADS, 1) rowchain_kernel(const __grid_co
     mbar_init(x_full, 1);
     for (int a = 0; a < 2; ++a) {
       mbar_init(&acc_full[a], 1);
-      mbar_init(&acc_empty[a], 8);
+      mbar_init(&acc_empty[a], RC_EPI_WARPS);
     }
     mbar_init(peer_free, CS > 1 ? CS - 1 : 1);
     fence_barrier_init();
@@ -318,7 +335,7 @@ __global__ void __launch_bounds__(RC_THREADS, 1) rowchain_kernel(const __grid_co
   } else if (warp >= 4) {
     // ===== epilogue =====
     const int q = warp & 3;
-    const int h = (warp - 4) >> 2;  // 32-column half of every chunk
+    const int h = (warp - 4) >> 2;  // column part of every chunk: columns [h*RC_CPW, (h+1)*RC_CPW)
     const int et = threadIdx.x - 128;
     const int rl = q * 32 + lane;
     const int grow = rb * 128 + rl;  // batch row
@@ -340,14 +357,14 @@ __global__ void __launch_bounds__(RC_THREADS, 1) rowchain_kernel(const __grid_co
         if (et < P.NH) sbias[et] = nn < n ? __ldg(P.bias[lo] + nn) : 0.f;
         epi_bar_sync_n(RC_EPI_THREADS);
       }
-      // dX: prefetch this row's sigma' (this warp's 32 columns of the first chunk) while the MMAs run
-      uint4 sv[4];
+      // dX: prefetch this row's sigma' (this warp's columns of the first chunk) while the MMAs run
+      uint4 sv[RC_NSV];
 #pragma unroll
-      for (int k = 0; k < 4; ++k) sv[k] = make_uint4(0, 0, 0, 0);
+      for (int k = 0; k < RC_NSV; ++k) sv[k] = make_uint4(0, 0, 0, 0);
       if (st.kind == RC_DX && row_ok && nmy > 0 && (rank * ncl + 1) * 64 <= n) {
-        const uint4* srow = reinterpret_cast<const uint4*>(Sg + (int64_t)grow * P.ldo + rank * ncl * 64 + h * 32);
+        const uint4* srow = reinterpret_cast<const uint4*>(Sg + (int64_t)grow * P.ldo + rank * ncl * 64 + h * RC_CPW);
 #pragma unroll
-        for (int k = 0; k < 4; ++k) sv[k] = __ldg(srow + k);
+        for (int k = 0; k < RC_NSV; ++k) sv[k] = __ldg(srow + k);
       }
       mbar_wait(&acc_full[buf], (s >> 1) & 1);
       tc_fence_after();
@@ -425,27 +442,27 @@ __global__ void __launch_bounds__(RC_THREADS, 1) rowchain_kernel(const __grid_co
             quad_bar_sync(q);
           }
           const uint32_t srow_s = smem_u32(sstage + (c & 1) * RC_CHUNK + q * RC_PIECE) + lane * 128;
-          const int nh = n0 + h * 32;  // first column of this warp's half
+          const int nh = n0 + h * RC_CPW;  // first column of this warp's part
           const bool full_chunk = n0 + 64 <= n;
-          uint32_t raw[32];
-          tmem_ld_32x32b_x32(tq + (uint32_t)(c * 64 + h * 32), raw);
+          uint32_t raw[RC_CPW];
+          rc_tmem_ld(tq + (uint32_t)(c * 64 + h * RC_CPW), raw);
           // sigma' of the NEXT chunk: its global load overlaps this chunk's work (chunk 0's was
           // issued before the accumulator wait)
-          uint4 svn[4];
+          uint4 svn[RC_NSV];
 #pragma unroll
-          for (int k = 0; k < 4; ++k) svn[k] = make_uint4(0, 0, 0, 0);
+          for (int k = 0; k < RC_NSV; ++k) svn[k] = make_uint4(0, 0, 0, 0);
           if (!fwd && c + 1 < nmy && row_ok && n0 + 128 <= n) {
             const uint4* srow = reinterpret_cast<const uint4*>(Sg + (int64_t)grow * P.ldo + nh + 64);
 #pragma unroll
-            for (int k = 0; k < 4; ++k) svn[k] = __ldg(srow + k);
+            for (int k = 0; k < RC_NSV; ++k) svn[k] = __ldg(srow + k);
           }
           tmem_ld_wait();
           if (dbg && c == 0) dbg[6] = gtimer();
           uint8_t* piece = abuf + g * RC_CHUNK + q * RC_PIECE;
           const uint32_t prow_s = smem_u32(piece) + lane * 128;
-          const uint32_t sb_s = smem_u32(sbias) + (uint32_t)(c * 64 + h * 32) * 4;
+          const uint32_t sb_s = smem_u32(sbias) + (uint32_t)(c * 64 + h * RC_CPW) * 4;
 #pragma unroll
-          for (int g2 = 0; g2 < 2; ++g2) {
+          for (int g2 = 0; g2 < RC_NG; ++g2) {
             const int nc = nh + g2 * 16;
             uint32_t pk[8];
             if (fwd) {
@@ -475,7 +492,7 @@ __global__ void __launch_bounds__(RC_THREADS, 1) rowchain_kernel(const __grid_co
                 sp[k] = pack_bf16x2(d0, d1);
               }
               if (P.s_tma) {  // swizzled like the H piece; rows >= b / columns >= n clipped by the store
-                const int js = h * 4 + g2 * 2;
+                const int js = h * (RC_CPW / 8) + g2 * 2;
                 sts128(srow_s + ((js ^ (lane & 7)) << 4), sp[0], sp[1], sp[2], sp[3]);
                 sts128(srow_s + (((js + 1) ^ (lane & 7)) << 4), sp[4], sp[5], sp[6], sp[7]);
               } else if (row_ok) {
@@ -513,7 +530,7 @@ __global__ void __launch_bounds__(RC_THREADS, 1) rowchain_kernel(const __grid_co
               const int col = nc + colsum16_col(lane);
               if (!(lane & 1) && col < n) P.bpart[lo][prow * n + col] = t;
             }
-            const int j0 = h * 4 + g2 * 2;  // 16-byte column chunk of the 128-byte row
+            const int j0 = h * (RC_CPW / 8) + g2 * 2;  // 16-byte column chunk of the 128-byte row
             sts128(prow_s + ((j0 ^ (lane & 7)) << 4), pk[0], pk[1], pk[2], pk[3]);
             sts128(prow_s + (((j0 + 1) ^ (lane & 7)) << 4), pk[4], pk[5], pk[6], pk[7]);
           }
@@ -544,7 +561,7 @@ __global__ void __launch_bounds__(RC_THREADS, 1) rowchain_kernel(const __grid_co
           }
           if (dbg) dbg[c == 0 ? 8 : 9] = gtimer();
 #pragma unroll
-          for (int k = 0; k < 4; ++k) sv[k] = svn[k];
+          for (int k = 0; k < RC_NSV; ++k) sv[k] = svn[k];
         }
         if (h == 0 && lane == 0) tma_store_commit();
       }
