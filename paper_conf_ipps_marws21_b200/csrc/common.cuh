@@ -290,12 +290,23 @@ __device__ __forceinline__ void sigmoid_d(float z, float& h, float& d) {
 // (1, 2], starts from the minimax line 24/17 - 8/17 y (relative error <= 1/17) and takes two
 // Newton steps s <- s (2 - y s) on the FMA pipe (error 1/17 -> 3.5e-3 -> 1.2e-5, far below the
 // bf16 rounding of H and S).  The fp32 check mode keeps sigmoid_d.
+__device__ __forceinline__ float ex2_ftz(float x) {  // MUFU.EX2 without __expf's denormal fix-up
+  float y;
+  asm("ex2.approx.ftz.f32 %0, %1;" : "=f"(y) : "f"(x));
+  return y;
+}
 __device__ __forceinline__ void sigmoid_d_fast(float z, float& h, float& d) {
-  const float e = __expf(-fabsf(z));
+  // e = exp(-|z|) flushed to 0 below 2^-126 (|z| > 87): then h = 0 or 1 and d = 0, exact in bf16
+  const float e = ex2_ftz(fabsf(z) * -1.4426950408889634f);
   const float y = 1.0f + e;
+#ifdef HB_SIG_RCP  // tuning only: MUFU reciprocal instead of the FMA-pipe Newton steps
+  float s;
+  asm("rcp.approx.ftz.f32 %0, %1;" : "=f"(s) : "f"(y));
+#else
   float s = fmaf(-8.0f / 17.0f, y, 24.0f / 17.0f);
   s = s * fmaf(-y, s, 2.0f);
   s = s * fmaf(-y, s, 2.0f);
+#endif
   const float es = e * s;
   h = z >= 0.f ? s : es;
   d = es * s;

@@ -60,6 +60,8 @@ constexpr int RC_EPI_THREADS = 32 * RC_EPI_WARPS;
 constexpr int RC_CPW = 64 / RC_PARTS;  // columns of a chunk per epilogue warp
 constexpr int RC_NG = RC_CPW / 16;     // 16-column groups per warp and chunk
 constexpr int RC_NSV = RC_CPW / 8;     // uint4 of sigma' per warp row and chunk
+constexpr int RC_H_COPY = RC_PARTS > 1 ? 1 : 0;  // epilogue part whose lane 0 ships pieces to peers
+constexpr int RC_H_S = RC_PARTS > 2 ? 2 : 0;     // ... and whose lane 0 stores the sigma' pieces
 constexpr int RC_CHUNK = 16384;  // 128 rows x 64 bf16 columns (SW128 K-major)
 constexpr int RC_PIECE = 4096;   // 32 rows of a chunk (one quadrant's share)
 constexpr int RC_MAX_STAGES = 12;
@@ -100,7 +102,7 @@ struct RcParams {
   unsigned long long* dbg;       // tuning only: per CTA, per step RC_DBG_W globaltimer stamps (nullable)
 };
 constexpr int RC_DBG_STEPS = 24;
-constexpr int RC_DBG_W = 10;  // stamps per step
+constexpr int RC_DBG_W = 14;  // stamps per step
 
 struct RcStep {
   int kind, layer, N, nkb, kkn;
@@ -429,16 +431,16 @@ __global__ void __launch_bounds__(RC_THREADS, 1) rowchain_kernel(const __grid_co
           }
         }
       } else {
-        // this quadrant's TMA stores of the previous step (issued by its h = 0 warp) have read
-        // abuf before either half writes the pieces again
-        if (h == 0 && lane == 0) tma_store_wait_read();
+        // this quadrant's TMA stores of the previous step (H / dZ pieces by its h = 0 warp, sigma'
+        // pieces by its h = RC_H_S warp) have read their smem before any part writes it again
+        if ((h == 0 || h == RC_H_S) && lane == 0) tma_store_wait_read();
         quad_bar_sync(q);
         const bool signal = fwd || st.layer >= 2;  // the output is the next step's A operand
         for (int c = 0; c < nmy; ++c) {
           const int g = rank * ncl + c;
           const int n0 = g * 64;
           if (fwd && P.s_tma && c >= 2) {  // staging buffer c % 2: chunk c-2's S store has read it
-            if (h == 0 && lane == 0) tma_store_wait_read_1();
+            if (h == RC_H_S && lane == 0) tma_store_wait_read_1();
             quad_bar_sync(q);
           }
           const uint32_t srow_s = smem_u32(sstage + (c & 1) * RC_CHUNK + q * RC_PIECE) + lane * 128;
@@ -536,34 +538,40 @@ __global__ void __launch_bounds__(RC_THREADS, 1) rowchain_kernel(const __grid_co
           }
           if (dbg && c == 0) dbg[7] = gtimer();
           fence_proxy_async();
+          if (dbg && c == 0) dbg[10] = gtimer();
           quad_bar_sync(q);  // both halves of the piece are written
-          if (h == 0) {
-            // lane p ships the piece to CTA p (remote ops issued in parallel); lane `rank` stores
-            // the piece to global and arrives locally
-            if (lane == 0) {
-              if (signal) {
-                // the receivers pre-armed their chunk_ready[g] with expect_tx (MMA thread), so a
-                // remote piece needs nothing but the bulk copy and its complete_tx; the copies go
-                // first (the peers' MMAs wait on them; the global store is off the critical path)
-                for (int p = 1; p < CS; ++p) {
-                  const int dst = (rank + p) % CS;
-                  bulk_copy_s2cluster(mapa_shared(smem_u32(piece), dst), piece, RC_PIECE,
-                                      mapa_shared(smem_u32(&chunk_ready[g]), dst));
-                }
-                mbar_arrive(&chunk_ready[g]);
+          if (dbg && c == 0) dbg[11] = gtimer();
+          // the piece's asynchronous operations are issued by lane 0 of different warps of the
+          // quadrant so their issue latencies overlap (each blocks ~0.1-0.3 us on B200):
+          //   RC_H_COPY: bulk copies to the peers (their MMAs wait on them) + the local arrival,
+          //   0:         TMA store of the H / dZ piece (one bulk group per chunk),
+          //   RC_H_S:    TMA store of the sigma' staging piece (one bulk group per chunk)
+          if (lane == 0) {
+            if (h == RC_H_COPY && signal) {
+              // the receivers pre-armed their chunk_ready[g] with expect_tx (MMA thread), so a
+              // remote piece needs nothing but the bulk copy and its complete_tx
+              for (int p = 1; p < CS; ++p) {
+                const int dst = (rank + p) % CS;
+                bulk_copy_s2cluster(mapa_shared(smem_u32(piece), dst), piece, RC_PIECE,
+                                    mapa_shared(smem_u32(&chunk_ready[g]), dst));
               }
+              mbar_arrive(&chunk_ready[g]);
+              if (dbg && c == 0) dbg[12] = gtimer();
+            }
+            if (h == 0) {
               tma_store_2d(fwd ? &P.mH[lo] : &P.mDZ[lo], piece, n0, rb * 128 + q * 32);
-              if (fwd && P.s_tma) {
-                tma_store_2d(&P.mS[lo], sstage + (c & 1) * RC_CHUNK + q * RC_PIECE, n0, rb * 128 + q * 32);
-                tma_store_commit();  // one group per chunk (the staging reuse waits on chunk c-2's)
-              }
+              tma_store_commit();
+              if (dbg && c == 0) dbg[13] = gtimer();
+            }
+            if (h == RC_H_S && fwd && P.s_tma) {
+              tma_store_2d(&P.mS[lo], sstage + (c & 1) * RC_CHUNK + q * RC_PIECE, n0, rb * 128 + q * 32);
+              tma_store_commit();  // one group per chunk (the staging reuse waits on chunk c-2's)
             }
           }
           if (dbg) dbg[c == 0 ? 8 : 9] = gtimer();
 #pragma unroll
           for (int k = 0; k < RC_NSV; ++k) sv[k] = svn[k];
         }
-        if (h == 0 && lane == 0) tma_store_commit();
       }
       // release the accumulator (all TMEM reads of this warp have completed)
       tc_fence_before();

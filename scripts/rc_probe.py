@@ -35,33 +35,33 @@ for b in batches:
     print(f"b={b:6d}: {e0.elapsed_time(e1) * 1000 / n:8.1f} us/step (direct launches incl. host encode)", flush=True)
 if m.fused_path():
     for b in [x for x in batches if x in (32, 8192)] or batches[-1:]:
-        cap = 1024 * 24 * 10
+        cap = 1024 * 24 * 14
         hb.lib.hb_rc_trace(None, cap)
         w.step(tX, ty, b, 0.0)
         buf = (C.c_uint64 * cap)()
         hb.lib.hb_rc_trace(buf, cap)
         hb.lib.hb_rc_trace(None, 0) if False else None
-        a = np.frombuffer(buf, dtype=np.uint64).reshape(1024, 24, 10).astype(np.int64)
+        a = np.frombuffer(buf, dtype=np.uint64).reshape(1024, 24, 14).astype(np.int64)
         grid = m.fused_path(b) * ((b + 127) // 128)
         ctas = np.arange(grid)
         a = a[ctas]
         t0 = a[:, 0, 0].min()
         L = len(dims) - 1
         nct = grid
-        base = 1024 * 24 * 10
+        base = 1024 * 24 * 14
         raw = np.frombuffer(buf, dtype=np.uint64).astype(np.int64)
         # the tail region is indexed with gridDim.x = nct CTAs
-        tail = raw[nct * 24 * 10: nct * 24 * 10 + 3 * nct * 16].reshape(3, nct, 16)
+        tail = raw[nct * 24 * 14: nct * 24 * 14 + 3 * nct * 16].reshape(3, nct, 16)
         for ci in range(min(2, nct)):
             iss, crdy, wrdy = tail[0, ci, :8], tail[1, ci, :8], tail[2, ci, :8]
             rel = lambda v: [round(float(x - t0) / 1000, 2) for x in v]
             print(f"   cta{ci} step2 k-blocks (us from kernel start): issue {rel(iss)}\n"
                   f"        chunk ready {rel(crdy)}\n        W ready     {rel(wrdy)}")
         print(f"--- b={b}: {len(ctas)} CTAs, span {(a[a > 0].max() - t0) / 1000:.2f} us; per step (median over CTAs, us from kernel start):")
-        print("   step  mma_start  first_w  mma_issued  epi_acc  epi_peer  epi_end  ld0  c0comp  c0sig  c1sig")
+        print("   step  mma_start  first_w  mma_issued  epi_acc  epi_peer  epi_end  ld0  c0comp  c0sig  c1sig  c0fence  c0bar  c0copies  c0hstore")
         for s in range(2 * L - 1):
             v = a[:, s, :]
-            row = [np.median(v[:, k][v[:, k] > 0] - t0) / 1000 if (v[:, k] > 0).any() else -1 for k in range(10)]
+            row = [np.median(v[:, k][v[:, k] > 0] - t0) / 1000 if (v[:, k] > 0).any() else -1 for k in range(14)]
             print(f"   {s:4d}  " + "  ".join(f"{x:8.2f}" for x in row))
 
 # device time per step (graph replay), whole step / chain only / dW only
