@@ -259,17 +259,25 @@ def main():
     # ---- lower threshold of the large worker: smallest power of 2 with >= 50% of the
     #      samples/s at the upper threshold ("GPU utilization for the lower
     #      threshold is about 50%") — calibrated on this GPU, outside the timed region ----
-    def step_rate(b, reps=6):
-        for _ in range(2):
-            wl.step(Xd, yd, b, 0.0)
-        s0, s1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-        torch.cuda.synchronize()
-        s0.record()
-        for i in range(reps):
-            wl.step(Xd[i * b:], yd[i * b:], b, 0.0)
-        s1.record()
-        torch.cuda.synchronize()
-        return b * reps / (s0.elapsed_time(s1) * 1e-3)
+    def step_rate(b, reps=20, trials=3):
+        # best of `trials` timings of `reps` steps after a warm-up long enough for the clocks to
+        # settle: a low first reading of the upper threshold's rate would admit a too-small
+        # lower threshold (and a much slower schedule)
+        nb = max(1, N // b - 1)  # batches that fit in the data set (row offsets stay in range)
+        for i in range(10):
+            wl.step(Xd[(i % nb) * b:], yd[(i % nb) * b:], b, 0.0)
+        best = 0.0
+        for _ in range(trials):
+            s0, s1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            torch.cuda.synchronize()
+            s0.record()
+            for i in range(reps):
+                j = i % nb
+                wl.step(Xd[j * b:], yd[j * b:], b, 0.0)
+            s1.record()
+            torch.cuda.synchronize()
+            best = max(best, b * reps / (s0.elapsed_time(s1) * 1e-3))
+        return best
     params0 = params_to_flat(init_params(dims, seed=2))
     if args.policy == "adaptive" and args.config != "tiny":
         r_max = step_rate(big_max)
