@@ -90,8 +90,8 @@ def test_graph_replay_is_bitwise_equal_to_direct_launches():
     assert np.array_equal(out[0], out[1])
 
 
-@pytest.mark.parametrize("det", [False, True])
-def test_host_dataset_is_staged_and_bitwise_equal_to_device_dataset(det, monkeypatch):
+@pytest.mark.parametrize("det,pinned", [(False, True), (True, True), (False, False)])
+def test_host_dataset_is_staged_and_bitwise_equal_to_device_dataset(det, pinned, monkeypatch):
     # hogbatch_run with HOST X / y (pinned): staged in chunks overlapped with training; the model
     # after two epochs equals the run on the device copy bit for bit (same batches, same kernels)
     monkeypatch.setenv("HB_STAGE_ROWS", "1000")  # several chunks, ragged last chunk
@@ -103,13 +103,23 @@ def test_host_dataset_is_staged_and_bitwise_equal_to_device_dataset(det, monkeyp
         w = hb.Worker(m, 512)
         pol = hb.Policy(kind=hb.HB_MINIBATCH, workers=[hb.WorkerSpec(512, 512, 512)], eta0=0.1, b0=32,
                         deterministic=det, eval_loss=True)
-        if host:
-            tX, ty = tX.cpu().pin_memory(), ty.cpu().pin_memory()
+        if host:  # pinned (overlapped copy) or pageable (synchronous staging) host memory
+            tX, ty = tX.cpu(), ty.cpu()
+            if pinned:
+                tX, ty = tX.pin_memory(), ty.pin_memory()
         st = hb.hogbatch_run([w], pol, tX, ty, epochs=2)
         assert st["total_samples"] == 2 * (N // 512) * 512
         out.append((m.get_params(), st["epoch_loss"]))
     assert np.array_equal(out[0][0], out[1][0])
     assert out[0][1] == out[1][1]
+
+
+def test_host_dataset_mixed_pointers_rejected():
+    X, y, m, params, tX, ty = setup([54, 64, 7], "bf16", 256, 1024)
+    w = hb.Worker(m, 256)
+    pol = hb.Policy(kind=hb.HB_MINIBATCH, workers=[hb.WorkerSpec(256, 256, 256)], eta0=0.1, b0=32)
+    with pytest.raises(hb.HogbatchError):
+        hb.hogbatch_run([w], pol, tX.cpu().pin_memory(), ty, epochs=1)
 
 
 def test_concurrent_adaptive_hogwild_trains_and_respects_thresholds():
