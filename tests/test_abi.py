@@ -102,3 +102,27 @@ def test_model_creation_without_sm100_device_fails_loudly():
     with pytest.raises(hb.HogbatchError) as e:
         hb.MLP([54, 64, 7])
     assert e.value.code in (hb._lib.HB_ECUDA, hb._lib.HB_EUNSUPPORTED)
+
+
+def test_cpp_coordinator_matches_oracle_exhaustive_two_workers():
+    # exhaustive small space (SURVEY §8(c) "brute-force enumeration" pin): every pair of worker
+    # specs from a grid of thresholds / initial batches / virtual-clock costs, two data-set sizes,
+    # both u-reset readings (R3) and both credit points (R21), two epochs — exact trace equality
+    specs = []
+    for lo, hi, init in [(1, 4, 1), (1, 4, 4), (2, 2, 2), (1, 2, 2), (2, 8, 8)]:
+        for c0 in (0.0, 1.0):
+            for c1 in (0.5, 2.0):
+                specs.append((lo, hi, init, c0, c1))
+    n = 0
+    for a in specs:
+        for b in specs:
+            ws = [ocoord.WorkerSpec(a[0], a[1], a[2], a[3], a[4]), ocoord.WorkerSpec(b[0], b[1], b[2], b[3], b[4])]
+            for N in (7, 23):
+                for reset in ("fastest", "none"):
+                    for credit in ("dispatch", "completion"):
+                        p = ocoord.Policy(kind=ocoord.ADAPTIVE, alpha=2, eta0=0.5, b0=2, reset=reset, credit=credit,
+                                          workers=ws)
+                        exp = [r.astuple() for r in ocoord.run(p, N, 2, max_records=2000)]
+                        same(hb.schedule_trace(to_c_policy(p), N, 2, cap=2000), exp)
+                        n += 1
+    assert n == 3200
