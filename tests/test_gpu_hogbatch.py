@@ -193,6 +193,31 @@ def test_full_size_gradient_parity(dims, kind, b):
     assert abs(loss - l_ref) / l_ref <= 1e-2
 
 
+def test_full_size_c4_batch_gradient_is_mean_of_subbatch_gradients():
+    # configs[3] at the full batch b = 8192 in the launch configuration the bench times (the
+    # oracle cannot afford 5 TFLOP of fp64 here): the batch gradient is the mean of the gradients
+    # of its 32 sub-batches of 256 (a property of Eq. (2) at any size), and those sub-batch
+    # gradients are oracle-checked by test_full_size_gradient_parity
+    _gpu()
+    dims, b, sb = [20958, 4096, 4096, 4096, 4096, 2], 8192, 256
+    X, y = dataset("realsim", b, d=dims[0], seed=5)
+    m = hb.MLP(dims)
+    m.set_params(params_to_flat(init_params(dims)))
+    w = hb.Worker(m, b)
+    tX, ty = to_device(X, y)
+    g_full, loss_full = w.step_grads(tX, ty, b)
+    acc, losses = None, []
+    for k in range(b // sb):
+        g, l = w.step_grads(tX[k * sb:], ty[k * sb:], sb)
+        acc = g.astype(np.float64) if acc is None else acc + g
+        losses.append(l)
+    g_mean = acc / (b // sb)
+    got, ref = split_flat(g_full, dims), split_flat(g_mean, dims)
+    errs = [max(rel_err(got[l][0], ref[l][0]), rel_err(got[l][1], ref[l][1])) for l in range(len(dims) - 1)]
+    assert max(errs) <= 1e-2, errs
+    assert abs(loss_full - np.mean(losses)) / np.mean(losses) <= 1e-3
+
+
 def test_nested_worker_serial_matches_oracle():
     # NEXT f1: Alg. 2's CPU worker as a nested GPU worker (t sub-batches, in-place updates);
     # in deterministic mode the sub-batches run in order == the oracle's serial sub-steps
