@@ -45,6 +45,18 @@ CONFIGS = {
 }
 
 
+def class_roof(v, peaks, ridge):
+    """Per kernel class: device ms, launches, achieved TFLOP/s and GB/s, and the fraction of the
+    roofline that bounds the class (tensor peak above the ridge, HBM below it)."""
+    tf = v["flops"] / (v["ms"] * 1e-3) / 1e12 if v["ms"] else 0.0
+    gb = v["bytes"] / (v["ms"] * 1e-3) / 1e9 if v["ms"] else 0.0
+    ai = v["flops"] / v["bytes"] if v["bytes"] else 0.0
+    bound = "tensor" if v["flops"] > 0 and ai >= ridge else "hbm"
+    frac = tf / peaks["bf16_sus"] if bound == "tensor" else gb / peaks["hbm"]
+    return {"ms": round(v["ms"], 3), "launches": v["launches"], "TFLOP/s": round(tf, 1), "GB/s": round(gb, 1),
+            "flop_per_byte": round(ai, 1), "bound": bound, "frac": round(frac, 4)}
+
+
 def flops_per_sample(dims):
     P = sum(dims[i] * dims[i - 1] for i in range(1, len(dims)))
     return 6 * P - 2 * dims[0] * dims[1]
@@ -442,10 +454,7 @@ def main():
                     "ms_per_launch": d["ms"] / d["launches"],
                     "flops_per_launch": d["flops"] / d["launches"], "bytes_per_launch": d["bytes"] / d["launches"],
                     "peak_source": f"{peaks['src']} ({'bf16_tflops_sustained' if bound == 'tensor' else 'hbm_gbs'})",
-                    "classes": {k: {"ms": round(v["ms"], 3), "launches": v["launches"],
-                                    "TFLOP/s": round(v["flops"] / (v["ms"] * 1e-3) / 1e12, 1) if v["ms"] else None,
-                                    "GB/s": round(v["bytes"] / (v["ms"] * 1e-3) / 1e9, 1) if v["ms"] else None}
-                                for k, v in gem.items()}}
+                    "classes": {k: class_roof(v, peaks, ridge) for k, v in gem.items()}}
         cpu = None
         if not args.no_cpu_baseline and world == 1:
             cpu = cpu_baseline(cfg, args)
