@@ -40,6 +40,7 @@ struct EpiArgs {
   float* ws;            // WGRAD split-K: fp32 partial tiles [tiles][splits][128][BN]
   unsigned long long* dbg;  // tuning only: per-CTA phase timestamps (globaltimer ns), nullable
   int force_bn, force_splits;  // host-side launch choices for dW GEMMs (0 = heuristic)
+  int pair;                    // host-side: dW GEMM on CTA pairs (tcgen05 cta_group::2) when eligible
   // softmax cross-entropy head fused into the output-layer GEMM (C <= 16):
   const int32_t* y;     // labels (dataset base when yoff != nullptr)
   const int* yoff;      // device row offset of the batch (graph replay), nullable

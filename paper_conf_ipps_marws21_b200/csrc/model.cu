@@ -133,17 +133,17 @@ static int make_out_map(CUtensorMap* out, const void* base, int64_t cols, int64_
   return make_map(out, base, cols, rows, ld * 2, 64, TC_BM);
 }
 
-template <int BN, bool A_MN, bool B_MN, int EPI>
+template <int BN, bool A_MN, bool B_MN, int EPI, bool PAIR = false>
 static int launch_tc(const CUtensorMap& ma, const CUtensorMap& mb, int M, int N, int K, const int* offA,
                      const int* offB, const EpiArgs& ep, cudaStream_t s, int splits = 1) {
-  using Cfg = TcCfg<BN, B_MN, EPI>;
+  using Cfg = TcCfg<BN, B_MN, EPI, PAIR>;
   CUtensorMap mo0 = ma, mo1 = ma;  // unused unless the epilogue stages its outputs for TMA stores
   if (TmaOut<BN, EPI>::on) {
     int rc = make_out_map(&mo0, ep.out0, N, M, ep.ld0 > 0 ? ep.ld0 : round_up(N, 8));
     if (!rc && EPI == EPI_FWD_SIG && ep.out1) rc = make_out_map(&mo1, ep.out1, N, M, ep.ld1);
     if (rc) return rc;
   }
-  auto kern = tc_gemm_kernel<BN, A_MN, B_MN, EPI>;
+  auto kern = tc_gemm_kernel<BN, A_MN, B_MN, EPI, PAIR>;
   int dev = 0;
   cudaGetDevice(&dev);
   {
@@ -163,6 +163,7 @@ static int launch_tc(const CUtensorMap& ma, const CUtensorMap& mb, int M, int N,
     if (nsm <= 0) nsm = 148;
   }
   dim3 grid = splits == 1 ? dim3(std::min(tiles, nsm), 1, 1)
+              : PAIR      ? dim3((M + TC_BM - 1) / TC_BM, (N + BN - 1) / BN, splits)
                           : dim3((N + BN - 1) / BN, (M + TC_BM - 1) / TC_BM, splits);
   cudaLaunchConfig_t cfg{};
   cfg.gridDim = grid;
@@ -177,9 +178,9 @@ static int launch_tc(const CUtensorMap& ma, const CUtensorMap& mb, int M, int N,
     attr[na].val.programmaticStreamSerializationAllowed = 1;
     ++na;
   }
-  if (splits > 1) {
+  if (splits > 1) {  // the splits of a tile (and, PAIR, the two M tiles of a CTA pair) form a cluster
     attr[na].id = cudaLaunchAttributeClusterDimension;
-    attr[na].val.clusterDim.x = 1;
+    attr[na].val.clusterDim.x = PAIR ? 2 : 1;
     attr[na].val.clusterDim.y = 1;
     attr[na].val.clusterDim.z = splits;
     ++na;
@@ -282,6 +283,12 @@ static int gemm_tc(int epi, bool a_mn, bool b_mn, int M, int N, int K, TcOp A, T
     if (epi == EPI_DGRAD_SIG) return launch_tc_bn<false, true, EPI_DGRAD_SIG>(bn, ma, mb, M, N, K, A.off, B.off, ep, s);
   } else if (a_mn && b_mn) {
     const int S = !ep.ws ? 1 : ep.force_splits ? ep.force_splits : choose_splits(M, N, K, bn);
+    // CTA pairs (256-row tiles over two SMs sharing the B tile): BN 256, >= 2 splits, even M tiles
+    if (ep.pair && bn == 256 && S >= 2 && S <= 4 && ((M + TC_BM - 1) / TC_BM) % 2 == 0) {
+      if (epi == EPI_WGRAD_SGD) return launch_tc<256, true, true, EPI_WGRAD_SGD, true>(ma, mb, M, N, K, A.off, B.off, ep, s, S);
+      if (epi == EPI_WGRAD_STORE)
+        return launch_tc<256, true, true, EPI_WGRAD_STORE, true>(ma, mb, M, N, K, A.off, B.off, ep, s, S);
+    }
     if (epi == EPI_WGRAD_SGD)
       return launch_tc_bn<true, true, EPI_WGRAD_SGD>(bn, ma, mb, M, N, K, A.off, B.off, ep, s, S);
     if (epi == EPI_WGRAD_STORE)
@@ -856,6 +863,8 @@ static int launch_wgrad(hb_worker* w, int l, const void* X, int64_t ldx, int64_t
   ep.n_mtiles = part_rows;
   ep.force_bn = force_bn;
   ep.force_splits = force_splits;
+  static const int pair = env_int("HB_DW_PAIR", 0);
+  ep.pair = pair;
   ep.bias_upd = m->master + Ly.b_off;
   ep.bias_grad = grads_only ? w->grads + Ly.b_off : nullptr;
   ep.ws = ws;
@@ -1541,6 +1550,8 @@ static int bench_gemm_impl(int32_t kind, int32_t M, int32_t N, int32_t K, int32_
     ep.bpart_in = bp;
     ep.ldp = M;
     ep.n_mtiles = (K + 127) / 128;
+    ep.pair = env_int("HB_DW_PAIR", 0);           // tuning: CTA-pair dW
+    ep.force_splits = env_int("HB_FORCE_SPLITS", 0);
     ep.bias_upd = bias;
   }
   TcOp a{A, lda, arows, nullptr}, b{B, ldb, brows, nullptr};

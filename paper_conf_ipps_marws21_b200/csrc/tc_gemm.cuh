@@ -49,10 +49,13 @@ struct TmaOut {
   static constexpr int BYTES = on ? NOUT * NBOX * TC_BM * 128 : 0;
 };
 
-template <int BN, bool B_MN, int EPI = EPI_WGRAD_SGD>
+// PAIR: a CTA pair (cluster x = 2) computes a 256 x BN tile with tcgen05.mma.cta_group::2 — each
+// CTA loads its own 128 A rows and HALF of the B tile (BN/2 rows), the leader issues the MMAs.
+template <int BN, bool B_MN, int EPI = EPI_WGRAD_SGD, bool PAIR = false>
 struct TcCfg {
   static constexpr int A_BYTES = TC_BM * TC_BK * 2;                     // 16 KB
-  static constexpr int B_ROWS = B_MN ? (BN < 64 ? 64 : BN) : BN;        // MN-major loads 64-wide boxes
+  static constexpr int B_TILE = PAIR ? BN / 2 : BN;                     // B rows this CTA loads
+  static constexpr int B_ROWS = B_MN ? (B_TILE < 64 ? 64 : B_TILE) : B_TILE;  // MN-major loads 64-wide boxes
   static constexpr int B_BYTES = B_ROWS * TC_BK * 2;
   static constexpr int STAGE_BYTES = A_BYTES + B_BYTES;
   static constexpr int OUT_BYTES = TmaOut<BN, EPI>::BYTES;
@@ -158,14 +161,15 @@ __device__ __forceinline__ void stage16(uint8_t* sout, int o, int rl, int c, con
   *reinterpret_cast<uint4*>(row + (((j0 + 1) ^ (rl & 7)) << 4)) = make_uint4(p[4], p[5], p[6], p[7]);
 }
 
-template <int BN, bool A_MN, bool B_MN, int EPI>
+template <int BN, bool A_MN, bool B_MN, int EPI, bool PAIR = false>
 __global__ void __launch_bounds__(TC_THREADS, 1)
     tc_gemm_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUtensorMap tmB,
                    const __grid_constant__ CUtensorMap tmO0, const __grid_constant__ CUtensorMap tmO1,
                    int K, const int* __restrict__ offA, const int* __restrict__ offB, EpiArgs ep) {
-  using Cfg = TcCfg<BN, B_MN, EPI>;
+  using Cfg = TcCfg<BN, B_MN, EPI, PAIR>;
   using TO = TmaOut<BN, EPI>;
   constexpr int STAGES = Cfg::STAGES;
+  static_assert(!PAIR || (A_MN && B_MN && BN >= 128 && !TO::on), "CTA pairs: split-K dW GEMMs only");
   extern __shared__ uint8_t smem_raw[];
   uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
   uint8_t* sout = smem + STAGES * Cfg::STAGE_BYTES;  // TMA-store staging [NOUT][NBOX][128 rows x 128 B]
@@ -193,6 +197,11 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
   const int t_first = splits == 1 ? (int)blockIdx.x : (int)(blockIdx.y * gridDim.x + blockIdx.x);
   const int t_step = splits == 1 ? (int)gridDim.x : num_tiles;
   const int kz = blockIdx.z;
+  // CTA pair (grid x = M tiles, y = N tiles, z = splits; cluster (2, 1, S) — pairs must be along
+  // the cluster's x): half = blockIdx.x & 1; cluster rank of split sp's CTA with the same half =
+  // half + 2 sp; the pair's leader (half 0) has rank 2 kz
+  const uint32_t half = PAIR ? (blockIdx.x & 1) : 0;
+  const uint16_t pair_mask = (uint16_t)(3u << (2 * kz));
   const int num_kb_all = (K + TC_BK - 1) / TC_BK;
   const int kpb = (num_kb_all + splits - 1) / splits;
   const int kb_lo = min(num_kb_all, kz * kpb);
@@ -211,9 +220,15 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
     }
     fence_barrier_init();
   }
-  if (warp == 2) tmem_alloc<Cfg::TMEM_COLS>(tmem_slot);
+  if (warp == 2) {
+    if (PAIR)
+      tmem_alloc_pair<Cfg::TMEM_COLS>(tmem_slot);
+    else
+      tmem_alloc<Cfg::TMEM_COLS>(tmem_slot);
+  }
   tc_fence_before();
   __syncthreads();
+  if (PAIR) cluster_sync_all();  // the leader's barriers are initialised before the peer's loads signal them
   tc_fence_after();
   const uint32_t tmem_base = *tmem_slot;
   // programmatic dependent launch: everything above overlapped the previous kernel's tail;
@@ -230,15 +245,29 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
     for (int t = t_first; t < num_tiles; t += t_step) {
     int mt_, nt_;
     tile_coords(t, tiles_m, tiles_n, mt_, nt_);
-    const int m0 = mt_ * TC_BM, n0 = nt_ * BN;
+    if (PAIR) {  // one tile per CTA: this CTA's own M tile, the pair's N tile (its half of it)
+      mt_ = blockIdx.x;
+      nt_ = blockIdx.y;
+    }
+    const int m0 = mt_ * TC_BM, n0 = nt_ * BN + (int)half * Cfg::B_TILE;
+    const uint32_t lead_full = PAIR ? mapa_shared(smem_u32(full_bar), 2 * kz) : 0;
     for (int kb = 0; kb < num_kb; ++kb, ++it) {
       const int s = it % STAGES;
       const uint32_t ph = (it / STAGES) & 1;
       mbar_wait(&empty_bar[s], ph ^ 1);
       uint8_t* sA = smem + s * Cfg::STAGE_BYTES;
       uint8_t* sB = sA + Cfg::A_BYTES;
-      mbar_arrive_expect_tx(&full_bar[s], Cfg::STAGE_BYTES);
       const int k0 = (kb_lo + kb) * TC_BK;
+      if (PAIR) {  // both CTAs' loads complete on the leader's barrier, which expects both
+        const uint32_t fb = lead_full + (uint32_t)(s * 8);
+        if (half == 0) mbar_arrive_expect_tx(&full_bar[s], 2 * Cfg::STAGE_BYTES);
+        tma_load_2d_pair(sA, &tmA, fb, m0, k0 + oa);
+        tma_load_2d_pair(sA + 8192, &tmA, fb, m0 + 64, k0 + oa);
+#pragma unroll
+        for (int j = 0; j < Cfg::B_ROWS / 64; ++j) tma_load_2d_pair(sB + j * 8192, &tmB, fb, n0 + 64 * j, k0 + ob);
+        continue;
+      }
+      mbar_arrive_expect_tx(&full_bar[s], Cfg::STAGE_BYTES);
       if (!A_MN) {
         tma_load_2d(sA, &tmA, &full_bar[s], k0, m0 + oa);
       } else {
@@ -254,9 +283,9 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
       }
     }
     }
-  } else if (warp == 1 && lane == 0) {
-    // ===== MMA issuer (single thread) =====
-    constexpr uint32_t idesc = make_idesc_bf16(TC_BM, BN, A_MN, B_MN);
+  } else if (warp == 1 && lane == 0 && half == 0) {
+    // ===== MMA issuer (single thread; in a pair the leader issues for both CTAs) =====
+    constexpr uint32_t idesc = make_idesc_bf16(PAIR ? 2 * TC_BM : TC_BM, BN, A_MN, B_MN);
     int it = 0, i = 0;
     for (int t = t_first; t < num_tiles; t += t_step, ++i) {
     const int acc = i & 1;
@@ -280,11 +309,20 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
                                  : make_sw128_desc(a_base + kk * 32, 16, 1024);
         const uint64_t bd = B_MN ? make_sw128_desc(b_base + kk * 2048, 8192, 1024)
                                  : make_sw128_desc(b_base + kk * 32, 16, 1024);
-        umma_bf16(tacc, ad, bd, idesc, (kb | kk) != 0);
+        if (PAIR)
+          umma_bf16_pair(tacc, ad, bd, idesc, (kb | kk) != 0);
+        else
+          umma_bf16(tacc, ad, bd, idesc, (kb | kk) != 0);
       }
-      umma_commit(&empty_bar[s]);  // frees the smem slot when these MMAs complete
+      if (PAIR)
+        umma_commit_pair(&empty_bar[s], pair_mask);  // both CTAs' slots
+      else
+        umma_commit(&empty_bar[s]);  // frees the smem slot when these MMAs complete
     }
-    umma_commit(&tmem_full_bar[acc]);  // accumulator ready (arrives even if num_kb == 0)
+    if (PAIR)
+      umma_commit_pair(&tmem_full_bar[acc], pair_mask);
+    else
+      umma_commit(&tmem_full_bar[acc]);  // accumulator ready (arrives even if num_kb == 0)
     if (dbg && i == 0) dbg[3] = gtimer();
     }
   } else if (warp >= 4) {
@@ -303,6 +341,10 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
     const int acc = i & 1;
     int m_tile, n_tile;
     tile_coords(t, tiles_m, tiles_n, m_tile, n_tile);
+    if (PAIR) {
+      m_tile = blockIdx.x;
+      n_tile = blockIdx.y;
+    }
     const int m0 = m_tile * TC_BM, n0 = n_tile * BN;
     const int r = m0 + rl;
     const bool row_ok = r < ep.M;
@@ -633,6 +675,10 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
       const int t = t_first;
       int m_tile, n_tile;
       tile_coords(t, tiles_m, tiles_n, m_tile, n_tile);
+      if (PAIR) {
+        m_tile = blockIdx.x;
+        n_tile = blockIdx.y;
+      }
       const int tid = threadIdx.x - 128;
       const int rps = TC_BM / splits;
 #pragma unroll
@@ -652,6 +698,10 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
       const int t = t_first;
       int m_tile, n_tile;
       tile_coords(t, tiles_m, tiles_n, m_tile, n_tile);
+      if (PAIR) {
+        m_tile = blockIdx.x;
+        n_tile = blockIdx.y;
+      }
       const int m0 = m_tile * TC_BM, n0 = n_tile * BN;
       const int tid = threadIdx.x - 128;  // 0..255
       const int rps = TC_BM / splits;
@@ -680,7 +730,7 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
         float4 part[8];
 #pragma unroll
         for (int sp = 0; sp < 8; ++sp)
-          if (sp < splits) part[sp] = ld_dsmem_f4(mapa_shared(tile_s + off, (uint32_t)sp));
+          if (sp < splits) part[sp] = ld_dsmem_f4(mapa_shared(tile_s + off, PAIR ? half + 2u * sp : (uint32_t)sp));
         float4 acc = make_float4(0.f, 0.f, 0.f, 0.f);
 #pragma unroll
         for (int sp = 0; sp < 8; ++sp)
@@ -732,7 +782,10 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
   __syncthreads();
   if (warp == 2) {
     tc_fence_after();
-    tmem_dealloc<Cfg::TMEM_COLS>(tmem_base);
+    if (PAIR)
+      tmem_dealloc_pair<Cfg::TMEM_COLS>(tmem_base);
+    else
+      tmem_dealloc<Cfg::TMEM_COLS>(tmem_base);
   }
   if (dbg && threadIdx.x == 64) dbg[7] = gtimer();
 }
