@@ -96,8 +96,8 @@ typedef struct hb_policy {
 
 /* Training data (borrowed; caller-owned).  X and y are both device pointers (used in place) or
  * both host pointers (pinned for overlap; pageable works but copies synchronously): host data
- * is staged by hogbatch_run into a device copy owned by the model, in chunks of
- * HB_STAGE_ROWS (default 32768) rows on a copy stream, and a batch waits only for the chunk
+ * is staged by hogbatch_run into a device copy owned by the model, in chunks (HB_STAGE_ROWS;
+ * default 32768 rows, at most 32 MB) on a copy stream, and a batch waits only for the chunk
  * holding its last row — the host->device transfer of the data set overlaps training on its
  * first rows ("the coordinator owns the data" [L123]; batches are row ranges [L141]). */
 typedef struct hb_dataset {

@@ -79,8 +79,13 @@ class MLP:
             _check(r)
         return cs.value if r == 1 else 0
 
-    def get_params(self) -> np.ndarray:
-        out = np.empty(self.num_params, dtype=np.float32)
+    def get_params(self, out: np.ndarray | None = None) -> np.ndarray:
+        """``mlp_get_params`` into `out` (float32, num_params; pass a view of pinned host memory
+        for a full-bandwidth copy) or a new array."""
+        if out is None:
+            out = np.empty(self.num_params, dtype=np.float32)
+        if out.dtype != np.float32 or out.size != self.num_params or not out.flags["C_CONTIGUOUS"]:
+            raise ValueError("out must be a contiguous float32 array of num_params elements")
         _check(lib.mlp_get_params(self.h, out.ctypes.data_as(C.POINTER(C.c_float)), out.size))
         return out
 

@@ -1338,16 +1338,18 @@ int mlp_get_params(const hb_model* m, float* host_dst, int64_t n) {
   if (rc) return rc;
   HB_CHECK_ARG(host_dst && n == need, "n must equal mlp_num_params");
   HB_CUDA_TRY(cudaSetDevice(m->device));
-  std::vector<float> h(m->total);
   HB_CUDA_TRY(cudaDeviceSynchronize());  // every worker's in-place updates are visible
-  HB_CUDA_TRY(cudaMemcpyAsync(h.data(), m->master, m->total * 4, cudaMemcpyDeviceToHost, m->stream));
-  HB_CUDA_TRY(cudaStreamSynchronize(m->stream));
+  // the copy engine drops the row padding (pitched copies straight into the caller's buffer)
   int64_t o = 0;
   for (const Layer& Ly : m->layers) {
-    for (int i = 0; i < Ly.n_out; ++i)
-      for (int j = 0; j < Ly.n_in; ++j) host_dst[o++] = h[Ly.w_off + (size_t)i * Ly.ldw + j];
-    for (int i = 0; i < Ly.n_out; ++i) host_dst[o++] = h[Ly.b_off + i];
+    HB_CUDA_TRY(cudaMemcpy2DAsync(host_dst + o, (size_t)Ly.n_in * 4, m->master + Ly.w_off, (size_t)Ly.ldw * 4,
+                                  (size_t)Ly.n_in * 4, (size_t)Ly.n_out, cudaMemcpyDeviceToHost, m->stream));
+    o += (int64_t)Ly.n_out * Ly.n_in;
+    HB_CUDA_TRY(cudaMemcpyAsync(host_dst + o, m->master + Ly.b_off, (size_t)Ly.n_out * 4, cudaMemcpyDeviceToHost,
+                                m->stream));
+    o += Ly.n_out;
   }
+  HB_CUDA_TRY(cudaStreamSynchronize(m->stream));
   return HB_OK;
 }
 
