@@ -227,7 +227,7 @@ int choose_splits(int M, int N, int K, int bn) {
 static int choose_bn_wgrad(int M, int N, int K) {
   static const int forced = env_int("HB_WGRAD_BN", 0);
   if (forced) return forced;
-  if (K < 2048) return choose_bn(M, N);  // short K: no split-K, spread tiles over the SMs
+  if (K < 2048) return choose_bn(M, N, K);  // short K: no split-K, spread tiles over the SMs
   int bn = choose_bn_base(M, N);          // long K: split-K supplies the parallelism
   while (bn > 64 && (long)((M + TC_BM - 1) / TC_BM) * ((N + bn - 1) / bn) * 4 < 148) bn /= 2;
   return bn;
@@ -245,14 +245,15 @@ static int choose_bn_base(int M, int N) {
 
 // Tile width: the base rule, narrowed while the grid would leave most SMs idle (small batches:
 // M = b <= a few hundred rows gives 1-2 row tiles; narrower tiles spread the epilogue)
-int choose_bn(int M, int N) {
+int choose_bn(int M, int N, int K) {
   static const int forced = env_int("HB_FWD_BN", 0);  // tuning only: forward / dX tile width
   if (forced && N > 16) return forced;
   int bn = choose_bn_base(M, N);
   const long mt = (M + TC_BM - 1) / TC_BM;
-  // fewer than ~4 waves of 256-wide tiles: 128-wide tiles balance the persistent CTAs better
-  // (measured on B200: C3 8192 x 1024 layers 30.8 vs 28.9 M samples/s; C4's 4096-wide layers keep 256)
-  if (bn == 256 && mt * ((N + 255) / 256) < 4 * 148) bn = 128;
+  // fewer than ~4 waves of 256-wide tiles and a short K: 128-wide tiles balance the persistent
+  // CTAs better (measured on B200: C3 8192 x 1024 x 1024 layers 30.8 vs 28.9 M samples/s); long-K
+  // tiles keep 256 (width 4096-8192 at b = 2048, K = 4096: 55 vs 49% of peak with 256)
+  if (bn == 256 && K > 0 && K <= 2048 && mt * ((N + 255) / 256) < 4 * 148) bn = 128;
   while (bn > 32 && mt * ((N + bn - 1) / bn) < 64) bn /= 2;
   return bn;
 }
@@ -271,7 +272,7 @@ static int gemm_tc(int epi, bool a_mn, bool b_mn, int M, int N, int K, TcOp A, T
                    cudaStream_t s) {
   const int bn = epi == EPI_HEAD_XENT                          ? 16
                  : (epi == EPI_WGRAD_SGD || epi == EPI_WGRAD_STORE) ? (ep.force_bn ? ep.force_bn : choose_bn_wgrad(M, N, K))
-                                                                    : choose_bn(M, N);
+                                                                    : choose_bn(M, N, K);
   CUtensorMap ma, mb;
   const int64_t ar = A.rows ? A.rows : (a_mn ? K : M);
   const int64_t br = B.rows ? B.rows : (b_mn ? K : N);

@@ -26,7 +26,7 @@ struct Layer {
   size_t w_off = 0, b_off = 0;
 };
 
-int choose_bn(int M, int N);
+int choose_bn(int M, int N, int K = 0);
 
 // Brackets the kernel launches of one hot-path operation: counts launches and, when profiling
 // is enabled (hb_prof_enable), records CUDA events on the launch stream.
