@@ -21,11 +21,12 @@
 // W bytes in flight per SM (the shared memory left next to abuf) — so small batches use wide
 // clusters and b = 8192 uses CS = 2 (64 row blocks x 2 CTAs fill the 148 SMs once).
 //
-// Roles (384 threads): warp 0 TMA producer (X once, W tiles of every step in MMA order), warp 1
+// Roles (RC_THREADS = 640): warp 0 TMA producer (X once, W tiles of every step in MMA order), warp 1
 // MMA issuer (one thread, tcgen05.mma M=128 N=NH into one of two TMEM accumulators), warp 2 TMEM
-// allocator, warps 4..11 epilogue: quadrant q = warp % 4 (TMEM lanes = tile rows 32q..32q+31),
-// half h = (warp-4)/4 (columns 32h..32h+31 of every 64-column chunk; the two warps of a quadrant
-// meet on a named barrier before the chunk's 32-row piece is shipped).
+// allocator, warps 4..19 epilogue: quadrant q = warp % 4 (TMEM lanes = tile rows 32q..32q+31),
+// part h = (warp-4)/4 (columns 16h..16h+15 of every 64-column chunk; the RC_PARTS warps of a
+// quadrant meet on a named barrier before the chunk's 32-row piece is shipped, and lane 0 of
+// three of them issue the peer bulk copies, the H/dZ TMA store and the sigma' TMA store).
 //
 // Synchronisation (mbarriers):
 //   w_full/w_empty[stage]   W ring (TMA complete_tx / tcgen05.commit)
