@@ -23,7 +23,7 @@ for wdt in widths:
     m = hb.MLP(dims)
     m.set_params(params_to_flat(init_params(dims, seed=2)))
     for b in batches:
-        rows = min(N, max(b * 16, 65536)) // b * b
+        rows = min(N, max(b * 32, 262144)) // b * b  # >= 32 steps per epoch: stable device time
         w = hb.Worker(m, b)
         pol = hb.Policy(kind=hb.HB_MINIBATCH, workers=[hb.WorkerSpec(b, b, b)], eta0=0.0, b0=32)
         for _ in range(2):
@@ -31,7 +31,7 @@ for wdt in widths:
         e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
         torch.cuda.synchronize()
         e0.record()
-        st = hb.hogbatch_run([w], pol, Xd, yd, epochs=3, n=rows)
+        st = hb.hogbatch_run([w], pol, Xd, yd, epochs=5, n=rows)
         e1.record()
         torch.cuda.synchronize()
         sps = st["total_samples"] / (e0.elapsed_time(e1) * 1e-3)
