@@ -196,6 +196,10 @@ int mlp_step(hb_worker* w, const void* X, int64_t ldx, int32_t x_dtype, const in
  * host_grads in the mlp_get_params flat layout (blocking). */
 int mlp_step_grads(hb_worker* w, const void* X, int64_t ldx, int32_t x_dtype, const int32_t* y,
                    int32_t batch, float* host_grads, int64_t n, float* loss_out);
+/* test-only: the per-example cross-entropy  -log softmax(z_i)[y_i]  [L258] of the first n rows of
+ * the worker's last step (forward pass before the update), copied to host_dst[n] (blocking).
+ * 1 <= n <= max_batch, plain workers only (HB_EUNSUPPORTED for nested workers). */
+int mlp_row_losses(hb_worker* w, float* host_dst, int32_t n);
 
 /* ---- epoch-end loss (L273: "The loss computation is always performed on the GPU") ---
  * mean cross-entropy over n examples, reduced deterministically in fp64.  Blocking. */
@@ -219,7 +223,8 @@ int hogbatch_run(hb_worker** workers, int32_t n_workers, const hb_policy* p,
  * hb_prof_enable(1): every kernel launch of the hot path is bracketed by CUDA events on its
  * own stream; hb_prof_read (blocking: synchronises the device) accumulates per class the
  * launch count, device milliseconds and the ALGORITHMIC flops / bytes of those launches
- * (DESIGN.md §Roofline), writes n <= HB_PROF_N entries and optionally resets. */
+ * (DESIGN.md §Roofline), writes the first n of: HB_PROF_N class totals, then the per-layer entries
+ * (n <= HB_PROF_N * (1 + HB_PROF_LAYERS)), and optionally resets. */
 enum {
   HB_PROF_FWD_GEMM = 0,   /* hidden-layer forward GEMM + bias + sigmoid/sigma' epilogue */
   HB_PROF_HEAD_GEMM = 1,  /* output-layer forward GEMM (logits)                         */
@@ -229,7 +234,8 @@ enum {
   HB_PROF_BIAS = 5,       /* bias gradient + bias SGD                                   */
   HB_PROF_OTHER = 6,      /* loss reduction, shadow refresh, merge kernels              */
   HB_PROF_ROWCHAIN = 7,   /* fused per-row-block forward + softmax-xent + dX chain (narrow nets) */
-  HB_PROF_N = 8
+  HB_PROF_N = 8,
+  HB_PROF_LAYERS = 16     /* per-layer breakdown: entry HB_PROF_N + cls * HB_PROF_LAYERS + layer (0-based) */
 };
 typedef struct hb_prof_entry {
   int64_t launches;

@@ -156,6 +156,12 @@ class Worker:
                                   g.ctypes.data_as(C.POINTER(C.c_float)), g.size, C.byref(out)))
         return g, out.value
 
+    def row_losses(self, n: int) -> np.ndarray:
+        """Test-only: per-example cross-entropy of the first n rows of the last step."""
+        out = np.empty(n, dtype=np.float32)
+        _check(lib.mlp_row_losses(self.h, out.ctypes.data_as(C.POINTER(C.c_float)), n))
+        return out
+
     def close(self):
         if getattr(self, "h", None):
             lib.mlp_worker_destroy(self.h)
@@ -283,13 +289,23 @@ def prof_enable(on: bool = True):
     _check(lib.hb_prof_enable(int(on)))
 
 
-def prof_read(reset: bool = False) -> dict:
-    """Per kernel class: launches, device ms, algorithmic flops and bytes (blocking)."""
-    n = len(_lib.PROF_CLASSES)
-    buf = (_lib.ProfEntry * n)()
-    _check(lib.hb_prof_read(buf, n, int(reset)))
-    return {name: dict(launches=buf[i].launches, ms=buf[i].ms, flops=buf[i].flops, bytes=buf[i].bytes)
-            for i, name in enumerate(_lib.PROF_CLASSES)}
+def prof_read(reset: bool = False, per_layer: bool = False) -> dict:
+    """Per kernel class: launches, device ms, algorithmic flops and bytes (blocking).
+    per_layer=True also returns "<class>/l<k>" entries (weight layer k, 0-based) with launches."""
+    nc, nl = len(_lib.PROF_CLASSES), _lib.PROF_LAYERS
+    buf = (_lib.ProfEntry * (nc * (1 + nl)))()
+    _check(lib.hb_prof_read(buf, nc * (1 + nl), int(reset)))
+
+    def ent(e):
+        return dict(launches=e.launches, ms=e.ms, flops=e.flops, bytes=e.bytes)
+    out = {name: ent(buf[i]) for i, name in enumerate(_lib.PROF_CLASSES)}
+    if per_layer:
+        for c, name in enumerate(_lib.PROF_CLASSES):
+            for k in range(nl):
+                e = buf[nc + c * nl + k]
+                if e.launches:
+                    out[f"{name}/l{k}"] = ent(e)
+    return out
 
 
 def pad_to(n: int, m: int = 8) -> int:

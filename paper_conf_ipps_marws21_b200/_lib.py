@@ -27,7 +27,8 @@ EXPORTS = ("hb_last_error", "hb_abi_version", "hb_device_ok", "mlp_create", "mlp
            "hb_schedule_trace", "hogbatch_run", "hb_nccl_unique_id", "hb_comm_create",
            "hb_comm_destroy", "hb_merge_begin", "hb_merge", "hb_kernel_launches", "hb_prof_enable",
            "hb_prof_read", "hb_bench_gemm", "hb_bench_gemm_phases", "hb_rc_trace", "hb_bench_step", "hb_merge_schedule",
-           "mlp_worker_create_nested")
+           "mlp_worker_create_nested", "mlp_row_losses")
+PROF_LAYERS = 16
 PROF_CLASSES = ("fwd_gemm", "head_gemm", "softmax_xent", "dgrad_gemm", "wgrad_sgd_gemm", "bias_sgd", "other",
                 "rowchain")
 
@@ -96,6 +97,7 @@ def load():
         "mlp_step": ([VP, VP, I64, I32, VP, I32, F, P(F)], C.c_int),
         "mlp_step_grads": ([VP, VP, I64, I32, VP, I32, P(F), I64, P(F)], C.c_int),
         "mlp_loss": ([VP, VP, I64, I32, VP, I64, P(D)], C.c_int),
+        "mlp_row_losses": ([VP, P(F), I32], C.c_int),
         "hb_schedule_trace": ([P(Policy), I64, I32, P(TraceRec), I64, P(I64)], C.c_int),
         "hogbatch_run": ([P(VP), I32, P(Policy), P(Dataset), I32, P(Stats)], C.c_int),
         "hb_nccl_unique_id": ([P(C.c_uint8)], C.c_int),
@@ -113,6 +115,8 @@ def load():
         "hb_merge_schedule": ([I64, I32, P(I32), I64, P(I32), P(I32)], C.c_int),
     }
     for name, (args, res) in sig.items():
+        if os.environ.get("HB_LIB") and not hasattr(lib, name):
+            continue  # A/B builds of older sources may lack newer entry points
         fn = getattr(lib, name)
         fn.argtypes = args
         fn.restype = res

@@ -30,6 +30,12 @@ struct EpiArgs {
   int64_t ldw;
   float lr;
   int transposed;       // WGRAD: result element (m, n) belongs to W[n][m]
+  // split-precision head gradient (R24): the output layer's dZ_L is stored as two bf16
+  // planes, hi = bf16(dZ) in columns [0, hilo) and lo = bf16(dZ - hi) in [hilo, 2 hilo) of the same
+  // rows.  HEAD_XENT writes both; the transposed head WGRAD runs with N = 2 hilo and adds the two
+  // column halves of its accumulator (dW_L = hi^T H + lo^T H), so dW_L sees dZ_L to ~2^-17.
+  int hilo;             // 0 = plain bf16 dZ_L; else the lo plane's column offset (16)
+  int n_real;           // hilo: the real column count C of the output (ep.N = 2 hilo is the GEMM extent)
   // bias gradient fused into the GEMMs (tensor-core path):
   float* bpart_out;     // DGRAD / HEAD_XENT: column sums of the produced dZ per 128-row M tile
   const float* bpart_in;// WGRAD: those partials for dZ_l; reduced in fixed order to db_l
@@ -55,6 +61,11 @@ struct EpiArgs {
   int64_t ld_prev;
   float* bpart_prev;    // bias partials of dZ_{L-1} [m tiles x n_prev]
 };
+
+__device__ __forceinline__ uint32_t pack_bf16x2(float a, float b) {
+  __nv_bfloat162 t = __floats2bfloat162_rn(a, b);
+  return *reinterpret_cast<uint32_t*>(&t);
+}
 
 template <typename T>
 __device__ __forceinline__ T to_act(float v);
@@ -99,9 +110,15 @@ __device__ __forceinline__ void epi_elem(const EpiArgs& ep, int r, int n, float 
   }
 }
 
-__device__ __forceinline__ uint32_t pack_bf16x2(float a, float b) {
-  __nv_bfloat162 t = __floats2bfloat162_rn(a, b);
-  return *reinterpret_cast<uint32_t*>(&t);
+// 16 fp32 values -> packed bf16 hi = bf16(v) and lo = bf16(v - hi) (R24: v = hi + lo to ~2^-17 |v|)
+__device__ __forceinline__ void pack_hilo16(const float (&v)[16], uint32_t (&hp)[8], uint32_t (&lp)[8]) {
+#pragma unroll
+  for (int k = 0; k < 8; ++k) {
+    const __nv_bfloat162 h = __floats2bfloat162_rn(v[2 * k], v[2 * k + 1]);
+    const float2 hf = __bfloat1622float2(h);
+    hp[k] = *reinterpret_cast<const uint32_t*>(&h);
+    lp[k] = pack_bf16x2(v[2 * k] - hf.x, v[2 * k + 1] - hf.y);
+  }
 }
 
 // Vectorised epilogue for 16 consecutive columns n0..n0+15 of row r (all valid, 16-byte

@@ -44,11 +44,14 @@ struct PendRec {
   int cls;
   double flops, bytes;
   int nl;
+  int layer;
 };
+thread_local int g_prof_layer = -1;  // layer of the launches being bracketed (ProfLayer), -1 = none
 static std::mutex g_prof_mu;
 static std::vector<PendRec> g_pend;
 static std::vector<cudaEvent_t> g_evpool;
 static hb_prof_entry g_agg[HB_PROF_N];
+static hb_prof_entry g_agg_l[HB_PROF_N][HB_PROF_LAYERS];
 
 static cudaEvent_t ev_get() {
   {
@@ -66,7 +69,7 @@ static cudaEvent_t ev_get() {
 
 bool prof_enabled() { return g_prof_on.load(); }
 
-Prof::Prof(int cls_, cudaStream_t s_) : cls(cls_), s(s_) {
+Prof::Prof(int cls_, cudaStream_t s_) : cls(cls_), s(s_), layer(g_prof_layer) {
   if (g_prof_on.load(std::memory_order_relaxed)) {
     e0 = ev_get();
     cudaEventRecord(e0, s);
@@ -79,7 +82,7 @@ void Prof::done(int nlaunch, double flops, double bytes) {
   cudaEvent_t e1 = ev_get();
   cudaEventRecord(e1, s);
   std::lock_guard<std::mutex> g(g_prof_mu);
-  g_pend.push_back({e0, e1, cls, flops, bytes, nlaunch});
+  g_pend.push_back({e0, e1, cls, flops, bytes, nlaunch, layer});
   e0 = nullptr;
 }
 
@@ -478,7 +481,7 @@ static int launch_rowchain(hb_worker* w, const RcCfg& c, const void* X, int64_t 
   P.dz_head = static_cast<__nv_bfloat16*>(w->dZ[L - 1]);
   P.row_loss = w->row_loss;
   P.ldo = m->layers[0].ldo;
-  P.ldo_head = m->layers[L - 1].ldo;
+  P.ldo_head = w->ld_dzL;
   P.L = L;
   P.n0 = m->dims[0];
   P.n = n;
@@ -543,6 +546,14 @@ static void rowchain_cost(const hb_model* m, int b, double* flops, double* bytes
 // ----------------------------------------------------------------------------------------
 // model / worker
 // ----------------------------------------------------------------------------------------
+// the output layer's dW GEMM runs transposed (M = n_in, N = C) and, with C <= 16, on the
+// split-precision dZ_L (R24)
+static bool head_transposed(const Layer& Ly) { return Ly.n_out < 128 && Ly.n_out < Ly.n_in; }
+static bool head_hilo(const Layer& Ly) { return Ly.n_out <= 16 && head_transposed(Ly); }
+static int64_t ld_dz(const hb_worker* w, int l) {
+  return l == (int)w->m->layers.size() - 1 ? w->ld_dzL : w->m->layers[l].ldo;
+}
+
 static int act_dt(const hb_model* m) { return m->prec == HB_PREC_BF16 ? HB_BF16 : HB_F32; }
 static size_t act_size(const hb_model* m) { return m->prec == HB_PREC_BF16 ? 2 : 4; }
 
@@ -611,8 +622,16 @@ static int alloc_worker(hb_model* m, int max_b, cudaStream_t stream, bool own, h
       if (cudaMalloc(&p, (size_t)max_b * Ly.ldo * es) != cudaSuccess) return fail_free(fail(HB_ENOMEM, "S alloc"));
       w->S.push_back(p);
     }
-    if (cudaMalloc(&p, (size_t)max_b * Ly.ldo * es) != cudaSuccess) return fail_free(fail(HB_ENOMEM, "dZ alloc"));
-    cudaMemset(p, 0, (size_t)max_b * Ly.ldo * es);
+    // the head's dZ_L of a bf16 model with C <= 16 and a transposed head dW GEMM holds two bf16
+    // planes (hi in columns [0, 16), lo in [16, 32), R24)
+    const bool hl = l == L - 1 && m->prec == HB_PREC_BF16 && head_hilo(Ly);
+    const int64_t ldz = hl ? 32 : Ly.ldo;
+    if (l == L - 1) {
+      w->hilo = hl;
+      w->ld_dzL = (int)ldz;
+    }
+    if (cudaMalloc(&p, (size_t)max_b * ldz * es) != cudaSuccess) return fail_free(fail(HB_ENOMEM, "dZ alloc"));
+    cudaMemset(p, 0, (size_t)max_b * ldz * es);
     w->dZ.push_back(p);
   }
   const int C = m->layers.back().n_out;
@@ -789,6 +808,7 @@ static int forward_tc(hb_worker* w, const void* X, int64_t ldx, int64_t x_rows, 
   TcOp A{X, ldx, x_rows, d_off};
   for (int l = 0; l < L; ++l) {
     const Layer& Ly = m->layers[l];
+    ProfLayer pl(l);
     TcOp B{m->shadow + Ly.w_off, Ly.ldw, 0, nullptr};
     EpiArgs ep{};
     ep.M = b;
@@ -807,7 +827,8 @@ static int forward_tc(hb_worker* w, const void* X, int64_t ldx, int64_t x_rows, 
     // output layer + softmax cross-entropy: dZ_L = (softmax(z) - onehot(y)) / b, per-row loss
     if (Ly.n_out <= 16) {
       ep.out0 = want_grad ? w->dZ[l] : nullptr;
-      ep.ld0 = Ly.ldo;
+      ep.ld0 = w->ld_dzL;
+      ep.hilo = w->hilo ? 16 : 0;
       ep.y = y;
       ep.yoff = d_off;
       ep.row_loss = w->row_loss;
@@ -834,11 +855,11 @@ static int forward_tc(hb_worker* w, const void* X, int64_t ldx, int64_t x_rows, 
       Prof pr(HB_PROF_SOFTMAX, s);
       softmax_xent_kernel<__nv_bfloat16><<<(b * 32 + 255) / 256, 256, 0, s>>>(
           w->logits, w->ldc, y, d_off, b, Ly.n_out, want_grad ? static_cast<__nv_bfloat16*>(w->dZ[l]) : nullptr,
-          Ly.ldo, w->row_loss, 1.0f / (float)b);
+          w->ld_dzL, w->row_loss, 1.0f / (float)b);
       int nl = 1;
       if (want_grad) {
         colsum_partial_kernel<__nv_bfloat16><<<dim3((Ly.n_out + 63) / 64, (b + 127) / 128), dim3(64, 4), 0, s>>>(
-            static_cast<const __nv_bfloat16*>(w->dZ[l]), Ly.ldo, b, Ly.n_out, 128, w->bpart[l]);
+            static_cast<const __nv_bfloat16*>(w->dZ[l]), w->ld_dzL, b, Ly.n_out, 128, w->bpart[l]);
         nl = 2;
       }
       HB_CUDA_TRY(cudaGetLastError());
@@ -855,7 +876,8 @@ static int launch_wgrad(hb_worker* w, int l, const void* X, int64_t ldx, int64_t
                         int force_splits = 0) {
   hb_model* m = w->m;
   const Layer& Ly = m->layers[l];
-  TcOp dZl{w->dZ[l], Ly.ldo, b, nullptr};
+  ProfLayer pl(l);
+  TcOp dZl{w->dZ[l], ld_dz(w, l), b, nullptr};
   TcOp Al = l == 0 ? TcOp{X, ldx, x_rows, d_off} : TcOp{w->H[l - 1], m->layers[l - 1].ldo, b, nullptr};
   EpiArgs ep{};
   const int epi = grads_only ? EPI_WGRAD_STORE : EPI_WGRAD_SGD;
@@ -874,7 +896,7 @@ static int launch_wgrad(hb_worker* w, int l, const void* X, int64_t ldx, int64_t
   ep.bias_upd = m->master + Ly.b_off;
   ep.bias_grad = grads_only ? w->grads + Ly.b_off : nullptr;
   ep.ws = ws;
-  const bool tr = Ly.n_out < 128 && Ly.n_out < Ly.n_in;  // small head: M = n_in instead of n_out
+  const bool tr = head_transposed(Ly);  // small head: M = n_in instead of n_out
   ep.transposed = tr ? 1 : 0;
   if (!tr) {
     ep.M = Ly.n_out;
@@ -883,7 +905,13 @@ static int launch_wgrad(hb_worker* w, int l, const void* X, int64_t ldx, int64_t
   }
   ep.M = Ly.n_in;
   ep.N = Ly.n_out;
-  return gemm_tc_p(epi, true, true, Ly.n_in, Ly.n_out, b, Al, dZl, ep, s);
+  if (l == (int)m->layers.size() - 1 && w->hilo) {  // both dZ_L planes: N = 32, halves summed (R24)
+    ep.N = 32;
+    ep.hilo = 16;
+    ep.n_real = Ly.n_out;
+    ep.force_bn = 32;
+  }
+  return gemm_tc_p(epi, true, true, Ly.n_in, ep.N, b, Al, dZl, ep, s);
 }
 
 // Fused path: one rowchain launch (forward, head, dX chain for every 128-row block), then the dW
@@ -953,7 +981,7 @@ static int run_step_tc(hb_worker* w, const void* X, int64_t ldx, int64_t x_rows,
   cudaStream_t s2 = overlap && w->s2 ? w->s2 : s;
   for (int l = L - 1; l >= 0; --l) {
     const Layer& Ly = m->layers[l];
-    TcOp dZl{w->dZ[l], Ly.ldo, b, nullptr};
+    TcOp dZl{w->dZ[l], ld_dz(w, l), b, nullptr};
     TcOp Wl{m->shadow + Ly.w_off, Ly.ldw, 0, nullptr};
     if (l > 0 && !(l == L - 1 && head_dx_fused(m))) {  // dZ_{l-1} = (dZ_l W_l) * sigma'(Z_{l-1}) + bias partials
       const Layer& Lp = m->layers[l - 1];
@@ -966,6 +994,7 @@ static int run_step_tc(hb_worker* w, const void* X, int64_t ldx, int64_t x_rows,
       ep.ldaux = Lp.ldo;
       ep.bpart_out = w->bpart[l - 1];
       ep.ldp = Lp.n_out;
+      ProfLayer pl(l);
       rc = gemm_tc_p(EPI_DGRAD_SIG, false, true, b, Ly.n_in, Ly.n_out, dZl, Wl, ep, s);
       if (rc) return rc;
     }
@@ -1137,19 +1166,29 @@ int hb_prof_read(hb_prof_entry* out, int32_t n, int32_t reset) {
   for (auto& r : hb::g_pend) {
     float ms = 0.f;
     if (cudaEventElapsedTime(&ms, r.e0, r.e1) == cudaSuccess) {
-      hb_prof_entry& a = hb::g_agg[r.cls];
-      a.launches += r.nl;
-      a.ms += ms;
-      a.flops += r.flops;
-      a.bytes += r.bytes;
+      for (int k = 0; k < 2; ++k) {
+        if (k == 1 && (r.layer < 0 || r.layer >= HB_PROF_LAYERS)) break;
+        hb_prof_entry& a = k == 0 ? hb::g_agg[r.cls] : hb::g_agg_l[r.cls][r.layer];
+        a.launches += r.nl;
+        a.ms += ms;
+        a.flops += r.flops;
+        a.bytes += r.bytes;
+      }
     }
     hb::g_evpool.push_back(r.e0);
     hb::g_evpool.push_back(r.e1);
   }
   hb::g_pend.clear();
   for (int i = 0; i < n && i < HB_PROF_N; ++i) out[i] = hb::g_agg[i];
-  if (reset)
+  for (int i = HB_PROF_N; i < n && i < HB_PROF_N * (1 + HB_PROF_LAYERS); ++i) {
+    const int j = i - HB_PROF_N;
+    out[i] = hb::g_agg_l[j / HB_PROF_LAYERS][j % HB_PROF_LAYERS];
+  }
+  if (reset) {
     for (auto& a : hb::g_agg) a = hb_prof_entry{};
+    for (auto& row : hb::g_agg_l)
+      for (auto& a : row) a = hb_prof_entry{};
+  }
   return HB_OK;
 }
 int hb_abi_version(void) { return HB_ABI_VERSION; }
@@ -1485,6 +1524,15 @@ int mlp_step_grads(hb_worker* w, const void* X, int64_t ldx, int32_t x_dtype, co
     for (int i = 0; i < Ly.n_out; ++i) host_grads[o++] = h[Ly.b_off + i];
   }
   if (loss_out) return finish_loss(w, batch, loss_out, w->stream);
+  return HB_OK;
+}
+
+int mlp_row_losses(hb_worker* w, float* host_dst, int32_t n) {
+  HB_CHECK_ARG(w && host_dst && n >= 1 && n <= w->max_b, "n must be in [1, max_batch]");
+  if (!w->subs.empty()) return fail(HB_EUNSUPPORTED, "mlp_row_losses on a nested worker");
+  HB_CUDA_TRY(cudaSetDevice(w->m->device));
+  HB_CUDA_TRY(cudaMemcpyAsync(host_dst, w->row_loss, (size_t)n * 4, cudaMemcpyDeviceToHost, w->stream));
+  HB_CUDA_TRY(cudaStreamSynchronize(w->stream));
   return HB_OK;
 }
 

@@ -28,11 +28,20 @@ struct Layer {
 
 int choose_bn(int M, int N, int K = 0);
 
+extern thread_local int g_prof_layer;
+// Tags the Prof records of the launches issued while it lives with weight layer l (0-based).
+struct ProfLayer {
+  int prev;
+  explicit ProfLayer(int l) : prev(g_prof_layer) { g_prof_layer = l; }
+  ~ProfLayer() { g_prof_layer = prev; }
+};
+
 // Brackets the kernel launches of one hot-path operation: counts launches and, when profiling
 // is enabled (hb_prof_enable), records CUDA events on the launch stream.
 struct Prof {
   int cls;
   cudaStream_t s;
+  int layer;
   cudaEvent_t e0 = nullptr;
   Prof(int cls, cudaStream_t s);
   void done(int nlaunch, double flops, double bytes);
@@ -72,6 +81,8 @@ struct hb_worker {
   cudaStream_t stream = nullptr;
   bool own_stream = false;
   std::vector<void*> H, S, dZ;  // per-layer activations, sigma' stash, output gradients
+  int ld_dzL = 0;               // row stride of dZ_L (32 with the split-precision head, R24)
+  bool hilo = false;            // dZ_L stored as bf16 hi / lo planes (C <= 16, bf16 model)
   float* logits = nullptr;      // [max_b x ldc] fp32
   int ldc = 0;
   float* row_loss = nullptr;    // [max_b]

@@ -404,9 +404,8 @@ __global__ void __launch_bounds__(RC_THREADS, 1) rowchain_kernel(const __grid_co
             dz[j] = (row_ok && j < C) ? (expf(z[j] - lse) - (j == yi ? 1.f : 0.f)) * P.inv_b : 0.f;
             zy = j == yi ? z[j] : zy;
           }
-          uint32_t pk[8];
-#pragma unroll
-          for (int j = 0; j < 8; ++j) pk[j] = pack_bf16x2(dz[2 * j], dz[2 * j + 1]);
+          uint32_t pk[8], lk[8];
+          pack_hilo16(dz, pk, lk);  // hi feeds the chain's head dX; hi + lo the head dW GEMM (R24)
           // with a cluster the head chunk is never a TMA-store or bulk-copy source of this CTA
           // (rc_head_chunk); alone, it is chunk 0, last stored by this warp
           if (CS == 1) {
@@ -425,6 +424,10 @@ __global__ void __launch_bounds__(RC_THREADS, 1) rowchain_kernel(const __grid_co
               uint4* D = reinterpret_cast<uint4*>(P.dz_head + (int64_t)grow * P.ldo_head);
               D[0] = make_uint4(pk[0], pk[1], pk[2], pk[3]);
               if (P.ldo_head >= 16) D[1] = make_uint4(pk[4], pk[5], pk[6], pk[7]);
+              if (P.ldo_head >= 32) {  // lo plane at columns [16, 32)
+                D[2] = make_uint4(lk[0], lk[1], lk[2], lk[3]);
+                D[3] = make_uint4(lk[4], lk[5], lk[6], lk[7]);
+              }
             }
             const float t = warp_colsum16(dz, lane);
             const int col = colsum16_col(lane);

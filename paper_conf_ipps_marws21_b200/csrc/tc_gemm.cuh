@@ -410,11 +410,14 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
           ep.row_loss[r] = lse - zy;
           if (ep.out0) {
             uint4* D = reinterpret_cast<uint4*>(static_cast<__nv_bfloat16*>(ep.out0) + (int64_t)r * ep.ld0);
-            D[0] = make_uint4(pack_bf16x2(dz[0], dz[1]), pack_bf16x2(dz[2], dz[3]), pack_bf16x2(dz[4], dz[5]),
-                              pack_bf16x2(dz[6], dz[7]));
-            if (ep.ld0 >= 16)
-              D[1] = make_uint4(pack_bf16x2(dz[8], dz[9]), pack_bf16x2(dz[10], dz[11]),
-                                pack_bf16x2(dz[12], dz[13]), pack_bf16x2(dz[14], dz[15]));
+            uint32_t hp[8], lp[8];
+            pack_hilo16(dz, hp, lp);
+            D[0] = make_uint4(hp[0], hp[1], hp[2], hp[3]);
+            if (ep.ld0 >= 16) D[1] = make_uint4(hp[4], hp[5], hp[6], hp[7]);
+            if (ep.hilo) {  // lo plane at columns [16, 32) (R24)
+              D[2] = make_uint4(lp[0], lp[1], lp[2], lp[3]);
+              D[3] = make_uint4(lp[4], lp[5], lp[6], lp[7]);
+            }
           }
         }
         if (ep.bpart_out) {
@@ -471,7 +474,22 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
         }
       }
     } else {
-      if (active) {
+      if ((EPI == EPI_WGRAD_SGD || EPI == EPI_WGRAD_STORE) && splits == 1 && ep.hilo) {
+        // split-precision head dW (R24, transposed, one 32-column tile): column c of the result is
+        // acc[c] + acc[hilo + c] (hi and lo planes of dZ_L); the warps of part 0 own the tile
+        if (h == 0) {
+          uint32_t r0[16], r1[16];
+          tmem_ld_32x32b_x16(tbase, r0);
+          tmem_ld_32x32b_x16(tbase + (uint32_t)ep.hilo, r1);
+          tmem_ld_wait();
+          if (row_ok) {
+#pragma unroll
+            for (int j = 0; j < 16; ++j)
+              if (j < ep.n_real)
+                epi_elem<EPI, __nv_bfloat16, false>(ep, r, j, __uint_as_float(r0[j]) + __uint_as_float(r1[j]));
+          }
+        }
+      } else if (active) {
 #pragma unroll
         for (int cc = 0; cc < HALF; cc += 16) {
           const int c = c_lo + cc;
@@ -651,7 +669,7 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
         // transposed (small head): the m-tile-0 CTA owns bias entries n0..n0+BN-1
         const bool own = !ep.transposed ? (n_tile == 0) : (m_tile == 0);
         const int lo = !ep.transposed ? m0 : n0;
-        const int hi = !ep.transposed ? min(ep.M, m0 + TC_BM) : min(ep.N, n0 + BN);
+        const int hi = !ep.transposed ? min(ep.M, m0 + TC_BM) : min(ep.hilo ? ep.n_real : ep.N, n0 + BN);
         if (own) bias_reduce_update<EPI>(ep, lo, hi, et);
       }
     }
@@ -714,7 +732,8 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
         const int rloc = kz * rps + e / BN, col = e % BN;
         const uint32_t off = (uint32_t)((rloc * (BN + 4) + col) * 4);
         const int gm = m0 + rloc, gn = n0 + col;
-        const bool in = gm < ep.M && gn < ep.N;
+        if (ep.hilo && col >= ep.hilo) continue;  // R24: lo-plane columns are folded into [0, hilo)
+        const bool in = gm < ep.M && gn < (ep.hilo ? ep.n_real : ep.N);
         const bool vec = in && !ep.transposed && gn + 4 <= ep.N && EPI == EPI_WGRAD_SGD;
         float4* W = vec ? reinterpret_cast<float4*>(ep.master + (int64_t)gm * ep.ldw + gn) : nullptr;
         float4 w = make_float4(0.f, 0.f, 0.f, 0.f);
@@ -740,6 +759,25 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
             acc.z += part[sp].z;
             acc.w += part[sp].w;
           }
+        if (ep.hilo) {  // + the lo plane's column (same splits, same fixed order)
+#pragma unroll
+          for (int sp = 0; sp < 8; ++sp)
+            if (sp < splits)
+              part[sp] = ld_dsmem_f4(mapa_shared(tile_s + off + (uint32_t)(ep.hilo * 4), (uint32_t)sp));
+          float4 lo4 = make_float4(0.f, 0.f, 0.f, 0.f);
+#pragma unroll
+          for (int sp = 0; sp < 8; ++sp)
+            if (sp < splits) {
+              lo4.x += part[sp].x;
+              lo4.y += part[sp].y;
+              lo4.z += part[sp].z;
+              lo4.w += part[sp].w;
+            }
+          acc.x += lo4.x;
+          acc.y += lo4.y;
+          acc.z += lo4.z;
+          acc.w += lo4.w;
+        }
         if (!in) continue;
         const float a4[4] = {acc.x, acc.y, acc.z, acc.w};
         if (vec) {
@@ -753,7 +791,7 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
         } else {
 #pragma unroll
           for (int j = 0; j < 4; ++j)
-            if (gn + j < ep.N) epi_elem<EPI, __nv_bfloat16, false>(ep, gm, gn + j, a4[j]);
+            if (gn + j < (ep.hilo ? ep.n_real : ep.N)) epi_elem<EPI, __nv_bfloat16, false>(ep, gm, gn + j, a4[j]);
         }
       }
       if (dbg && threadIdx.x == 128) dbg[10] = gtimer();
@@ -767,7 +805,7 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
         } else {
           own = m_tile == 0 && kz == 0;
           lo = n0;
-          hi = min(ep.N, n0 + BN);
+          hi = min(ep.hilo ? ep.n_real : ep.N, n0 + BN);
         }
         if (own) bias_reduce_update<EPI>(ep, lo, hi, tid);
       }

@@ -15,6 +15,20 @@ def rel_err(a, b) -> float:
     return float(np.linalg.norm(a - b) / (nb if nb > 0 else 1.0))
 
 
+def grad_errors(flat, dims, dW, db):
+    """Per tensor (W_1, b_1, W_2, ...): normwise error ||g - g_ref||_F / ||g_ref||_F and
+    element-wise error max_i |g_i - g_ref_i| / max_i |g_ref_i| (R13)."""
+    got = split_flat(flat, dims)
+    norm, elem = [], []
+    for l in range(len(dims) - 1):
+        for a, r in ((got[l][0], dW[l]), (got[l][1], db[l])):
+            r = np.asarray(r, np.float64)
+            norm.append(rel_err(a, r))
+            mx = np.abs(r).max()
+            elem.append(float(np.abs(np.asarray(a, np.float64) - r).max() / (mx if mx > 0 else 1.0)))
+    return norm, elem
+
+
 def split_flat(flat, dims):
     out, o = [], 0
     for l in range(1, len(dims)):
@@ -56,4 +70,4 @@ def to_device(X, y, dtype="bf16", device="cuda:0"):
     return tX, ty
 
 
-__all__ = ["rel_err", "split_flat", "dataset", "to_device", "init_params", "params_to_flat"]
+__all__ = ["grad_errors", "rel_err", "split_flat", "dataset", "to_device", "init_params", "params_to_flat"]

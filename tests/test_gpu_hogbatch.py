@@ -9,7 +9,8 @@ pytestmark = pytest.mark.gpu
 import paper_conf_ipps_marws21_b200 as hb  # noqa: E402
 from oracle import coord as ocoord  # noqa: E402
 from oracle import mlp64, serial  # noqa: E402
-from tests.helpers import dataset, init_params, params_to_flat, rel_err, split_flat, to_device  # noqa: E402
+from tests.helpers import (dataset, grad_errors, init_params, params_to_flat, rel_err, split_flat,  # noqa: E402
+                           to_device)
 
 
 def _gpu():
@@ -35,22 +36,47 @@ def o_policy(kind, workers, eta0, b0):
 
 @pytest.mark.parametrize("prec,tol", [("bf16", 1e-2), ("fp32", 1e-5)])
 def test_deterministic_minibatch_trajectory_100_steps(prec, tol):
-    # C1: 54-64-64-7, b = 32, SERIAL mode: per-step batch loss within tol of the oracle for 100 steps
+    # C1: 54-64-64-7, b = 32, SERIAL mode at the survey's eta0 = 1: per-step batch loss within tol of
+    # the oracle for 100 steps.  The round-1 kernels drifted 1.3e-2 at step 6 — reproduced exactly by
+    # scripts/bf16_emulation.py and traced to the bf16 rounding of dZ_L in the head's dW GEMM; the
+    # split-precision head (R24) predicts 4.5e-3 (profiles/r02_bf16_emulation.txt)
     dims = [54, 64, 64, 7]
     X, y, m, params, tX, ty = setup(dims, prec, 32, 10000)
     specs = [hb.WorkerSpec(32, 32, 32)]
-    # eta0 = 0.3: at eta0 = 1 the bf16 rounding of the activations alone moves step 6 by 1.3e-2
-    # (reproduced exactly by a bf16 emulation of the same arithmetic)
-    pol = hb.Policy(kind=hb.HB_MINIBATCH, workers=specs, eta0=0.3, b0=32, deterministic=True, max_steps=100)
+    pol = hb.Policy(kind=hb.HB_MINIBATCH, workers=specs, eta0=1.0, b0=32, deterministic=True, max_steps=100)
     w = hb.Worker(m, 32)
     st = hb.hogbatch_run([w], pol, tX, ty, epochs=1, trace_cap=200, step_loss_cap=100)
     assert st["n_steps"] == 100
-    recs = ocoord.run(o_policy(ocoord.MINIBATCH, specs, 0.3, 32), 10000, 1)
+    recs = ocoord.run(o_policy(ocoord.MINIBATCH, specs, 1.0, 32), 10000, 1)
     _, ref = serial.run_trace(params, X.astype(np.float64), y, recs, max_steps=100)
     got = np.array(st["step_loss"])
     rel = np.abs(got - np.array(ref)) / np.array(ref)
+    print("C1 trajectory max rel", prec, rel.max(), rel.argmax())
     assert rel.max() <= tol, (rel.max(), rel.argmax())
     assert ref[-1] < ref[0]
+
+
+def test_c2_fused_chain_trajectory_100_steps():
+    # SURVEY §8(c) "C2 truncated to 100 steps": 54-512x4-7 at b = 8192 — the fused row-block chain
+    # plus the concurrent dW GEMMs, the bench's launch configuration — in SERIAL mode for 100 steps,
+    # per-step batch loss within 1e-2 of the fp64 oracle's (tests/golden/c2_trajectory.json, written
+    # by scripts/make_goldens.py from oracle/ only; eta0 = 0.001 at b0 = 32 -> lr 0.256 [L179, L258])
+    import json
+    import os
+    gold = json.load(open(os.path.join(os.path.dirname(__file__), "golden", "c2_trajectory.json")))
+    dims, b = gold["dims"], gold["b"]
+    X, y, m, params, tX, ty = setup(dims, "bf16", b, gold["N"])
+    w = hb.Worker(m, b)
+    assert m.fused_path(b) > 0  # the fused chain is the path under test
+    spec = hb.WorkerSpec(b, b, b)
+    pol = hb.Policy(kind=hb.HB_MINIBATCH, workers=[spec], eta0=gold["eta0"], b0=gold["b0"], deterministic=True,
+                    max_steps=gold["steps"])
+    st = hb.hogbatch_run([w], pol, tX, ty, epochs=2, step_loss_cap=gold["steps"])
+    assert st["n_steps"] == gold["steps"]
+    ref = np.array(gold["losses"])
+    rel = np.abs(np.array(st["step_loss"]) - ref) / ref
+    print("C2 fused trajectory max rel", rel.max(), rel.argmax())
+    assert rel.max() <= 1e-2, (rel.max(), rel.argmax())
 
 
 def test_deterministic_adaptive_serial_matches_oracle():
@@ -60,6 +86,10 @@ def test_deterministic_adaptive_serial_matches_oracle():
     N = 4096
     X, y, m, params, tX, ty = setup(dims, "bf16", 512, N)
     specs = [hb.WorkerSpec(16, 128, 16, 1.0, 0.0, 1.0), hb.WorkerSpec(64, 512, 512, 1.0, 20.0, 0.05)]
+    # eta0 = 0.05: at 0.5 (lr 8 at b = 512) the fp64 trajectory itself is unstable (batch loss
+    # 2.3 -> 1.3 -> 9.1 -> 17.7), where any rounding is amplified without bound: the bf16 emulation
+    # gives 4.9e-3 with the round-1 head and 1.9e-2 with the more precise R24 head — chance, not
+    # accuracy (R25, profiles/r02_bf16_emulation.txt); at 0.05 both stay below 3e-3
     pol = hb.Policy(kind=hb.HB_ADAPTIVE, workers=specs, eta0=0.05, b0=32, deterministic=True)
     ws = [hb.Worker(m, 128), hb.Worker(m, 512)]
     st = hb.hogbatch_run(ws, pol, tX, ty, epochs=2, trace_cap=10000, step_loss_cap=10000)
@@ -71,6 +101,22 @@ def test_deterministic_adaptive_serial_matches_oracle():
     assert len(got) == len(ref) > 20
     assert (np.abs(got - ref) / np.array(ref)).max() <= 1e-2
     assert {r[6] for r in st["trace"]} >= {"halve", "double"}
+
+
+@pytest.mark.parametrize("dims", [[54, 256, 128, 7], [54, 512, 512, 512, 7]])
+def test_serial_run_is_bitwise_reproducible(dims):
+    # deterministic mode (SERIAL, direct launches with the backward overlap and programmatic
+    # dependent launches): every run of the same schedule gives the same bits — caught an
+    # out-of-range column write of the split-K head dW epilogue racing with the bias update
+    out = set()
+    for _ in range(4):
+        X, y, m, params, tX, ty = setup(dims, "bf16", 512, 4500)
+        w = hb.Worker(m, 512)
+        pol = hb.Policy(kind=hb.HB_MINIBATCH, workers=[hb.WorkerSpec(512, 512, 512)], eta0=0.1, b0=32,
+                        deterministic=True)
+        hb.hogbatch_run([w], pol, tX, ty, epochs=2)
+        out.add(m.get_params().tobytes())
+    assert len(out) == 1
 
 
 def test_graph_replay_is_bitwise_equal_to_direct_launches():
@@ -127,6 +173,8 @@ def test_concurrent_adaptive_hogwild_trains_and_respects_thresholds():
     N = 40000
     X, y, m, params, tX, ty = setup(dims, "bf16", 2048, N)
     specs = [hb.WorkerSpec(256, 2048, 2048), hb.WorkerSpec(32, 256, 32)]
+    # eta0 = 0.02: at 0.5 (lr 32 at b = 2048) plain fp64 mini-batch SGD on this net diverges
+    # (full loss 2.09 -> 80 after 3 epochs; 0.05 -> 0.99, 0.02 -> 1.23), R25
     pol = hb.Policy(kind=hb.HB_ADAPTIVE, workers=specs, eta0=0.02, b0=32, eval_loss=True)
     ws = [hb.Worker(m, 2048), hb.Worker(m, 256)]
     l0 = mlp64.full_loss(params, X.astype(np.float64), y)
@@ -193,29 +241,33 @@ def test_full_size_gradient_parity(dims, kind, b):
     assert abs(loss - l_ref) / l_ref <= 1e-2
 
 
-def test_full_size_c4_batch_gradient_is_mean_of_subbatch_gradients():
-    # configs[3] at the full batch b = 8192 in the launch configuration the bench times (the
-    # oracle cannot afford 5 TFLOP of fp64 here): the batch gradient is the mean of the gradients
-    # of its 32 sub-batches of 256 (a property of Eq. (2) at any size), and those sub-batch
-    # gradients are oracle-checked by test_full_size_gradient_parity
+def test_full_size_c4_step_matches_oracle_at_b8192():
+    # configs[3] (C4, 20958-4096x4-2) at b = 8192, the launch configuration bench.py times, against
+    # the fp64 oracle (about 5 TFLOP of fp64: ~30-60 s on the box's host cores).  Gradient bound
+    # (R25): normwise <= 1e-2 per tensor (north star); element-wise <= 2.5e-2 of the
+    # tensor's max — the bf16 emulation of this step (scripts/bf16_emulation.py) gives 9.4e-3 /
+    # 1.5e-2 here, the cancellations of a 4096-wide sigmoid chain in its near-linear regime
     _gpu()
-    dims, b, sb = [20958, 4096, 4096, 4096, 4096, 2], 8192, 256
+    dims, b = [20958, 4096, 4096, 4096, 4096, 2], 8192
     X, y = dataset("realsim", b, d=dims[0], seed=5)
     m = hb.MLP(dims)
-    m.set_params(params_to_flat(init_params(dims)))
+    params = init_params(dims)
+    m.set_params(params_to_flat(params))
     w = hb.Worker(m, b)
+    assert m.fused_path(b) == 0  # the per-layer tcgen05 GEMM chain, as benched
     tX, ty = to_device(X, y)
-    g_full, loss_full = w.step_grads(tX, ty, b)
-    acc, losses = None, []
-    for k in range(b // sb):
-        g, l = w.step_grads(tX[k * sb:], ty[k * sb:], sb)
-        acc = g.astype(np.float64) if acc is None else acc + g
-        losses.append(l)
-    g_mean = acc / (b // sb)
-    got, ref = split_flat(g_full, dims), split_flat(g_mean, dims)
-    errs = [max(rel_err(got[l][0], ref[l][0]), rel_err(got[l][1], ref[l][1])) for l in range(len(dims) - 1)]
-    assert max(errs) <= 1e-2, errs
-    assert abs(loss_full - np.mean(losses)) / np.mean(losses) <= 1e-3
+    g, loss = w.step_grads(tX, ty, b)
+    rows = w.row_losses(b)
+    del tX
+    dW, db, l_ref = mlp64.grads(params, X.astype(np.float64), y)
+    norm, elem = grad_errors(g, dims, dW, db)
+    print("C4 b=8192 normwise", np.round(norm, 5).tolist(), "element-wise", np.round(elem, 5).tolist())
+    assert max(norm) <= 1e-2, norm
+    assert max(elem) <= 2.5e-2, elem
+    assert abs(loss - l_ref) / l_ref <= 1e-2
+    Z, _ = mlp64.forward(params, X[:512].astype(np.float64))
+    ref_rows = mlp64.xent_rows(Z[-1], y[:512])
+    assert (np.abs(rows[:512] - ref_rows) / np.maximum(1.0, ref_rows)).max() <= 1e-2
 
 
 def test_nested_worker_serial_matches_oracle():
@@ -269,7 +321,7 @@ def test_nested_hogwild_worker_in_adaptive_run():
     st = hb.hogbatch_run(ws, pol, tX, ty, epochs=2, trace_cap=100000)
     assert st["epoch_loss"][-1] < 0.95 * l0
     small = [r for r in st["trace"] if r[2] == 1 and r[9]]
-    assert small and all(r[8] - r[4] in (0.0,) or True for r in small)
+    assert small
     # the nested worker's counter advances by t*beta = 8 per served batch (dispatch credit, R21)
     prev = None
     for r in st["trace"]:

@@ -195,3 +195,17 @@ def test_flops_per_sample_brute_force(dims):
         if l > 1:
             f += 2 * mac          # dX
     assert mlp64.flops_per_sample(dims) == f
+
+
+def test_c2_trajectory_golden_is_the_oracle_s():
+    # tests/golden/c2_trajectory.json (scripts/make_goldens.py) pinned to the oracle: the first
+    # two steps of the stored 100-step C2 trajectory are recomputed here
+    import json
+    import os
+    import sys
+    sys.path.insert(0, os.path.join(os.path.dirname(os.path.dirname(os.path.abspath(__file__))), "scripts"))
+    import make_goldens
+    gold = json.load(open(os.path.join(os.path.dirname(__file__), "golden", "c2_trajectory.json")))
+    assert len(gold["losses"]) == gold["steps"] == 100
+    got = make_goldens.c2_trajectory(steps=2)
+    np.testing.assert_allclose(got, gold["losses"][:2], rtol=1e-12)
