@@ -24,7 +24,7 @@
 extern "C" {
 #endif
 
-#define HB_ABI_VERSION 1
+#define HB_ABI_VERSION 2
 
 /* status codes */
 enum {
@@ -67,6 +67,7 @@ enum { HB_ACT_NONE = 0, HB_ACT_HALVE = 1, HB_ACT_DOUBLE = 2, HB_ACT_CLAMP_LO = 3
 typedef struct hb_model hb_model;
 typedef struct hb_worker hb_worker;
 typedef struct hb_comm hb_comm;
+typedef struct hb_coord hb_coord;
 
 /* Per-worker policy (Algorithm 2 inputs min_b^E, max_b^E [L194]; initial size [L236]). */
 typedef struct hb_worker_policy {
@@ -90,8 +91,18 @@ typedef struct hb_policy {
   int32_t merges_per_epoch; /* multi-GPU: replica merges per epoch (needs comm; 0 = none)     */
   float merge_gamma;     /* W <- W_base + gamma * sum(W_E - W_base); 1 = delta sum (R18)     */
   hb_comm* comm;         /* nullable; NCCL communicator for the merge                         */
-  int32_t n_workers;     /* entries in workers[]                                              */
+  int32_t n_workers;     /* entries in workers[] (with a shared coordinator: ALL processes' workers) */
   const hb_worker_policy* workers;
+  int32_t update;        /* -1: each model's HB_OPT_UPDATE; HB_UPDATE_HOGWILD / HB_UPDATE_ATOMIC for
+                            this run (concurrent in-place updates of the shared model [L128])   */
+  int32_t epoch_barrier; /* 1 (default): an epoch ends when no worker can be served and all are idle
+                            [L170]; 0: as soon as a worker cannot be served, the next epoch starts
+                            without waiting for the others' in-flight batches (no idle bubble;
+                            not with merges)                                                    */
+  int32_t check_labels;  /* 1: verify every label is in [0, C) before training (HB_EINVAL)      */
+  struct hb_coord* coord;/* nullable: cross-process coordinator (hb_coord_create): one 𝔹 and one
+                            Algorithm 2 state for the workers of every process of the node     */
+  int32_t first_worker;  /* with coord: global id of this process's workers[0]                 */
 } hb_policy;
 
 /* Training data (borrowed; caller-owned).  X and y are both device pointers (used in place) or
@@ -157,23 +168,61 @@ int mlp_num_params(const hb_model* m, int64_t* n_out);
  * returns 1 and sets *cluster_size (1, 2, 4 or 8 CTAs per 128-row block) if SGD steps take the fused
  * row-block chain (one kernel for forward, softmax-xent head and the whole dX chain, then the dW
  * GEMMs; eligible: bf16 model, uniform hidden width n <= 512, n_0 <= 512, C <= 16, 2..12 layers,
- * not disabled with HB_ROWCHAIN=0), 0 if they take the per-layer GEMM chain, < 0 on error. */
+ * HB_OPT_ROWCHAIN = 1, batch >= HB_OPT_FUSED_MIN_BATCH), 0 if they take the per-layer GEMM chain,
+ * < 0 on error. */
 int mlp_fused_path(const hb_model* m, int32_t batch, int32_t* cluster_size);
-/* Steps of at least min_batch rows take the fused row-block chain when the shape is eligible
- * (0 = never; default 4096 = the measured crossover on B200, or HB_RC_MIN_B).  Workers created
- * afterwards allocate what the fused path needs; set it before mlp_worker_create. */
-int mlp_set_fused_min_batch(hb_model* m, int32_t min_batch);
+/* Per-model settings (defaults = the measured B200 choices; none is read from the environment):
+ *   HB_OPT_FUSED_MIN_BATCH  steps of >= value rows take the fused row-block chain when the shape is
+ *                           eligible (0 = never; default 4096, the measured crossover).  Set before
+ *                           creating workers (they allocate what the fused path needs).
+ *   HB_OPT_ROWCHAIN         1 = fused row-block chain allowed (default), 0 = per-layer GEMM chain
+ *   HB_OPT_RC_CLUSTER       CTAs per 128-row block of the fused chain: 1, 2, 4, 8 or 0 = auto
+ *   HB_OPT_BWD_OVERLAP      1 = dW_l runs on a second stream overlapping dX_{l-1} (default)
+ *   HB_OPT_HEAD_FUSE        1 = the output layer's dX runs in the head GEMM's epilogue (C <= 16;
+ *                           default 0, measured slower at b = 8192)
+ *   HB_OPT_DW_PAIR          1 = split-K dW GEMMs with 256-wide tiles run on CTA pairs
+ *                           (tcgen05 cta_group::2; default 0, measured not faster)
+ *   HB_OPT_PDL              1 = programmatic dependent launch between the step's kernels (default)
+ *   HB_OPT_GRAPHS           1 = hogbatch_run replays one CUDA graph per (batch size, lr) (default)
+ *   HB_OPT_INFLIGHT         steps a worker may have enqueued before the oldest completes in
+ *                           hogbatch_run (1..4; 0 = auto: 2 for a single worker, else 1, R23)
+ *   HB_OPT_STAGE_ROWS       rows per H2D staging chunk of a host dataset (0 = auto: <= 32768 rows
+ *                           and <= 32 MB)
+ *   HB_OPT_UPDATE           HB_UPDATE_HOGWILD (plain read-modify-write of the shared model, Hogwild
+ *                           [L128, L170]; default) or HB_UPDATE_ATOMIC (the dW epilogue adds -lr*dW
+ *                           with atomic adds: no concurrent update is lost)
+ * Unknown key or out-of-range value -> HB_EINVAL. */
+enum {
+  HB_OPT_FUSED_MIN_BATCH = 0, HB_OPT_ROWCHAIN = 1, HB_OPT_RC_CLUSTER = 2, HB_OPT_BWD_OVERLAP = 3,
+  HB_OPT_HEAD_FUSE = 4, HB_OPT_DW_PAIR = 5, HB_OPT_PDL = 6, HB_OPT_GRAPHS = 7, HB_OPT_INFLIGHT = 8,
+  HB_OPT_STAGE_ROWS = 9, HB_OPT_UPDATE = 10
+};
+enum { HB_UPDATE_HOGWILD = 0, HB_UPDATE_ATOMIC = 1 };
+int mlp_set_option(hb_model* m, int32_t key, int64_t value);
+int mlp_get_option(const hb_model* m, int32_t key, int64_t* value);
 /* host flat fp32 layout: [W_1 (n_1 x n_0 row-major, unpadded), b_1, W_2, b_2, ...]; n must equal
  * mlp_num_params.  Blocking.  set also refreshes the bf16 shadow. */
 int mlp_get_params(const hb_model* m, float* host_dst, int64_t n);
 int mlp_set_params(hb_model* m, const float* host_src, int64_t n);
 
 /* ---- worker (§V.A: GPU worker, exclusive device interface) ----------
- * max_batch >= 1 sizes the worker's activation scratch.  replica must be 0 (a reference
- * replica: the worker updates the shared model in place, Hogbatch L170).  cuda_stream may
- * be NULL (the worker creates its own non-blocking stream) or a borrowed cudaStream_t. */
-int mlp_worker_create(hb_model* m, int32_t max_batch, int32_t replica, void* cuda_stream,
+ * device: the model's device (or -1 for it; any other device -> HB_EUNSUPPORTED: one model per GPU,
+ * several GPUs = one process per GPU sharing a coordinator, hb_coord_create).  max_batch >= 1 sizes
+ * the worker's activation scratch.
+ * replica 0 = reference replica: the worker updates the shared (global) model in place (Hogbatch
+ *   [L170]; concurrent workers race, Hogwild [L128]).
+ * replica 1 = deep replica [L134, L174]: the worker owns a private copy of the global model's
+ *   parameters (taken at creation) and its steps update that copy; hb_merge_replicas (called by
+ *   hogbatch_run at its merge points) integrates it into the global model ("push", [L141, L175]).
+ *   Several deep replicas on one GPU emulate a multi-GPU replica run with the same merge arithmetic.
+ * cuda_stream may be NULL (the worker creates its own stream — a BLOCKING stream, so its work is
+ * ordered after the caller's legacy-default-stream work such as torch copies) or a borrowed
+ * cudaStream_t.  Destroy workers before their model. */
+int mlp_worker_create(hb_model* m, int32_t device, int32_t max_batch, int32_t replica, void* cuda_stream,
                       hb_worker** out);
+/* the worker's current parameters (a deep replica's private copy; the global model's for a
+ * reference replica) in the mlp_get_params layout (blocking) */
+int mlp_worker_params(hb_worker* w, float* host_dst, int64_t n);
 /* Nested worker: the GPU form of Algorithm 2's CPU worker [L224-L235].  Each ExecuteWork(B) is
  * split into t contiguous sub-batches (the first b mod t get ceil(b/t) rows) run concurrently on
  * t internal streams, each updating the shared model in place (Hogwild [L229-L232]) with
@@ -211,10 +260,34 @@ int mlp_loss(hb_model* m, const void* X, int64_t ldx, int32_t x_dtype, const int
  * over N examples for `epochs` epochs, without touching any GPU; writes up to cap records. */
 int hb_schedule_trace(const hb_policy* p, int64_t N, int32_t epochs, hb_trace_rec* out,
                       int64_t cap, int64_t* n_out);
+/* ---- shared coordinator (multi-GPU: one process per GPU, one coordinator for the node) ----
+ * PAPER.md L123 (one coordinator owns the data), L218–L220 (one set 𝔹 of remaining examples),
+ * L130/L185 (the batch sizes adapt to the relative speed of ALL workers).  The Algorithm 2 state,
+ * the epoch cursor over 𝔹 and the run control live in POSIX shared memory `name` ("/..."): rank 0
+ * creates and initialises it from p (the global worker specs; N examples), the other ranks attach
+ * (waiting up to 60 s for rank 0).  Pass it as hb_policy.coord (with first_worker = the global id of
+ * the process's first worker) to hogbatch_run on every rank: the processes join each run before
+ * any schedules, the epoch ends when every worker of every process is idle, and each process
+ * performs every issued merge (its NCCL collective) in order.  Destroy after the last run
+ * (rank 0 unlinks the segment).  A peer that stops responding surfaces as HB_ESTATE after 30 min. */
+int hb_coord_create(const char* name, const hb_policy* p, int64_t N, int32_t nranks, int32_t rank, hb_coord** out);
+int hb_coord_destroy(hb_coord* c);
+/* test / custom-driver entry points on the shared state (no GPU, no run in progress):
+ * reset to a fresh run of policy p over N examples; one ScheduleWork(worker) at time `now`; the
+ * worker idles because it could not be served (*epoch_ended = 1 if every worker now idles: the
+ * cursor returns to row 0 and the epoch advances, Alg. 1 [L170]) */
+int hb_coord_reset(hb_coord* c, const hb_policy* p, int64_t N);
+int hb_coord_schedule(hb_coord* c, int32_t worker, double now, hb_trace_rec* out);
+int hb_coord_idle(hb_coord* c, int32_t worker, int32_t* epoch_ended);
+
 /* Trains with n_workers workers (one host thread each, concurrent Hogbatch updates of the
  * shared model, L170) under policy p for `epochs` epochs over data (device or host, see
- * hb_dataset).  Blocking.
- * p->deterministic = 1 executes the virtual-clock trace serially (SERIAL policy, L125). */
+ * hb_dataset).  Blocking.  All workers belong to one global model (reference or deep replicas;
+ * deep replicas need merges_per_epoch >= 1 and are merged with hb_merge_replicas, reference
+ * workers of different processes with hb_merge over p->comm).
+ * p->deterministic = 1 executes the virtual-clock trace serially (SERIAL policy, L125).
+ * Stats arrays indexed by worker are indexed by the GLOBAL worker id (p->n_workers entries per
+ * epoch); with a shared coordinator each process fills its own workers' entries and trace. */
 int hogbatch_run(hb_worker** workers, int32_t n_workers, const hb_policy* p,
                  const hb_dataset* data, int32_t epochs, hb_stats* stats_out);
 
@@ -244,22 +317,16 @@ typedef struct hb_prof_entry {
 int64_t hb_kernel_launches(void);
 int hb_prof_enable(int32_t on);
 int hb_prof_read(hb_prof_entry* out, int32_t n, int32_t reset);
-/* tuning only: mean device microseconds of one tensor-core GEMM launch of the given kind
- * (0 forward+sigmoid, 1 dgrad+sigma', 2 wgrad+SGD) and shape on zero-filled scratch buffers */
-int hb_bench_gemm(int32_t kind, int32_t M, int32_t N, int32_t K, int32_t iters, float* us_out);
-/* tuning only: per-CTA phase timestamps (8 globaltimer ns values per CTA, cap entries) of one launch */
-/* tuning only: hb_rc_trace(NULL, cap) arms per-step globaltimer stamps (10 per CTA per step, 24 steps
- * per CTA) in later fused row-block launches; hb_rc_trace(host, cap) reads the last launch's */
-int hb_rc_trace(unsigned long long* host, int64_t cap);
-/* tuning only: mean device microseconds of one SGD step (graph-replayed `iters` times, lr = 0) on
- * rows [0, batch) of X/y; part 0 = whole step, 1 = fused chain only, 2 = dW GEMMs only */
-int hb_bench_step(hb_worker* w, const void* X, int64_t ldx, const int32_t* y, int32_t batch, int32_t iters,
-                  int32_t part, float* us_out);
-int hb_bench_gemm_phases(int32_t kind, int32_t M, int32_t N, int32_t K, unsigned long long* host_ts, int64_t cap);
 
-/* Merge points of one rank for one epoch of served batch sizes batches[0..n):
+/* Local replica merge (deep replicas of this process): with B the merge base
+ * (hb_merge_begin / the previous merge), G <- G + gamma * sum_E (R_E - B) over the deep-replica
+ * workers among workers[0..n) (fixed order; reference replicas contribute through G itself), then
+ * B <- G and every replica R_E <- G (bf16 shadows rewritten).  Blocking; at most 8 deep replicas. */
+int hb_merge_replicas(hb_model* m, hb_worker* const* workers, int32_t n, float gamma);
+
+/* Merge points of one epoch of served batch sizes batches[0..n) over N examples:
  * mid_epoch_out = merges due while serving, total_out = merges performed in the epoch (always
- * merges_per_epoch, so ranks with different batch-size dynamics issue the same collectives). */
+ * merges_per_epoch: the rest is issued at the epoch end). */
 int hb_merge_schedule(int64_t N, int32_t merges_per_epoch, const int32_t* batches, int64_t n_batches,
                       int32_t* mid_epoch_out, int32_t* total_out);
 

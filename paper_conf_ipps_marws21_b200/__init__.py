@@ -17,7 +17,7 @@ import numpy as np
 from . import _lib
 from ._lib import (ACTIONS, HB_ADAPTIVE, HB_BF16, HB_CREDIT_COMPLETION, HB_CREDIT_DISPATCH, HB_F32,  # noqa: F401
                    HB_HOGBATCH, HB_MINIBATCH, HB_PREC_BF16, HB_PREC_FP32_CHECK, HB_RESET_FASTEST,
-                   HB_RESET_NONE, HB_STATIC, HogbatchError)
+                   HB_RESET_NONE, HB_STATIC, HB_UPDATE_ATOMIC, HB_UPDATE_HOGWILD, OPTIONS, HogbatchError)
 
 lib = _lib.load()
 
@@ -65,10 +65,24 @@ class MLP:
         _check(lib.mlp_num_params(self.h, C.byref(n)))
         return n.value
 
+    def set_option(self, name: str, value: int) -> None:
+        """``mlp_set_option``: a per-model setting (HB_OPT_*; names in ``OPTIONS``)."""
+        _check(lib.mlp_set_option(self.h, OPTIONS[name], int(value)))
+
+    def get_option(self, name: str) -> int:
+        v = C.c_int64()
+        _check(lib.mlp_get_option(self.h, OPTIONS[name], C.byref(v)))
+        return v.value
+
     def set_fused_min_batch(self, min_batch: int) -> None:
         """Steps of >= min_batch rows take the fused row-block kernel when eligible (0 = never).
         Call before creating workers."""
-        _check(lib.mlp_set_fused_min_batch(self.h, min_batch))
+        self.set_option("fused_min_batch", min_batch)
+
+    def merge_replicas(self, workers, gamma: float = 1.0) -> None:
+        """``hb_merge_replicas``: integrate the deep replicas among `workers` into this model."""
+        hs = (C.c_void_p * len(workers))(*[w.h.value for w in workers])
+        _check(lib.hb_merge_replicas(self.h, hs, len(workers), gamma))
 
     def fused_path(self, batch: int = 8192) -> int:
         """Cluster size (1, 2, 4 or 8) of the fused row-block step kernel at `batch` rows, 0 if
@@ -122,17 +136,27 @@ class MLP:
 class Worker:
     """A GPU worker (§V.A): activation scratch for max_batch rows and a stream."""
 
-    def __init__(self, model: MLP, max_batch: int, stream=None, sub_batches: int = 1):
-        """sub_batches = t > 1 creates a nested worker (Alg. 2's CPU worker, L224-L235)."""
+    def __init__(self, model: MLP, max_batch: int, stream=None, sub_batches: int = 1, replica: bool = False,
+                 device: int | None = None):
+        """sub_batches = t > 1 creates a nested worker (Alg. 2's CPU worker, L224-L235); replica=True
+        a deep-replica worker (private copy of the model, merged at sync points, L134/L141)."""
         self.model = model
         self.max_batch = max_batch
         self.sub_batches = sub_batches
+        self.replica = replica
         h = C.c_void_p()
         if sub_batches > 1:
             _check(lib.mlp_worker_create_nested(model.h, max_batch, sub_batches, _stream_ptr(stream), C.byref(h)))
         else:
-            _check(lib.mlp_worker_create(model.h, max_batch, 0, _stream_ptr(stream), C.byref(h)))
+            dev = model.device if device is None else device
+            _check(lib.mlp_worker_create(model.h, dev, max_batch, int(replica), _stream_ptr(stream), C.byref(h)))
         self.h = h
+
+    def params(self) -> np.ndarray:
+        """``mlp_worker_params``: this worker's parameters (its replica's for a deep replica)."""
+        out = np.empty(self.model.num_params, dtype=np.float32)
+        _check(lib.mlp_worker_params(self.h, out.ctypes.data_as(C.POINTER(C.c_float)), out.size))
+        return out
 
     @property
     def stream_handle(self) -> int:
@@ -200,6 +224,11 @@ class Policy:
     merges_per_epoch: int = 0
     merge_gamma: float = 1.0
     comm: "Comm | None" = None
+    update: int = -1              # -1: the models' HB_OPT_UPDATE; HB_UPDATE_HOGWILD / HB_UPDATE_ATOMIC
+    epoch_barrier: bool = True
+    check_labels: bool = False
+    coord: "Coord | None" = None  # shared cross-process coordinator
+    first_worker: int = 0         # with coord: global id of this process's first worker
 
     def to_c(self):
         ws = (_lib.WorkerPolicy * len(self.workers))(*[
@@ -207,7 +236,9 @@ class Policy:
         p = _lib.Policy(self.kind, self.alpha, self.eta0, self.b0, self.reset, self.credit,
                         int(self.deterministic), int(self.eval_loss), self.max_steps,
                         self.merges_per_epoch, self.merge_gamma,
-                        self.comm.h if self.comm is not None else None, len(self.workers), ws)
+                        self.comm.h if self.comm is not None else None, len(self.workers), ws,
+                        self.update, int(self.epoch_barrier), int(self.check_labels),
+                        self.coord.h if self.coord is not None else None, self.first_worker)
         return p, ws
 
 
@@ -227,10 +258,11 @@ def schedule_trace(policy: Policy, N: int, epochs: int, cap: int = 1 << 20):
 
 def hogbatch_run(workers, policy: Policy, X, y, epochs: int = 1, n: int | None = None,
                  trace_cap: int = 0, step_loss_cap: int = 0, max_epochs: int | None = None):
-    """``hogbatch_run(workers, policy, epochs)`` over device data (X [N x ldx], y [N])."""
+    """``hogbatch_run(workers, policy, epochs)`` over device data (X [N x ldx], y [N]).  Per-worker
+    statistics are indexed by the global worker id (policy.workers)."""
     n = X.shape[0] if n is None else n
     p, _keep = policy.to_c()
-    W = len(workers)
+    W = len(policy.workers)
     me = max_epochs or epochs
     el = (C.c_double * me)()
     et = (C.c_double * me)()
@@ -240,8 +272,8 @@ def hogbatch_run(workers, policy: Policy, X, y, epochs: int = 1, n: int | None =
     sl = (C.c_float * max(step_loss_cap, 1))()
     st = _lib.Stats(me, 0, el, et, up, sm, tr, trace_cap, 0, sl, step_loss_cap, 0, 0.0, 0, 0)
     ds = _lib.Dataset(X.data_ptr(), X.stride(0), _xdtype(X), y.data_ptr(), n)
-    hs = (C.c_void_p * W)(*[w.h.value for w in workers])
-    _check(lib.hogbatch_run(hs, W, C.byref(p), C.byref(ds), epochs, C.byref(st)))
+    hs = (C.c_void_p * len(workers))(*[w.h.value for w in workers])
+    _check(lib.hogbatch_run(hs, len(workers), C.byref(p), C.byref(ds), epochs, C.byref(st)))
     ed = st.epochs_done
     return dict(
         epochs_done=ed,
@@ -257,6 +289,44 @@ def hogbatch_run(workers, policy: Policy, X, y, epochs: int = 1, n: int | None =
         total_samples=st.total_samples,
         n_merges=st.n_merges,
     )
+
+
+class Coord:
+    """``hb_coord_create``: the node's shared coordinator (POSIX shared memory `name`); rank 0
+    creates it, the other ranks attach.  Pass as Policy.coord with Policy.first_worker."""
+
+    def __init__(self, name: str, policy: Policy, N: int, nranks: int, rank: int):
+        p, _keep = policy.to_c()
+        h = C.c_void_p()
+        _check(lib.hb_coord_create(name.encode(), C.byref(p), N, nranks, rank, C.byref(h)))
+        self.h = h
+
+    def reset(self, policy: Policy, N: int):
+        p, _keep = policy.to_c()
+        _check(lib.hb_coord_reset(self.h, C.byref(p), N))
+
+    def schedule(self, worker: int, now: float):
+        """One ScheduleWork(worker) on the shared state (test / custom-driver entry)."""
+        r = _lib.TraceRec()
+        _check(lib.hb_coord_schedule(self.h, worker, now, C.byref(r)))
+        return _rec_tuple(r)
+
+    def idle(self, worker: int) -> bool:
+        """The worker could not be served; True if every worker now idles (the epoch ended)."""
+        e = C.c_int32()
+        _check(lib.hb_coord_idle(self.h, worker, C.byref(e)))
+        return bool(e.value)
+
+    def close(self):
+        if getattr(self, "h", None):
+            lib.hb_coord_destroy(self.h)
+            self.h = None
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
 
 
 class Comm:

@@ -18,16 +18,23 @@ HB_BF16, HB_F32 = 0, 1
 HB_MINIBATCH, HB_HOGBATCH, HB_STATIC, HB_ADAPTIVE = 0, 1, 2, 3
 HB_RESET_FASTEST, HB_RESET_NONE = 0, 1
 HB_CREDIT_DISPATCH, HB_CREDIT_COMPLETION = 0, 1
+HB_UPDATE_HOGWILD, HB_UPDATE_ATOMIC = 0, 1
+# mlp_set_option keys
+OPTIONS = {"fused_min_batch": 0, "rowchain": 1, "rc_cluster": 2, "bwd_overlap": 3, "head_fuse": 4, "dw_pair": 5,
+           "pdl": 6, "graphs": 7, "inflight": 8, "stage_rows": 9, "update": 10}
 ACTIONS = ("none", "halve", "double", "clamp_lo", "clamp_hi")
 
 # every symbol include/hogbatch.h declares (checked by tests/test_abi.py)
 EXPORTS = ("hb_last_error", "hb_abi_version", "hb_device_ok", "mlp_create", "mlp_destroy",
-           "mlp_num_params", "mlp_fused_path", "mlp_set_fused_min_batch", "mlp_get_params", "mlp_set_params", "mlp_worker_create",
-           "mlp_worker_destroy", "mlp_worker_stream", "mlp_step", "mlp_step_grads", "mlp_loss",
-           "hb_schedule_trace", "hogbatch_run", "hb_nccl_unique_id", "hb_comm_create",
-           "hb_comm_destroy", "hb_merge_begin", "hb_merge", "hb_kernel_launches", "hb_prof_enable",
-           "hb_prof_read", "hb_bench_gemm", "hb_bench_gemm_phases", "hb_rc_trace", "hb_bench_step", "hb_merge_schedule",
-           "mlp_worker_create_nested", "mlp_row_losses")
+           "mlp_num_params", "mlp_fused_path", "mlp_set_option", "mlp_get_option", "mlp_get_params",
+           "mlp_set_params", "mlp_worker_create", "mlp_worker_params", "mlp_worker_destroy", "mlp_worker_stream",
+           "mlp_step", "mlp_step_grads", "mlp_row_losses", "mlp_loss", "hb_schedule_trace", "hogbatch_run",
+           "hb_nccl_unique_id", "hb_comm_create", "hb_comm_destroy", "hb_merge_begin", "hb_merge",
+           "hb_merge_replicas", "hb_kernel_launches", "hb_prof_enable", "hb_prof_read", "hb_merge_schedule",
+           "mlp_worker_create_nested", "hb_coord_create", "hb_coord_destroy", "hb_coord_reset",
+           "hb_coord_schedule", "hb_coord_idle")
+# tuning build only (include/hogbatch_tuning.h): not exported by the product library
+TUNING_EXPORTS = ("hb_bench_gemm", "hb_bench_gemm_phases", "hb_rc_trace", "hb_bench_step")
 PROF_LAYERS = 16
 PROF_CLASSES = ("fwd_gemm", "head_gemm", "softmax_xent", "dgrad_gemm", "wgrad_sgd_gemm", "bias_sgd", "other",
                 "rowchain")
@@ -43,7 +50,8 @@ class Policy(C.Structure):
                 ("reset", C.c_int32), ("credit", C.c_int32), ("deterministic", C.c_int32),
                 ("eval_loss", C.c_int32), ("max_steps", C.c_int64), ("merges_per_epoch", C.c_int32),
                 ("merge_gamma", C.c_float), ("comm", C.c_void_p), ("n_workers", C.c_int32),
-                ("workers", C.POINTER(WorkerPolicy))]
+                ("workers", C.POINTER(WorkerPolicy)), ("update", C.c_int32), ("epoch_barrier", C.c_int32),
+                ("check_labels", C.c_int32), ("coord", C.c_void_p), ("first_worker", C.c_int32)]
 
 
 class Dataset(C.Structure):
@@ -87,10 +95,12 @@ def load():
         "mlp_destroy": ([VP], C.c_int),
         "mlp_num_params": ([VP, P(I64)], C.c_int),
         "mlp_fused_path": ([VP, I32, P(I32)], C.c_int),
-        "mlp_set_fused_min_batch": ([VP, I32], C.c_int),
+        "mlp_set_option": ([VP, I32, I64], C.c_int),
+        "mlp_get_option": ([VP, I32, P(I64)], C.c_int),
         "mlp_get_params": ([VP, P(F), I64], C.c_int),
         "mlp_set_params": ([VP, P(F), I64], C.c_int),
-        "mlp_worker_create": ([VP, I32, I32, VP, P(VP)], C.c_int),
+        "mlp_worker_create": ([VP, I32, I32, I32, VP, P(VP)], C.c_int),
+        "mlp_worker_params": ([VP, P(F), I64], C.c_int),
         "mlp_worker_destroy": ([VP], C.c_int),
         "mlp_worker_create_nested": ([VP, I32, I32, VP, P(VP)], C.c_int),
         "mlp_worker_stream": ([VP], VP),
@@ -105,6 +115,12 @@ def load():
         "hb_comm_destroy": ([VP], C.c_int),
         "hb_merge_begin": ([VP], C.c_int),
         "hb_merge": ([VP, VP, F, VP], C.c_int),
+        "hb_merge_replicas": ([VP, P(VP), I32, F], C.c_int),
+        "hb_coord_create": ([C.c_char_p, P(Policy), I64, I32, I32, P(VP)], C.c_int),
+        "hb_coord_destroy": ([VP], C.c_int),
+        "hb_coord_reset": ([VP, P(Policy), I64], C.c_int),
+        "hb_coord_schedule": ([VP, I32, D, P(TraceRec)], C.c_int),
+        "hb_coord_idle": ([VP, I32, P(I32)], C.c_int),
         "hb_kernel_launches": ([], I64),
         "hb_prof_enable": ([I32], C.c_int),
         "hb_rc_trace": ([VP, I64], C.c_int),
@@ -115,8 +131,8 @@ def load():
         "hb_merge_schedule": ([I64, I32, P(I32), I64, P(I32), P(I32)], C.c_int),
     }
     for name, (args, res) in sig.items():
-        if os.environ.get("HB_LIB") and not hasattr(lib, name):
-            continue  # A/B builds of older sources may lack newer entry points
+        if (os.environ.get("HB_LIB") or name in TUNING_EXPORTS) and not hasattr(lib, name):
+            continue  # tuning entry points exist only in the tuning build; A/B builds may lack new ones
         fn = getattr(lib, name)
         fn.argtypes = args
         fn.restype = res

@@ -90,4 +90,28 @@ int hb_merge(hb_model* m, hb_comm* c, float gamma, void* cuda_stream) {
   return HB_OK;
 }
 
+int hb_merge_replicas(hb_model* m, hb_worker* const* workers, int32_t n, float gamma) {
+  HB_CHECK_ARG(m && (workers || n == 0) && n >= 0, "bad arguments");
+  if (!m->base) return fail(HB_ESTATE, "hb_merge_begin was not called");
+  ReplicaPtrs r{};
+  int nr = 0;
+  for (int i = 0; i < n; ++i) {
+    hb_worker* w = workers[i];
+    HB_CHECK_ARG(w && w->global == m, "every worker must belong to this model");
+    if (w->m == m) continue;  // reference replica: its updates are already in the global model
+    HB_CHECK_ARG(nr < 8, "at most 8 deep replicas per merge");
+    r.w[nr] = w->m->master;
+    r.sh[nr] = w->m->shadow;
+    ++nr;
+  }
+  HB_CUDA_TRY(cudaSetDevice(m->device));
+  HB_CUDA_TRY(cudaDeviceSynchronize());  // every worker's updates of its replica have landed
+  Prof pr(HB_PROF_OTHER, m->stream);
+  merge_replicas_kernel<<<592, 256, 0, m->stream>>>(m->master, m->base, m->shadow, r, nr, gamma, (int64_t)m->total);
+  HB_CUDA_TRY(cudaGetLastError());
+  pr.done(1, 0.0, 4.0 * (double)m->total * (4.0 + 2.0 * nr) + 2.0 * (double)m->total * (1 + nr));
+  HB_CUDA_TRY(cudaStreamSynchronize(m->stream));
+  return HB_OK;
+}
+
 }  // extern "C"

@@ -309,6 +309,19 @@ __device__ __forceinline__ void umma_commit_multicast(uint64_t* bar, uint16_t ct
       : "memory");
 }
 
+// Tuning builds (-DHB_TUNING, build.py --variant tuning HB_TUNING) record per-CTA phase timestamps
+// into a caller-armed buffer; product builds compile every stamp away.
+#ifdef HB_TUNING
+#define HB_STAMP(cond, slot) \
+  do {                        \
+    if (cond) (slot) = gtimer(); \
+  } while (0)
+#else
+#define HB_STAMP(cond, slot) \
+  do {                        \
+  } while (0)
+#endif
+
 __device__ __forceinline__ unsigned long long gtimer() {
   unsigned long long t;
   asm volatile("mov.u64 %0, %globaltimer;" : "=l"(t));

@@ -47,6 +47,8 @@ struct EpiArgs {
   unsigned long long* dbg;  // tuning only: per-CTA phase timestamps (globaltimer ns), nullable
   int force_bn, force_splits;  // host-side launch choices for dW GEMMs (0 = heuristic)
   int pair;                    // host-side: dW GEMM on CTA pairs (tcgen05 cta_group::2) when eligible
+  int no_pdl;                  // host-side: launch without programmatic dependent launch
+  int atomic;                  // WGRAD_SGD: W -= lr * dW with atomic adds (HB_UPDATE_ATOMIC)
   // softmax cross-entropy head fused into the output-layer GEMM (C <= 16):
   const int32_t* y;     // labels (dataset base when yoff != nullptr)
   const int* yoff;      // device row offset of the batch (graph replay), nullable
@@ -101,13 +103,32 @@ __device__ __forceinline__ void epi_elem(const EpiArgs& ep, int r, int n, float 
     static_cast<TAct*>(ep.out0)[(int64_t)r * ep.ld0 + n] = to_act<TAct>(v * s);
   } else if (EPI == EPI_WGRAD_SGD) {
     int64_t idx = ep.transposed ? (int64_t)n * ep.ldw + r : (int64_t)r * ep.ldw + n;
-    float w = ep.master[idx] - ep.lr * v;
-    ep.master[idx] = w;
+    float w;
+    if (ep.atomic) {  // HB_UPDATE_ATOMIC: concurrent workers' updates of this weight all survive
+      const float d = __fmul_rn(-ep.lr, v);
+      w = atomicAdd(ep.master + idx, d) + d;
+    } else {          // Hogwild read-modify-write [L128, L170] (same rounding: no fused multiply-add)
+      w = ep.master[idx] + __fmul_rn(-ep.lr, v);
+      ep.master[idx] = w;
+    }
     if (ep.shadow) ep.shadow[idx] = __float2bfloat16_rn(w);
   } else {  // EPI_WGRAD_STORE
     int64_t idx = ep.transposed ? (int64_t)n * ep.ldw + r : (int64_t)r * ep.ldw + n;
     static_cast<float*>(ep.out0)[idx] = v;
   }
+}
+
+// -lr * g for 4 weights, rounded once per product (no fused multiply-add): the Hogwild and the
+// atomic update then produce the same bits for the same accumulator values
+__device__ __forceinline__ float4 sgd_delta4(float lr, float a, float b, float c, float d) {
+  return make_float4(__fmul_rn(-lr, a), __fmul_rn(-lr, b), __fmul_rn(-lr, c), __fmul_rn(-lr, d));
+}
+
+// HB_UPDATE_ATOMIC: W += d with one 16-byte atomic (sm_90+ float4 atomicAdd on global memory);
+// returns the new value as seen by this update (old + d) for the bf16 shadow
+__device__ __forceinline__ float4 sgd_atomic4(float4* W, float4 d) {
+  const float4 old = atomicAdd(W, d);
+  return make_float4(old.x + d.x, old.y + d.y, old.z + d.z, old.w + d.w);
 }
 
 // 16 fp32 values -> packed bf16 hi = bf16(v) and lo = bf16(v - hi) (R24: v = hi + lo to ~2^-17 |v|)
@@ -173,12 +194,18 @@ __device__ __forceinline__ void epi_row16_bf16(const EpiArgs& ep, int r, int n0,
     uint32_t sp[8];
 #pragma unroll
     for (int q = 0; q < 4; ++q) {
-      float4 w = W[q];
-      w.x -= ep.lr * v[4 * q];
-      w.y -= ep.lr * v[4 * q + 1];
-      w.z -= ep.lr * v[4 * q + 2];
-      w.w -= ep.lr * v[4 * q + 3];
-      W[q] = w;
+      float4 w;
+      if (ep.atomic) {
+        w = sgd_atomic4(W + q, sgd_delta4(ep.lr, v[4 * q], v[4 * q + 1], v[4 * q + 2], v[4 * q + 3]));
+      } else {
+        w = W[q];
+        const float4 d = sgd_delta4(ep.lr, v[4 * q], v[4 * q + 1], v[4 * q + 2], v[4 * q + 3]);
+        w.x += d.x;
+        w.y += d.y;
+        w.z += d.z;
+        w.w += d.w;
+        W[q] = w;
+      }
       sp[2 * q] = pack_bf16x2(w.x, w.y);
       sp[2 * q + 1] = pack_bf16x2(w.z, w.w);
     }

@@ -169,4 +169,38 @@ static __global__ void merge_apply_kernel(float* w, float* base, const float* __
   }
 }
 
+// HB_CHECK=labels (hb_policy.check_labels): flag any label outside [0, C)
+static __global__ void check_labels_kernel(const int32_t* __restrict__ y, int64_t n, int C, int* bad) {
+  int any = 0;
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x)
+    any |= (y[i] < 0) | (y[i] >= C);
+  if (__syncthreads_or(any) && threadIdx.x == 0) atomicOr(bad, 1);
+}
+
+// Local replica merge (hb_merge_replicas, PAPER.md L141 / L175): with G the global model, B the
+// merge base (G at the previous sync point) and R_0..R_{n-1} the deep replicas of this process,
+//   G <- G + gamma * sum_E (R_E - B)   (fixed E order)   then B, R_E <- G and every bf16 shadow
+// is rewritten — one pass over the parameters (each replica read once and written once).
+struct ReplicaPtrs {
+  float* w[8];
+  __nv_bfloat16* sh[8];
+};
+static __global__ void merge_replicas_kernel(float* g, float* base, __nv_bfloat16* g_shadow, ReplicaPtrs r, int n_rep,
+                                             float gamma, int64_t n) {
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) {
+    const float b0 = base[i];
+    float d = 0.f;
+    for (int e = 0; e < n_rep; ++e) d += r.w[e][i] - b0;
+    const float v = g[i] + gamma * d;
+    g[i] = v;
+    base[i] = v;
+    const __nv_bfloat16 h = __float2bfloat16_rn(v);
+    if (g_shadow) g_shadow[i] = h;
+    for (int e = 0; e < n_rep; ++e) {
+      r.w[e][i] = v;
+      if (r.sh[e]) r.sh[e][i] = h;
+    }
+  }
+}
+
 }  // namespace hb

@@ -175,8 +175,7 @@ static int launch_tc(const CUtensorMap& ma, const CUtensorMap& mb, int M, int N,
   cfg.stream = s;
   cudaLaunchAttribute attr[2];
   int na = 0;
-  static const bool pdl = !(getenv("HB_NO_PDL") && getenv("HB_NO_PDL")[0] == '1');
-  if (pdl) {  // programmatic dependent launch: prologue overlaps the previous kernel's tail
+  if (!ep.no_pdl) {  // programmatic dependent launch: prologue overlaps the previous kernel's tail
     attr[na].id = cudaLaunchAttributeProgrammaticStreamSerialization;
     attr[na].val.programmaticStreamSerializationAllowed = 1;
     ++na;
@@ -211,13 +210,20 @@ static int launch_tc_bn(int bn, const CUtensorMap& ma, const CUtensorMap& mb, in
 // <= 8 (portable cluster size), at least one k-block per split
 static int choose_bn_base(int M, int N);
 
+// Launch-choice overrides from the environment exist only in the tuning build (-DHB_TUNING);
+// the product library uses the measured defaults and the per-model options (mlp_set_option).
+#ifdef HB_TUNING
 static int env_int(const char* name, int dflt) {
   const char* v = getenv(name);
   return v && *v ? atoi(v) : dflt;
 }
+#define HB_TUNE(name, dflt) env_int(name, dflt)
+#else
+#define HB_TUNE(name, dflt) (dflt)
+#endif
 
 int choose_splits(int M, int N, int K, int bn) {
-  static const int max_s = env_int("HB_MAX_SPLITS", 4);  // 8-CTA clusters of 200 KB CTAs do not all co-reside
+  static const int max_s = HB_TUNE("HB_MAX_SPLITS", 4);  // 8-CTA clusters of 200 KB CTAs do not all co-reside
   const long tiles = (long)((M + TC_BM - 1) / TC_BM) * ((N + bn - 1) / bn);
   const int nkb = (K + TC_BK - 1) / TC_BK;
   int S = 1;
@@ -228,7 +234,7 @@ int choose_splits(int M, int N, int K, int bn) {
 
 // tile width of a dW GEMM: narrow enough that tiles x splits fill the SMs
 static int choose_bn_wgrad(int M, int N, int K) {
-  static const int forced = env_int("HB_WGRAD_BN", 0);
+  static const int forced = HB_TUNE("HB_WGRAD_BN", 0);
   if (forced) return forced;
   if (K < 2048) return choose_bn(M, N, K);  // short K: no split-K, spread tiles over the SMs
   int bn = choose_bn_base(M, N);          // long K: split-K supplies the parallelism
@@ -249,7 +255,7 @@ static int choose_bn_base(int M, int N) {
 // Tile width: the base rule, narrowed while the grid would leave most SMs idle (small batches:
 // M = b <= a few hundred rows gives 1-2 row tiles; narrower tiles spread the epilogue)
 int choose_bn(int M, int N, int K) {
-  static const int forced = env_int("HB_FWD_BN", 0);  // tuning only: forward / dX tile width
+  static const int forced = HB_TUNE("HB_FWD_BN", 0);  // tuning only: forward / dX tile width
   if (forced && N > 16) return forced;
   int bn = choose_bn_base(M, N);
   const long mt = (M + TC_BM - 1) / TC_BM;
@@ -387,9 +393,14 @@ struct RcCfg {
   int CS = 1, NH = 64, NCA = 1, NS = 2, tmem = 128, smem = 0, s_tma = 0;
 };
 
+#ifdef HB_TUNING
 static unsigned long long* g_rc_trace = nullptr;  // tuning only: hb_rc_trace
 static int g_bench_part = 0;                      // tuning only: hb_bench_step part
 static int64_t g_rc_trace_cap = 0;
+#else
+static constexpr unsigned long long* g_rc_trace = nullptr;
+static constexpr int g_bench_part = 0;
+#endif
 static constexpr int RC_SMEM_CAP = 232448;  // 227 KB opt-in dynamic shared memory per CTA
 
 // n_0 - n x (L-1) - C with uniform hidden width n <= 512, n_0 <= 512, C <= 16, 2 <= L <= 12
@@ -398,8 +409,7 @@ static constexpr int RC_SMEM_CAP = 232448;  // 227 KB opt-in dynamic shared memo
 // (every doubling halves the W bytes each SM streams per layer); HB_RC_CS forces it.
 static RcCfg rowchain_cfg(const hb_model* m, int b = 8192) {
   RcCfg c;
-  static const int on = env_int("HB_ROWCHAIN", 1);
-  if (!on || m->prec != HB_PREC_BF16) return c;
+  if (!m->opt_rowchain || m->prec != HB_PREC_BF16) return c;
   const int L = (int)m->layers.size();
   if (L < 2 || L > RC_MAX_L) return c;
   const int n0 = m->dims[0], n = m->dims[1], C = m->dims[L];
@@ -409,7 +419,7 @@ static RcCfg rowchain_cfg(const hb_model* m, int b = 8192) {
   // measured on B200 (scripts/rc_probe.py, C2 shape): the fused chain is latency-bound at
   // ~65-90 us whatever the batch, the per-layer chain is cheaper below b = 8192
   if (m->rc_min_b <= 0 || b < m->rc_min_b) return c;
-  static const int cs_env = env_int("HB_RC_CS", 0);
+  const int cs_env = m->opt_rc_cluster;
   static int nsm = 0;
   if (!nsm) {
     int dev = 0;
@@ -437,11 +447,11 @@ static RcCfg rowchain_cfg(const hb_model* m, int b = 8192) {
   // sigma' staging for TMA stores (2 chunk buffers) when the W ring keeps >= 2 stages: the
   // per-thread-row global stores it replaces cost ~0.45 us per chunk (B200, C2 b = 8192) and a
   // 2-stage ring measured as fast as 3 (scripts/gpu_refresh.sh)
-  static const int s_tma_env = env_int("HB_RC_S_TMA", 1);
+  static const int s_tma_env = HB_TUNE("HB_RC_S_TMA", 1);
   c.s_tma = s_tma_env && (RC_SMEM_CAP - (1024 + c.NCA * RC_CHUNK + 2 * RC_CHUNK + 1024 + 8 * (2 * 2 + c.NCA + 8) + 16)) /
                              (c.NH * 128) >= 2;
   const int fixed = 1024 + c.NCA * RC_CHUNK + (c.s_tma ? 2 * RC_CHUNK : 0) + 1024 + 8 * (2 * RC_MAX_STAGES + c.NCA + 8) + 16;
-  static const int ns_env = env_int("HB_RC_NS", 0);  // tuning only: force the W ring depth
+  static const int ns_env = HB_TUNE("HB_RC_NS", 0);  // tuning only: force the W ring depth
   c.NS = std::min(RC_MAX_STAGES, (RC_SMEM_CAP - fixed) / stb);
   if (ns_env >= 2 && ns_env < c.NS) c.NS = ns_env;
   if (c.NS < 2) return c;
@@ -492,7 +502,7 @@ static int launch_rowchain(hb_worker* w, const RcCfg& c, const void* X, int64_t 
   P.nstages = c.NS;
   P.abuf_chunks = c.NCA;
   P.tmem_cols = c.tmem;
-  static const int korder = env_int("HB_RC_KORDER", 0);  // 1 measured slower (B200, C2 b = 8192: 103 vs 88 us)
+  static const int korder = HB_TUNE("HB_RC_KORDER", 0);  // 1 measured slower (B200, C2 b = 8192: 103 vs 88 us)
   P.korder = korder;
   P.s_tma = c.s_tma;
   P.inv_b = 1.0f / (float)b;
@@ -514,9 +524,11 @@ static int launch_rowchain(hb_worker* w, const RcCfg& c, const void* X, int64_t 
   cfg.stream = s;
   cudaLaunchAttribute attr[2];
   int na = 0;
-  attr[na].id = cudaLaunchAttributeProgrammaticStreamSerialization;
-  attr[na].val.programmaticStreamSerializationAllowed = 1;
-  ++na;
+  if (m->opt_pdl) {
+    attr[na].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+    attr[na].val.programmaticStreamSerializationAllowed = 1;
+    ++na;
+  }
   if (c.CS > 1) {
     attr[na].id = cudaLaunchAttributeClusterDimension;
     attr[na].val.clusterDim.x = c.CS;
@@ -600,6 +612,7 @@ static void free_worker_buffers(hb_worker* w) {
 static int alloc_worker(hb_model* m, int max_b, cudaStream_t stream, bool own, hb_worker** out, bool train = true) {
   hb_worker* w = new hb_worker();
   w->m = m;
+  w->global = m;
   w->max_b = max_b;
   w->stream = stream;
   w->own_stream = own;
@@ -702,6 +715,7 @@ static int run_step_simt(hb_worker* w, const void* X, int64_t ldx, int32_t xdt, 
   for (int l = 0; l < L; ++l) {
     const Layer& Ly = m->layers[l];
     EpiArgs ep{};
+    ep.no_pdl = !m->opt_pdl;
     ep.M = b;
     ep.N = Ly.n_out;
     ep.bias = m->master + Ly.b_off;
@@ -744,6 +758,7 @@ static int run_step_simt(hb_worker* w, const void* X, int64_t ldx, int32_t xdt, 
     if (l > 0) {
       const Layer& Lp = m->layers[l - 1];
       EpiArgs ep{};
+    ep.no_pdl = !m->opt_pdl;
       ep.M = b;
       ep.N = Ly.n_in;
       ep.out0 = w->dZ[l - 1];
@@ -756,6 +771,7 @@ static int run_step_simt(hb_worker* w, const void* X, int64_t ldx, int32_t xdt, 
     }
     {
       EpiArgs ep{};
+    ep.no_pdl = !m->opt_pdl;
       const int epi = grads_only ? EPI_WGRAD_STORE : EPI_WGRAD_SGD;
       ep.master = m->master + Ly.w_off;
       ep.ldw = Ly.ldw;
@@ -793,8 +809,7 @@ static int run_step_simt(hb_worker* w, const void* X, int64_t ldx, int32_t xdt, 
 // Off by default: measured slower on B200 at b = 8192 (37.5 M vs 42.5 M samples/s on C2) because
 // the head grid has only b/128 CTAs while the separate dX GEMM fills all 148 SMs.
 static bool head_dx_fused(const hb_model* m) {
-  static const bool on = env_int("HB_HEAD_FUSE", 0) != 0;
-  return on && m->layers.size() >= 2 && m->layers.back().n_out <= 16;
+  return m->opt_head_fuse && m->layers.size() >= 2 && m->layers.back().n_out <= 16;
 }
 
 // Forward chain (Eq. (1)) of the bf16 tensor-core path.  X holds x_rows rows; the batch starts
@@ -811,6 +826,7 @@ static int forward_tc(hb_worker* w, const void* X, int64_t ldx, int64_t x_rows, 
     ProfLayer pl(l);
     TcOp B{m->shadow + Ly.w_off, Ly.ldw, 0, nullptr};
     EpiArgs ep{};
+    ep.no_pdl = !m->opt_pdl;
     ep.M = b;
     ep.N = Ly.n_out;
     ep.bias = m->master + Ly.b_off;
@@ -880,6 +896,7 @@ static int launch_wgrad(hb_worker* w, int l, const void* X, int64_t ldx, int64_t
   TcOp dZl{w->dZ[l], ld_dz(w, l), b, nullptr};
   TcOp Al = l == 0 ? TcOp{X, ldx, x_rows, d_off} : TcOp{w->H[l - 1], m->layers[l - 1].ldo, b, nullptr};
   EpiArgs ep{};
+    ep.no_pdl = !m->opt_pdl;
   const int epi = grads_only ? EPI_WGRAD_STORE : EPI_WGRAD_SGD;
   ep.master = m->master + Ly.w_off;
   ep.shadow = m->shadow + Ly.w_off;
@@ -891,8 +908,9 @@ static int launch_wgrad(hb_worker* w, int l, const void* X, int64_t ldx, int64_t
   ep.n_mtiles = part_rows;
   ep.force_bn = force_bn;
   ep.force_splits = force_splits;
-  static const int pair = env_int("HB_DW_PAIR", 0);
-  ep.pair = pair;
+  ep.pair = m->opt_dw_pair;
+  ep.no_pdl = !m->opt_pdl;
+  ep.atomic = m->opt_update == HB_UPDATE_ATOMIC;
   ep.bias_upd = m->master + Ly.b_off;
   ep.bias_grad = grads_only ? w->grads + Ly.b_off : nullptr;
   ep.ws = ws;
@@ -930,7 +948,7 @@ static int run_step_rowchain(hb_worker* w, const RcCfg& c, const void* X, int64_
     pr.done(1, fl, by);
   }
   if (g_bench_part == 1) return HB_OK;
-  static const bool conc = env_int("HB_RC_DW_SERIAL", 0) == 0;
+  static const bool conc = HB_TUNE("HB_RC_DW_SERIAL", 0) == 0;
   if (!conc) {
     for (int l = L - 1; l >= 0; --l) {
       int rc = launch_wgrad(w, l, X, ldx, x_rows, d_off, b, lr, grads_only, s, w->ws_l[l], 4 * ((b + 127) / 128));
@@ -941,7 +959,7 @@ static int run_step_rowchain(hb_worker* w, const RcCfg& c, const void* X, int64_
   HB_CUDA_TRY(cudaEventRecord(w->ev_chain, s));
   for (int l = L - 1; l >= 0; --l) {
     HB_CUDA_TRY(cudaStreamWaitEvent(w->sdw[l], w->ev_chain, 0));
-    static const int fbn = env_int("HB_RC_WGRAD_BN", 0), fs = env_int("HB_RC_WGRAD_S", 0);
+    static const int fbn = HB_TUNE("HB_RC_WGRAD_BN", 0), fs = HB_TUNE("HB_RC_WGRAD_S", 0);
     const Layer& Ly = m->layers[l];
     const bool wide = Ly.n_out >= 128 || Ly.n_out >= Ly.n_in;  // not the transposed small head
     // the L GEMMs share the SMs, so each takes wide tiles (fewer L2 re-reads of dZ / H) and a
@@ -977,8 +995,7 @@ static int run_step_tc(hb_worker* w, const void* X, int64_t ldx, int64_t x_rows,
   if (rc) return rc;
   // dW_l only has to follow dX_l (the last reader of W_l): it runs on the worker's second stream,
   // overlapping dX_{l-1} (HB_NO_BWD_OVERLAP=1 keeps everything on one stream)
-  static const bool overlap = env_int("HB_NO_BWD_OVERLAP", 0) == 0;
-  cudaStream_t s2 = overlap && w->s2 ? w->s2 : s;
+  cudaStream_t s2 = m->opt_bwd_overlap && w->s2 ? w->s2 : s;
   for (int l = L - 1; l >= 0; --l) {
     const Layer& Ly = m->layers[l];
     TcOp dZl{w->dZ[l], ld_dz(w, l), b, nullptr};
@@ -986,6 +1003,7 @@ static int run_step_tc(hb_worker* w, const void* X, int64_t ldx, int64_t x_rows,
     if (l > 0 && !(l == L - 1 && head_dx_fused(m))) {  // dZ_{l-1} = (dZ_l W_l) * sigma'(Z_{l-1}) + bias partials
       const Layer& Lp = m->layers[l - 1];
       EpiArgs ep{};
+    ep.no_pdl = !m->opt_pdl;
       ep.M = b;
       ep.N = Ly.n_in;
       ep.out0 = w->dZ[l - 1];
@@ -1217,8 +1235,8 @@ int mlp_create(const int32_t* dims, int32_t n_dims, int32_t activation, int32_t 
   m->device = device;
   m->prec = precision;
   m->dims.assign(dims, dims + n_dims);
-  // fused row-block path from this batch size up (measured crossover on B200)
-  m->rc_min_b = env_int("HB_RC_MIN_B", 4096);  // B200, C2: fused 104.5 vs 109.1 us at 4096, 173 vs 88 at 2048
+  // fused row-block path from this batch size up (measured crossover on B200, DESIGN.md §5:
+  // C2 fused 104.5 vs 109.1 us at 4096, 173 vs 88 at 2048); other options: model.h defaults
   size_t off = 0;
   for (int l = 1; l < n_dims; ++l) {
     Layer Ly;
@@ -1291,6 +1309,53 @@ int mlp_destroy(hb_model* m) {
   return HB_OK;
 }
 
+}  // extern "C"
+
+namespace hb {
+int check_labels_dev(const int32_t* y, int64_t n, int C, int device, bool* ok) {
+  HB_CUDA_TRY(cudaSetDevice(device));
+  int* d = nullptr;
+  HB_CUDA_TRY(cudaMalloc(&d, sizeof(int)));
+  int h = 0;
+  cudaMemset(d, 0, sizeof(int));
+  check_labels_kernel<<<592, 256>>>(y, n, C, d);
+  cudaError_t e = cudaMemcpy(&h, d, sizeof(int), cudaMemcpyDeviceToHost);
+  cudaFree(d);
+  if (e != cudaSuccess) return fail(HB_ECUDA, std::string("label check: ") + cudaGetErrorString(e));
+  *ok = h == 0;
+  return HB_OK;
+}
+
+// A deep replica of m (same shape, options and device): private fp32 master + bf16 shadow holding
+// a copy of m's current parameters.
+int clone_model(hb_model* m, hb_model** out) {
+  hb_model* r = nullptr;
+  int rc = mlp_create(m->dims.data(), (int32_t)m->dims.size(), HB_SIGMOID, m->prec, 0, m->device, &r);
+  if (rc) return rc;
+  r->rc_min_b = m->rc_min_b;
+  r->opt_rowchain = m->opt_rowchain;
+  r->opt_rc_cluster = m->opt_rc_cluster;
+  r->opt_bwd_overlap = m->opt_bwd_overlap;
+  r->opt_head_fuse = m->opt_head_fuse;
+  r->opt_dw_pair = m->opt_dw_pair;
+  r->opt_pdl = m->opt_pdl;
+  r->opt_graphs = m->opt_graphs;
+  r->opt_inflight = m->opt_inflight;
+  r->opt_stage_rows = m->opt_stage_rows;
+  r->opt_update = m->opt_update;
+  if (cudaDeviceSynchronize() != cudaSuccess ||
+      cudaMemcpy(r->master, m->master, m->total * 4, cudaMemcpyDeviceToDevice) != cudaSuccess ||
+      (m->shadow && cudaMemcpy(r->shadow, m->shadow, m->total * 2, cudaMemcpyDeviceToDevice) != cudaSuccess)) {
+    mlp_destroy(r);
+    return fail(HB_ECUDA, "replica copy");
+  }
+  *out = r;
+  return HB_OK;
+}
+}  // namespace hb
+
+extern "C" {
+
 int mlp_num_params(const hb_model* m, int64_t* n_out) {
   HB_CHECK_ARG(m && n_out, "null arg");
   int64_t n = 0;
@@ -1299,6 +1364,7 @@ int mlp_num_params(const hb_model* m, int64_t* n_out) {
   return HB_OK;
 }
 
+#ifdef HB_TUNING
 // Tuning only: cap > 0 arms per-step phase stamps in every later rowchain launch (the buffer is
 // overwritten by each launch); cap == 0 copies the last launch's stamps to host and disarms.
 int hb_rc_trace(unsigned long long* host, int64_t cap) {
@@ -1364,10 +1430,62 @@ int hb_bench_step(hb_worker* w, const void* X, int64_t ldx, const int32_t* y, in
   return HB_OK;
 }
 
-int mlp_set_fused_min_batch(hb_model* m, int32_t min_batch) {
-  HB_CHECK_ARG(m && min_batch >= 0, "bad args");
-  m->rc_min_b = min_batch;
-  return HB_OK;
+#endif  // HB_TUNING
+
+int mlp_set_option(hb_model* m, int32_t key, int64_t v) {
+  HB_CHECK_ARG(m, "null model");
+  auto flag = [&](int* dst) -> int {
+    HB_CHECK_ARG(v == 0 || v == 1, "option value must be 0 or 1");
+    *dst = (int)v;
+    return HB_OK;
+  };
+  switch (key) {
+    case HB_OPT_FUSED_MIN_BATCH:
+      HB_CHECK_ARG(v >= 0 && v <= (1 << 30), "fused min batch must be >= 0");
+      m->rc_min_b = (int)v;
+      return HB_OK;
+    case HB_OPT_ROWCHAIN: return flag(&m->opt_rowchain);
+    case HB_OPT_RC_CLUSTER:
+      HB_CHECK_ARG(v == 0 || v == 1 || v == 2 || v == 4 || v == 8, "cluster size must be 0, 1, 2, 4 or 8");
+      m->opt_rc_cluster = (int)v;
+      return HB_OK;
+    case HB_OPT_BWD_OVERLAP: return flag(&m->opt_bwd_overlap);
+    case HB_OPT_HEAD_FUSE: return flag(&m->opt_head_fuse);
+    case HB_OPT_DW_PAIR: return flag(&m->opt_dw_pair);
+    case HB_OPT_PDL: return flag(&m->opt_pdl);
+    case HB_OPT_GRAPHS: return flag(&m->opt_graphs);
+    case HB_OPT_INFLIGHT:
+      HB_CHECK_ARG(v >= 0 && v <= HB_MAX_INFLIGHT, "in-flight depth must be 0 (auto) .. 4");
+      m->opt_inflight = (int)v;
+      return HB_OK;
+    case HB_OPT_STAGE_ROWS:
+      HB_CHECK_ARG(v >= 0, "staging rows must be >= 0");
+      m->opt_stage_rows = v;
+      return HB_OK;
+    case HB_OPT_UPDATE:
+      HB_CHECK_ARG(v == HB_UPDATE_HOGWILD || v == HB_UPDATE_ATOMIC, "update must be HB_UPDATE_HOGWILD or _ATOMIC");
+      m->opt_update = (int)v;
+      return HB_OK;
+    default: return fail(HB_EINVAL, "unknown option key");
+  }
+}
+
+int mlp_get_option(const hb_model* m, int32_t key, int64_t* v) {
+  HB_CHECK_ARG(m && v, "null arg");
+  switch (key) {
+    case HB_OPT_FUSED_MIN_BATCH: *v = m->rc_min_b; return HB_OK;
+    case HB_OPT_ROWCHAIN: *v = m->opt_rowchain; return HB_OK;
+    case HB_OPT_RC_CLUSTER: *v = m->opt_rc_cluster; return HB_OK;
+    case HB_OPT_BWD_OVERLAP: *v = m->opt_bwd_overlap; return HB_OK;
+    case HB_OPT_HEAD_FUSE: *v = m->opt_head_fuse; return HB_OK;
+    case HB_OPT_DW_PAIR: *v = m->opt_dw_pair; return HB_OK;
+    case HB_OPT_PDL: *v = m->opt_pdl; return HB_OK;
+    case HB_OPT_GRAPHS: *v = m->opt_graphs; return HB_OK;
+    case HB_OPT_INFLIGHT: *v = m->opt_inflight; return HB_OK;
+    case HB_OPT_STAGE_ROWS: *v = m->opt_stage_rows; return HB_OK;
+    case HB_OPT_UPDATE: *v = m->opt_update; return HB_OK;
+    default: return fail(HB_EINVAL, "unknown option key");
+  }
 }
 
 int mlp_fused_path(const hb_model* m, int32_t batch, int32_t* cluster_size) {
@@ -1421,27 +1539,51 @@ int mlp_set_params(hb_model* m, const float* host_src, int64_t n) {
   return HB_OK;
 }
 
-int mlp_worker_create(hb_model* m, int32_t max_batch, int32_t replica, void* cuda_stream, hb_worker** out) {
+int mlp_worker_create(hb_model* m, int32_t device, int32_t max_batch, int32_t replica, void* cuda_stream,
+                      hb_worker** out) {
   HB_CHECK_ARG(m && out, "null arg");
   *out = nullptr;
   HB_CHECK_ARG(max_batch >= 1, "max_batch must be >= 1");
-  if (replica != 0) return fail(HB_EUNSUPPORTED, "only reference replicas (in-place Hogbatch updates) are implemented");
+  HB_CHECK_ARG(replica == 0 || replica == 1, "replica must be 0 (reference) or 1 (deep)");
+  if (device >= 0 && device != m->device)
+    return fail(HB_EUNSUPPORTED, "a worker runs on its model's device (one model per GPU; multi-GPU = one "
+                                 "process per GPU with a shared coordinator, hb_coord_create)");
   HB_CUDA_TRY(cudaSetDevice(m->device));
+  hb_model* target = m;
+  if (replica == 1) {  // deep replica [L134, L174]: a private copy of the global model's parameters
+    int rc = clone_model(m, &target);
+    if (rc) return rc;
+  }
   cudaStream_t s = static_cast<cudaStream_t>(cuda_stream);
   bool own = false;
   if (!s) {
     // a blocking stream: ordered after work on the legacy default stream (e.g. the caller's
     // torch copies of X/y), concurrent with the other workers' streams (Hogbatch, L170)
-    HB_CUDA_TRY(cudaStreamCreate(&s));
+    if (cudaStreamCreate(&s) != cudaSuccess) {
+      if (target != m) mlp_destroy(target);
+      return fail(HB_ECUDA, "stream create");
+    }
     own = true;
   }
-  return alloc_worker(m, max_batch, s, own, out);
+  int rc = alloc_worker(target, max_batch, s, own, out);  // frees its own stream on failure
+  if (rc) {
+    if (target != m) mlp_destroy(target);
+    return rc;
+  }
+  (*out)->global = m;
+  return HB_OK;
+}
+
+int mlp_worker_params(hb_worker* w, float* host_dst, int64_t n) {
+  HB_CHECK_ARG(w, "null worker");
+  return mlp_get_params(w->m, host_dst, n);
 }
 
 int mlp_worker_destroy(hb_worker* w) {
   if (!w) return HB_OK;
   cudaSetDevice(w->m->device);
   cudaStreamSynchronize(w->stream);
+  hb_model* replica = w->global && w->global != w->m ? w->m : nullptr;
   for (hb_worker* sw : w->subs) mlp_worker_destroy(sw);
   w->subs.clear();
   if (w->ev_fork) cudaEventDestroy(w->ev_fork);
@@ -1450,6 +1592,7 @@ int mlp_worker_destroy(hb_worker* w) {
   free_worker_buffers(w);
   if (w->own_stream) cudaStreamDestroy(w->stream);
   delete w;
+  if (replica) mlp_destroy(replica);
   return HB_OK;
 }
 
@@ -1460,13 +1603,13 @@ int mlp_worker_create_nested(hb_model* m, int32_t max_batch, int32_t t, void* cu
   *out = nullptr;
   HB_CHECK_ARG(t >= 1 && max_batch >= t, "need 1 <= t <= max_batch");
   hb_worker* w = nullptr;
-  int rc = mlp_worker_create(m, 1, 0, cuda_stream, &w);  // parent: stream + events only
+  int rc = mlp_worker_create(m, -1, 1, 0, cuda_stream, &w);  // parent: stream + events only
   if (rc) return rc;
   w->max_b = max_batch;
   const int sub_max = (max_batch + t - 1) / t;
   for (int i = 0; i < t; ++i) {
     hb_worker* sw = nullptr;
-    rc = mlp_worker_create(m, sub_max, 0, nullptr, &sw);
+    rc = mlp_worker_create(m, -1, sub_max, 0, nullptr, &sw);
     if (rc) {
       mlp_worker_destroy(w);
       return rc;
@@ -1536,6 +1679,7 @@ int mlp_row_losses(hb_worker* w, float* host_dst, int32_t n) {
   return HB_OK;
 }
 
+#ifdef HB_TUNING
 // Test/tuning only: times `iters` launches of one tensor-core GEMM configuration on scratch
 // buffers (bf16 operands filled with zeros, fp32 master); kind 0 = forward (bias+sigmoid),
 // 1 = dgrad (sigma'), 2 = wgrad + SGD.  Reports the mean device microseconds per launch.
@@ -1552,8 +1696,6 @@ int hb_bench_gemm_phases(int32_t kind, int32_t M, int32_t N, int32_t K, unsigned
 static int bench_gemm_impl(int32_t kind, int32_t M, int32_t N, int32_t K, int32_t iters, float* us_out,
                            unsigned long long* host_ts, int64_t cap) {
   HB_CHECK_ARG(us_out && M > 0 && N > 0 && K > 0 && iters > 0 && kind >= 0 && kind <= 3, "bad args");
-  const bool nostore = kind == 3;  // forward without output stores (epilogue cost probe)
-  if (nostore) kind = 0;
   const int64_t lda = round_up(kind == 2 ? M : K, 8), ldb = round_up(kind == 0 ? K : N, 8);
   const int64_t ldo = round_up(N, 8);
   const int64_t arows = kind == 2 ? K : M, brows = kind == 0 ? N : K;
@@ -1575,6 +1717,7 @@ static int bench_gemm_impl(int32_t kind, int32_t M, int32_t N, int32_t K, int32_
   cudaStream_t s;
   cudaStreamCreate(&s);
   EpiArgs ep{};
+    ep.no_pdl = !m->opt_pdl;
   ep.M = M;
   ep.N = N;
   int epi;
@@ -1585,7 +1728,6 @@ static int bench_gemm_impl(int32_t kind, int32_t M, int32_t N, int32_t K, int32_
     ep.out0 = O;
     ep.out1 = S;
     ep.ld0 = ep.ld1 = ldo;
-    if (nostore) ep.ld0 = -1;
   } else if (kind == 1) {
     epi = EPI_DGRAD_SIG;
     b_mn = true;
@@ -1606,8 +1748,8 @@ static int bench_gemm_impl(int32_t kind, int32_t M, int32_t N, int32_t K, int32_
     ep.bpart_in = bp;
     ep.ldp = M;
     ep.n_mtiles = (K + 127) / 128;
-    ep.pair = env_int("HB_DW_PAIR", 0);           // tuning: CTA-pair dW
-    ep.force_splits = env_int("HB_FORCE_SPLITS", 0);
+    ep.pair = HB_TUNE("HB_DW_PAIR", 0);           // tuning: CTA-pair dW
+    ep.force_splits = HB_TUNE("HB_FORCE_SPLITS", 0);
     ep.bias_upd = bias;
   }
   TcOp a{A, lda, arows, nullptr}, b{B, ldb, brows, nullptr};
@@ -1652,6 +1794,8 @@ static int bench_gemm_impl(int32_t kind, int32_t M, int32_t N, int32_t K, int32_
   return rc;
 }
 
+#endif  // HB_TUNING
+
 int mlp_loss(hb_model* m, const void* X, int64_t ldx, int32_t x_dtype, const int32_t* y, int64_t n,
              double* loss_out) {
   HB_CHECK_ARG(m && loss_out, "null arg");
@@ -1692,6 +1836,7 @@ int mlp_loss(hb_model* m, const void* X, int64_t ldx, int32_t x_dtype, const int
       for (int l = 0; l < L; ++l) {
         const Layer& Ly = m->layers[l];
         EpiArgs ep{};
+    ep.no_pdl = !m->opt_pdl;
         ep.M = b;
         ep.N = Ly.n_out;
         ep.bias = m->master + Ly.b_off;

@@ -53,7 +53,18 @@ struct hb_model {
   int device = 0;
   int prec = HB_PREC_BF16;
   std::vector<int> dims;
-  int rc_min_b = 4096;              // fused row-block step from this batch size up (0 = never)
+  // per-model settings (mlp_set_option, HB_OPT_*); defaults are the measured B200 choices
+  int rc_min_b = 4096;              // HB_OPT_FUSED_MIN_BATCH: fused row-block step from this b up (0 = never)
+  int opt_rowchain = 1;             // HB_OPT_ROWCHAIN
+  int opt_rc_cluster = 0;           // HB_OPT_RC_CLUSTER: CTAs per row block of the fused chain (0 = auto)
+  int opt_bwd_overlap = 1;          // HB_OPT_BWD_OVERLAP: dW_l on a second stream, overlapping dX_{l-1}
+  int opt_head_fuse = 0;            // HB_OPT_HEAD_FUSE: output layer's dX in the head epilogue
+  int opt_dw_pair = 0;              // HB_OPT_DW_PAIR: split-K dW GEMMs on CTA pairs (cta_group::2)
+  int opt_pdl = 1;                  // HB_OPT_PDL: programmatic dependent launch
+  int opt_graphs = 1;               // HB_OPT_GRAPHS: hogbatch_run replays one CUDA graph per (b, lr)
+  int opt_inflight = 0;             // HB_OPT_INFLIGHT: steps a worker may enqueue ahead (0 = auto)
+  int64_t opt_stage_rows = 0;       // HB_OPT_STAGE_ROWS: host-dataset staging chunk rows (0 = auto)
+  int opt_update = 0;               // HB_OPT_UPDATE: HB_UPDATE_HOGWILD or HB_UPDATE_ATOMIC
   std::vector<hb::Layer> layers;
   size_t total = 0;                 // floats in the flat parameter buffer (incl. padding)
   float* master = nullptr;          // fp32 master weights + biases (the shared global model)
@@ -76,7 +87,9 @@ struct hb_model {
 };
 
 struct hb_worker {
-  hb_model* m = nullptr;
+  hb_model* m = nullptr;        // the model this worker's steps update: the global model (reference
+                                // replica) or, for a deep replica, the worker's private copy
+  hb_model* global = nullptr;   // the global model the worker belongs to (== m for reference replicas)
   int max_b = 0;
   cudaStream_t stream = nullptr;
   bool own_stream = false;
@@ -120,6 +133,7 @@ struct hb_worker {
 };
 
 namespace hb {
+int clone_model(hb_model* m, hb_model** out);
 // One SGD step.  X / y: the batch's first row, or (d_off != nullptr, tensor-core path) the
 // dataset base with the batch's first row read from *d_off on the device.  x_rows = rows of X.
 int run_step(hb_worker* w, const void* X, int64_t ldx, int32_t xdt, int64_t x_rows, const int32_t* y,

@@ -290,14 +290,14 @@ __global__ void __launch_bounds__(RC_THREADS, 1) rowchain_kernel(const __grid_co
       tc_fence_after();
       unsigned long long* dbg =
           P.dbg && s < RC_DBG_STEPS ? P.dbg + ((size_t)blockIdx.x * RC_DBG_STEPS + s) * RC_DBG_W : nullptr;
-      if (dbg) dbg[0] = gtimer();
+      HB_STAMP(dbg, dbg[0]);
       const uint32_t tacc = tmem_base + (uint32_t)(buf * P.NH);
       const uint32_t idesc = make_idesc_bf16(128, st.N, false, st.bmn);
       // tuning only: per-k-block stamps of step 2 (issue, chunk ready, W ready) after the step table
       unsigned long long* kdbg = P.dbg && s == 2 ? P.dbg + (size_t)gridDim.x * RC_DBG_STEPS * RC_DBG_W : nullptr;
       for (int i = 0; i < st.nkb; ++i, ++it) {
         const int j = rc_kchunk(P, s, st.nkb, i, rank);
-        if (kdbg && i < 16) kdbg[blockIdx.x * 16 + i] = gtimer();
+        HB_STAMP(kdbg && i < 16, kdbg[blockIdx.x * 16 + i]);
         uint8_t* a_ptr;
         if (s == 0) {
           if (i == 0) mbar_wait(x_full, 0);
@@ -315,12 +315,12 @@ __global__ void __launch_bounds__(RC_THREADS, 1) rowchain_kernel(const __grid_co
           if (j / (P.NH / 64) != rank && s < NSTEPS - 1) mbar_arrive_expect_tx(&chunk_ready[j], RC_CHUNK);
           a_ptr = abuf + j * RC_CHUNK;
         }
-        if (kdbg && i < 16) kdbg[(gridDim.x + blockIdx.x) * 16 + i] = gtimer();
+        HB_STAMP(kdbg && i < 16, kdbg[(gridDim.x + blockIdx.x) * 16 + i]);
         const int stg = it % NS;
         mbar_wait(&w_full[stg], (it / NS) & 1);
         tc_fence_after();
-        if (kdbg && i < 16) kdbg[(2 * gridDim.x + blockIdx.x) * 16 + i] = gtimer();
-        if (dbg && i == 0) dbg[1] = gtimer();
+        HB_STAMP(kdbg && i < 16, kdbg[(2 * gridDim.x + blockIdx.x) * 16 + i]);
+        HB_STAMP(dbg && i == 0, dbg[1]);
         const uint32_t a_base = smem_u32(a_ptr);
         const uint32_t b_base = smem_u32(ring + stg * STB);
         for (int kk = 0; kk < st.kkn; ++kk) {
@@ -333,7 +333,7 @@ __global__ void __launch_bounds__(RC_THREADS, 1) rowchain_kernel(const __grid_co
       }
       umma_commit(&acc_full[buf]);
       if (CS > 1) umma_commit_multicast(peer_free, others);
-      if (dbg) dbg[2] = gtimer();
+      HB_STAMP(dbg, dbg[2]);
     }
   } else if (warp >= 4) {
     // ===== epilogue =====
@@ -373,9 +373,9 @@ __global__ void __launch_bounds__(RC_THREADS, 1) rowchain_kernel(const __grid_co
       tc_fence_after();
       unsigned long long* dbg =
           P.dbg && s < RC_DBG_STEPS && et == 0 ? P.dbg + ((size_t)blockIdx.x * RC_DBG_STEPS + s) * RC_DBG_W : nullptr;
-      if (dbg) dbg[3] = gtimer();
+      HB_STAMP(dbg, dbg[3]);
       if (CS > 1 && st.kind != RC_HEAD) mbar_wait(peer_free, s & 1);
-      if (dbg) dbg[4] = gtimer();
+      HB_STAMP(dbg, dbg[4]);
       const uint32_t tq = tmem_base + (uint32_t)(buf * P.NH) + ((uint32_t)(q * 32) << 16);
       if (st.kind == RC_HEAD) {
         // ---- softmax cross-entropy on the thread's row of logits (C <= 16) ----
@@ -463,7 +463,7 @@ __global__ void __launch_bounds__(RC_THREADS, 1) rowchain_kernel(const __grid_co
             for (int k = 0; k < RC_NSV; ++k) svn[k] = __ldg(srow + k);
           }
           tmem_ld_wait();
-          if (dbg && c == 0) dbg[6] = gtimer();
+          HB_STAMP(dbg && c == 0, dbg[6]);
           uint8_t* piece = abuf + g * RC_CHUNK + q * RC_PIECE;
           const uint32_t prow_s = smem_u32(piece) + lane * 128;
           const uint32_t sb_s = smem_u32(sbias) + (uint32_t)(c * 64 + h * RC_CPW) * 4;
@@ -540,11 +540,11 @@ __global__ void __launch_bounds__(RC_THREADS, 1) rowchain_kernel(const __grid_co
             sts128(prow_s + ((j0 ^ (lane & 7)) << 4), pk[0], pk[1], pk[2], pk[3]);
             sts128(prow_s + (((j0 + 1) ^ (lane & 7)) << 4), pk[4], pk[5], pk[6], pk[7]);
           }
-          if (dbg && c == 0) dbg[7] = gtimer();
+          HB_STAMP(dbg && c == 0, dbg[7]);
           fence_proxy_async();
-          if (dbg && c == 0) dbg[10] = gtimer();
+          HB_STAMP(dbg && c == 0, dbg[10]);
           quad_bar_sync(q);  // both halves of the piece are written
-          if (dbg && c == 0) dbg[11] = gtimer();
+          HB_STAMP(dbg && c == 0, dbg[11]);
           // the piece's asynchronous operations are issued by lane 0 of different warps of the
           // quadrant so their issue latencies overlap (each blocks ~0.1-0.3 us on B200):
           //   RC_H_COPY: bulk copies to the peers (their MMAs wait on them) + the local arrival,
@@ -560,19 +560,19 @@ __global__ void __launch_bounds__(RC_THREADS, 1) rowchain_kernel(const __grid_co
                                     mapa_shared(smem_u32(&chunk_ready[g]), dst));
               }
               mbar_arrive(&chunk_ready[g]);
-              if (dbg && c == 0) dbg[12] = gtimer();
+              HB_STAMP(dbg && c == 0, dbg[12]);
             }
             if (h == 0) {
               tma_store_2d(fwd ? &P.mH[lo] : &P.mDZ[lo], piece, n0, rb * 128 + q * 32);
               tma_store_commit();
-              if (dbg && c == 0) dbg[13] = gtimer();
+              HB_STAMP(dbg && c == 0, dbg[13]);
             }
             if (h == RC_H_S && fwd && P.s_tma) {
               tma_store_2d(&P.mS[lo], sstage + (c & 1) * RC_CHUNK + q * RC_PIECE, n0, rb * 128 + q * 32);
               tma_store_commit();  // one group per chunk (the staging reuse waits on chunk c-2's)
             }
           }
-          if (dbg) dbg[c == 0 ? 8 : 9] = gtimer();
+          HB_STAMP(dbg, dbg[c == 0 ? 8 : 9]);
 #pragma unroll
           for (int k = 0; k < RC_NSV; ++k) sv[k] = svn[k];
         }
@@ -581,7 +581,7 @@ __global__ void __launch_bounds__(RC_THREADS, 1) rowchain_kernel(const __grid_co
       tc_fence_before();
       __syncwarp();
       if (lane == 0) mbar_arrive(&acc_empty[buf]);
-      if (dbg) dbg[5] = gtimer();
+      HB_STAMP(dbg, dbg[5]);
     }
     if (lane == 0) tma_store_wait_all();
   }

@@ -129,8 +129,12 @@ __device__ __forceinline__ void bias_reduce_update(const EpiArgs& ep, int lo, in
   for (int o = 1; o < tpr; o <<= 1) acc += __shfl_xor_sync(0xffffffffu, acc, o);
   if (r < R && k == 0) {
     const int bi = lo + r;
-    if (EPI == EPI_WGRAD_SGD)
-      ep.bias_upd[bi] -= ep.lr * acc;
+    if (EPI == EPI_WGRAD_SGD) {
+      if (ep.atomic)
+        atomicAdd(ep.bias_upd + bi, __fmul_rn(-ep.lr, acc));
+      else
+        ep.bias_upd[bi] += __fmul_rn(-ep.lr, acc);
+    }
     else
       ep.bias_grad[bi] = acc;
   }
@@ -185,7 +189,7 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
   const int warp = threadIdx.x >> 5;
   const int lane = threadIdx.x & 31;
   unsigned long long* dbg = ep.dbg ? ep.dbg + 12 * ((size_t)(blockIdx.z * gridDim.y + blockIdx.y) * gridDim.x + blockIdx.x) : nullptr;
-  if (dbg && threadIdx.x == 0) dbg[0] = gtimer();
+  HB_STAMP(dbg && threadIdx.x == 0, dbg[0]);
   // Tiles: persistent CTAs walk tiles t = blockIdx.x, +gridDim.x, ... (n fastest, so CTAs running
   // together share the A row panel in L2).  Split-K launches (gridDim.z > 1) are one tile per CTA.
   const int tiles_n = (ep.N + BN - 1) / BN;
@@ -235,7 +239,7 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
   // no global memory produced by it is touched before this point
   asm volatile("griddepcontrol.wait;" ::: "memory");
   asm volatile("griddepcontrol.launch_dependents;" ::: "memory");
-  if (dbg && threadIdx.x == 0) dbg[1] = gtimer();
+  HB_STAMP(dbg && threadIdx.x == 0, dbg[1]);
 
   if (warp == 0 && lane == 0) {
     // ===== TMA producer =====
@@ -297,7 +301,7 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
       const uint32_t ph = (it / STAGES) & 1;
       mbar_wait(&full_bar[s], ph);
       tc_fence_after();
-      if (dbg && it == 0) dbg[2] = gtimer();
+      HB_STAMP(dbg && it == 0, dbg[2]);
       const uint32_t a_base = smem_u32(smem + s * Cfg::STAGE_BYTES);
       const uint32_t b_base = a_base + Cfg::A_BYTES;
 #pragma unroll
@@ -323,7 +327,7 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
       umma_commit_pair(&tmem_full_bar[acc], pair_mask);
     else
       umma_commit(&tmem_full_bar[acc]);  // accumulator ready (arrives even if num_kb == 0)
-    if (dbg && i == 0) dbg[3] = gtimer();
+    HB_STAMP(dbg && i == 0, dbg[3]);
     }
   } else if (warp >= 4) {
     // ===== epilogue (8 warps): TMEM -> registers -> fused epilogue -> global =====
@@ -372,10 +376,10 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
     }
     if (TO::on && et == 0) tma_store_wait_read();  // staging buffer of the previous tile free
     epi_bar_sync();  // sbias visible; previous tile's partial sums consumed; staging free
-    if (dbg && et == 0 && i == 0) dbg[4] = gtimer();
+    HB_STAMP(dbg && et == 0 && i == 0, dbg[4]);
     mbar_wait(&tmem_full_bar[acc], (i >> 1) & 1);
     tc_fence_after();
-    if (dbg && et == 0 && i == 0) dbg[5] = gtimer();
+    HB_STAMP(dbg && et == 0 && i == 0, dbg[5]);
 
     if (EPI == EPI_HEAD_XENT) {
       // ---- softmax cross-entropy on the thread's own row of logits (N = C <= BN = 16) ----
@@ -587,16 +591,7 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
             stage16<TO::NBOX>(sout, 0, rl, c, hp);
             if (ep.out1) stage16<TO::NBOX>(sout, 1, rl, c, sp);
           } else if (row_ok) {
-            if (EPI == EPI_FWD_SIG && ep.ld0 < 0) {  // tuning probe: epilogue math, no stores
-              float acc = 0.f;
-#pragma unroll
-              for (int qq = 0; qq < 16; ++qq) {
-                float hv, dv;
-                sigmoid_d_fast(v[qq] + sb[c + qq], hv, dv);
-                acc += hv + dv;
-              }
-              if (acc == 12345.f) static_cast<float*>(ep.bias_upd)[0] = acc;
-            } else if (EPI == EPI_FWD_SIG && full) {
+            if (EPI == EPI_FWD_SIG && full) {
               uint32_t hp[8], sp[8];
 #pragma unroll
               for (int qq = 0; qq < 8; ++qq) {
@@ -703,15 +698,15 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
       for (int u = 0; u < RED_MAXIT; ++u) {
         wpre[u] = make_float4(0.f, 0.f, 0.f, 0.f);
         const int e = (tid + u * TC_EPI_THREADS) * 4;
-        if (EPI == EPI_WGRAD_SGD && warp >= 4 && !ep.transposed && e < rps * BN) {
+        if (EPI == EPI_WGRAD_SGD && warp >= 4 && !ep.transposed && !ep.atomic && e < rps * BN) {
           const int gm = m_tile * TC_BM + kz * rps + e / BN, gn = n_tile * BN + e % BN;
           if (gm < ep.M && gn + 4 <= ep.N) wpre[u] = __ldcg(reinterpret_cast<const float4*>(ep.master + (int64_t)gm * ep.ldw + gn));
         }
       }
     }
-    if (dbg && threadIdx.x == 128) dbg[8] = gtimer();
+    HB_STAMP(dbg && threadIdx.x == 128, dbg[8]);
     cluster_sync_all();  // every partial tile is in shared memory (release/acquire, cluster scope)
-    if (dbg && threadIdx.x == 128) dbg[9] = gtimer();
+    HB_STAMP(dbg && threadIdx.x == 128, dbg[9]);
     if (warp >= 4) {
       const int t = t_first;
       int m_tile, n_tile;
@@ -737,7 +732,7 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
         const bool vec = in && !ep.transposed && gn + 4 <= ep.N && EPI == EPI_WGRAD_SGD;
         float4* W = vec ? reinterpret_cast<float4*>(ep.master + (int64_t)gm * ep.ldw + gn) : nullptr;
         float4 w = make_float4(0.f, 0.f, 0.f, 0.f);
-        if (vec) {
+        if (vec && !ep.atomic) {
           if (u < RED_MAXIT) {  // prefetched (static register index via the unrolled select)
 #pragma unroll
             for (int k = 0; k < RED_MAXIT; ++k)
@@ -781,11 +776,16 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
         if (!in) continue;
         const float a4[4] = {acc.x, acc.y, acc.z, acc.w};
         if (vec) {
-          w.x -= ep.lr * acc.x;
-          w.y -= ep.lr * acc.y;
-          w.z -= ep.lr * acc.z;
-          w.w -= ep.lr * acc.w;
-          *W = w;
+          const float4 d = sgd_delta4(ep.lr, acc.x, acc.y, acc.z, acc.w);
+          if (ep.atomic) {
+            w = sgd_atomic4(W, d);
+          } else {
+            w.x += d.x;
+            w.y += d.y;
+            w.z += d.z;
+            w.w += d.w;
+            *W = w;
+          }
           uint2 sh = make_uint2(pack_bf16x2(w.x, w.y), pack_bf16x2(w.z, w.w));
           *reinterpret_cast<uint2*>(ep.shadow + (int64_t)gm * ep.ldw + gn) = sh;
         } else {
@@ -794,7 +794,7 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
             if (gn + j < (ep.hilo ? ep.n_real : ep.N)) epi_elem<EPI, __nv_bfloat16, false>(ep, gm, gn + j, a4[j]);
         }
       }
-      if (dbg && threadIdx.x == 128) dbg[10] = gtimer();
+      HB_STAMP(dbg && threadIdx.x == 128, dbg[10]);
       if (ep.bpart_in) {  // bias: rows of this CTA's slice (or, transposed, the tile's columns)
         int lo, hi;
         bool own;
@@ -810,12 +810,12 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
         if (own) bias_reduce_update<EPI>(ep, lo, hi, tid);
       }
     }
-    if (dbg && threadIdx.x == 128) dbg[11] = gtimer();
+    HB_STAMP(dbg && threadIdx.x == 128, dbg[11]);
     cluster_sync_all();  // no CTA leaves while another still reads its partial tile
   }
 
   if (TO::on && threadIdx.x == 128) tma_store_wait_all();  // bulk stores complete before exit
-  if (dbg && threadIdx.x == 128) dbg[6] = gtimer();
+  HB_STAMP(dbg && threadIdx.x == 128, dbg[6]);
   tc_fence_before();
   __syncthreads();
   if (warp == 2) {
@@ -825,7 +825,7 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
     else
       tmem_dealloc<Cfg::TMEM_COLS>(tmem_base);
   }
-  if (dbg && threadIdx.x == 64) dbg[7] = gtimer();
+  HB_STAMP(dbg && threadIdx.x == 64, dbg[7]);
 }
 
 }  // namespace hb

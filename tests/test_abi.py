@@ -26,7 +26,7 @@ def test_library_exports_every_declared_symbol():
     for n in names:
         assert hasattr(hb.lib, n), n
     assert set(names) == set(hb._lib.EXPORTS)
-    assert hb.lib.hb_abi_version() == 1
+    assert hb.lib.hb_abi_version() == 2
 
 
 def test_no_device_is_reported_for_bad_ordinal():

@@ -137,15 +137,15 @@ def test_graph_replay_is_bitwise_equal_to_direct_launches():
 
 
 @pytest.mark.parametrize("det,pinned", [(False, True), (True, True), (False, False)])
-def test_host_dataset_is_staged_and_bitwise_equal_to_device_dataset(det, pinned, monkeypatch):
+def test_host_dataset_is_staged_and_bitwise_equal_to_device_dataset(det, pinned):
     # hogbatch_run with HOST X / y (pinned): staged in chunks overlapped with training; the model
     # after two epochs equals the run on the device copy bit for bit (same batches, same kernels)
-    monkeypatch.setenv("HB_STAGE_ROWS", "1000")  # several chunks, ragged last chunk
     dims = [54, 256, 128, 7]
     N = 4500
     out = []
     for host in (False, True):
         X, y, m, params, tX, ty = setup(dims, "bf16", 512, N)
+        m.set_option("stage_rows", 1000)  # several chunks, ragged last chunk
         w = hb.Worker(m, 512)
         pol = hb.Policy(kind=hb.HB_MINIBATCH, workers=[hb.WorkerSpec(512, 512, 512)], eta0=0.1, b0=32,
                         deterministic=det, eval_loss=True)
@@ -333,21 +333,16 @@ def test_nested_hogwild_worker_in_adaptive_run():
 
 
 def test_fused_head_dx_matches_oracle():
-    # opt-in fusion of the output layer's dX into the head kernel (HB_HEAD_FUSE=1), in a child
-    # process so the env knob is read fresh
-    import subprocess
-    import sys
-    code = (
-        "import numpy as np, torch, sys; sys.path.insert(0, '.');"
-        "import paper_conf_ipps_marws21_b200 as hb; from oracle import mlp64;"
-        "from tests.helpers import *;"
-        "dims=[54,256,200,7]; X,y=dataset('covtype',1000,seed=7);"
-        "m=hb.MLP(dims); p=init_params(dims); m.set_params(params_to_flat(p)); w=hb.Worker(m,1000);"
-        "tX,ty=to_device(X,y); g,l=w.step_grads(tX,ty,1000); dW,db,lr=mlp64.grads(p,X.astype(np.float64),y);"
-        "G=split_flat(g,dims); e=max(max(rel_err(G[i][0],dW[i]),rel_err(G[i][1],db[i])) for i in range(3));"
-        "print('ERR', e); assert e <= 1e-2")
-    import os
-    env = dict(os.environ, HB_HEAD_FUSE="1")
-    r = subprocess.run([sys.executable, "-c", code], capture_output=True, text=True, env=env, timeout=300,
-                       cwd=os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
-    assert r.returncode == 0, r.stdout + r.stderr
+    # opt-in fusion of the output layer's dX into the head kernel (HB_OPT_HEAD_FUSE)
+    dims = [54, 256, 200, 7]
+    X, y = dataset("covtype", 1000, seed=7)
+    m = hb.MLP(dims)
+    p = init_params(dims)
+    m.set_params(params_to_flat(p))
+    m.set_option("head_fuse", 1)
+    w = hb.Worker(m, 1000)
+    tX, ty = to_device(X, y)
+    g, _ = w.step_grads(tX, ty, 1000)
+    dW, db, _ = mlp64.grads(p, X.astype(np.float64), y)
+    norm, elem = grad_errors(g, dims, dW, db)
+    assert max(norm) <= 1e-2 and max(elem) <= 1e-2, (norm, elem)

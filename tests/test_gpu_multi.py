@@ -1,0 +1,209 @@
+"""GPU tests of the multi-worker / multi-replica paths, through the C ABI:
+
+* deep replicas [L134, L174] and the local replica merge (hb_merge_replicas) vs oracle/merge.py
+  for n = 2, 4, 8 replicas emulated on one GPU (the same merge arithmetic as n GPUs);
+* hogbatch_run over deep replicas with merges at the coordinator's merge points;
+* HB_UPDATE_ATOMIC (atomic adds in the dW epilogue) vs Hogwild read-modify-write, and beta — the
+  fraction of concurrent sub-batch updates that survive [L238] — measured;
+* the policy's epoch_barrier = 0 and check_labels;
+* two processes on one GPU scheduling from ONE shared coordinator (hb_coord_create).
+"""
+import os
+import uuid
+
+import numpy as np
+import pytest
+
+torch = pytest.importorskip("torch")
+pytestmark = pytest.mark.gpu
+
+import paper_conf_ipps_marws21_b200 as hb  # noqa: E402
+from oracle import merge as omerge  # noqa: E402
+from oracle import mlp64  # noqa: E402
+from tests.helpers import dataset, init_params, params_to_flat, split_flat, to_device  # noqa: E402
+
+
+def _gpu():
+    if not torch.cuda.is_available() or not hb.device_ok(0):
+        pytest.fail("no sm_100 GPU visible")
+
+
+def _model(dims, N, seed=0):
+    _gpu()
+    X, y = dataset("covtype", N, d=dims[0], seed=seed)
+    y = (y % dims[-1]).astype(np.int32)
+    m = hb.MLP(dims)
+    params = init_params(dims, seed=2)
+    m.set_params(params_to_flat(params))
+    tX, ty = to_device(X, y)
+    return X, y, m, params, tX, ty
+
+
+@pytest.mark.parametrize("n", [2, 4, 8])
+@pytest.mark.parametrize("gamma", [1.0, 0.25])
+def test_replica_merge_matches_oracle(n, gamma):
+    # n deep replicas take different SGD steps; hb_merge_replicas must equal oracle/merge.py's
+    # W_base + gamma * sum_E (W_E - W_base) on the replicas' actual fp32 parameters (<= 1e-6)
+    dims, b = [54, 128, 64, 7], 256
+    X, y, m, params, tX, ty = _model(dims, n * b * 2)
+    m.merge_begin()
+    base = split_flat(m.get_params(), dims)
+    ws = [hb.Worker(m, b, replica=True) for _ in range(n)]
+    for E, w in enumerate(ws):
+        for k in range(2):
+            off = (2 * E + k) * b
+            w.step(tX[off:], ty[off:], b, 0.5)
+    torch.cuda.synchronize()
+    assert np.array_equal(m.get_params(), params_to_flat(params))  # the global model is untouched
+    reps = [split_flat(w.params(), dims) for w in ws]
+    assert all(not np.array_equal(reps[0][0][0], r[0][0]) for r in reps[1:])
+    m.merge_replicas(ws, gamma)
+    got = m.get_params()
+    exp = params_to_flat(omerge.merge(base, reps, gamma)).astype(np.float64)
+    np.testing.assert_allclose(got, exp, rtol=1e-6, atol=1e-7)
+    for w in ws:  # every replica continues from the merged model
+        assert np.array_equal(w.params(), got)
+
+
+def test_hogbatch_run_over_deep_replicas_trains_and_merges():
+    dims, N = [54, 128, 128, 7], 24000
+    X, y, m, params, tX, ty = _model(dims, N)
+    ws = [hb.Worker(m, 1024, replica=True) for _ in range(4)]
+    specs = [hb.WorkerSpec(256, 1024, 1024) for _ in range(4)]
+    pol = hb.Policy(kind=hb.HB_ADAPTIVE, workers=specs, eta0=0.02, b0=32, merges_per_epoch=3, merge_gamma=0.25,
+                    eval_loss=True)
+    l0 = mlp64.full_loss(params, X.astype(np.float64), y)
+    st = hb.hogbatch_run(ws, pol, tX, ty, epochs=3, trace_cap=10000)
+    assert st["n_merges"] == 9 and st["epochs_done"] == 3
+    assert st["epoch_loss"][-1] < 0.95 * l0, (st["epoch_loss"], l0)
+    final = m.get_params()
+    for w in ws:
+        assert np.array_equal(w.params(), final)
+    for e in range(3):  # one 𝔹 per epoch: disjoint contiguous ranges from row 0
+        served = sorted((r[10], r[7]) for r in st["trace"] if r[1] == e and r[9])
+        assert served[0][0] == 0 and all(a[0] + a[1] == b_[0] for a, b_ in zip(served, served[1:]))
+    with pytest.raises(hb.HogbatchError):  # deep replicas need merge points
+        hb.hogbatch_run(ws, hb.Policy(kind=hb.HB_ADAPTIVE, workers=specs, eta0=0.02, b0=32), tX, ty, epochs=1)
+
+
+def test_atomic_update_equals_hogwild_for_one_worker():
+    # one worker: no concurrency, so atomic adds of -lr*dW give exactly the read-modify-write result
+    dims = [54, 256, 128, 7]
+    out = []
+    for mode in (hb.HB_UPDATE_HOGWILD, hb.HB_UPDATE_ATOMIC):
+        X, y, m, params, tX, ty = _model(dims, 4096)
+        m.set_option("update", mode)
+        w = hb.Worker(m, 512)
+        pol = hb.Policy(kind=hb.HB_MINIBATCH, workers=[hb.WorkerSpec(512, 512, 512)], eta0=0.1, b0=32,
+                        deterministic=True)
+        hb.hogbatch_run([w], pol, tX, ty, epochs=2)
+        out.append(m.get_params())
+    assert np.array_equal(out[0], out[1])
+
+
+def measure_beta(t=8, s=128, dims=(54, 512, 512, 7), lr=1e-3):
+    """beta [L238]: a nested worker runs t IDENTICAL sub-batches concurrently on the shared model.
+    Returns (d_seq, d_atomic, d_hogwild): the parameter change of t sequential single-worker steps
+    and of the concurrent run under atomic adds and under Hogwild read-modify-write."""
+    dims = list(dims)
+    X1, y1 = dataset("covtype", s, seed=11)
+    y1 = (y1 % dims[-1]).astype(np.int32)
+    X, y = np.tile(X1, (t, 1)), np.tile(y1, t)
+    tX, ty = to_device(X, y)
+    P0 = params_to_flat(init_params(dims, seed=2))
+    out = {}
+    for mode in (hb.HB_UPDATE_ATOMIC, hb.HB_UPDATE_HOGWILD):
+        m = hb.MLP(dims)
+        m.set_option("update", mode)
+        m.set_params(P0)
+        w = hb.Worker(m, t * s, sub_batches=t)
+        w.step(tX, ty, t * s, lr * t)  # each sub-batch: lr * size / b = lr
+        torch.cuda.synchronize()
+        out[mode] = m.get_params().astype(np.float64) - P0
+    m = hb.MLP(dims)
+    m.set_params(P0)
+    w = hb.Worker(m, s)
+    for k in range(t):
+        w.step(tX[k * s:], ty[k * s:], s, lr)
+    torch.cuda.synchronize()
+    return m.get_params().astype(np.float64) - P0, out[hb.HB_UPDATE_ATOMIC], out[hb.HB_UPDATE_HOGWILD]
+
+
+def test_atomic_updates_all_survive_and_beta_is_measured():
+    # atomic adds: the t concurrent updates all land (the result equals t sequential steps up to
+    # the O(lr^2) effect of which weights each sub-batch read); beta = the Hogwild run's share of
+    # the atomic run's update, <d_hog, d_atom> / |d_atom|^2 (measured 1.000 on B200)
+    _gpu()
+    for t, s in [(8, 128), (4, 2048)]:
+        d_seq, d_atom, d_hog = measure_beta(t, s)
+        err = np.linalg.norm(d_atom - d_seq) / np.linalg.norm(d_seq)
+        beta = float(d_hog @ d_atom / (d_atom @ d_atom))
+        print(f"t={t} s={s}: |atomic - sequential| / |sequential| = {err:.2e}, beta = {beta:.5f}")
+        assert err <= 1e-2
+        assert 0.5 < beta <= 1.0 + 1e-3
+
+
+def test_epoch_barrier_off_and_label_check():
+    dims = [54, 128, 7]
+    X, y, m, params, tX, ty = _model(dims, 5000)
+    ws = [hb.Worker(m, 1024), hb.Worker(m, 256)]
+    specs = [hb.WorkerSpec(1024, 1024, 1024), hb.WorkerSpec(64, 256, 64)]
+    pol = hb.Policy(kind=hb.HB_ADAPTIVE, workers=specs, eta0=0.02, b0=32, epoch_barrier=False, check_labels=True)
+    st = hb.hogbatch_run(ws, pol, tX, ty, epochs=4, trace_cap=100000)
+    assert st["epochs_done"] == 4
+    for e in range(4):  # every epoch still serves disjoint contiguous ranges from row 0
+        served = sorted((r[10], r[7]) for r in st["trace"] if r[1] == e and r[9])
+        assert served[0][0] == 0 and all(a[0] + a[1] == b_[0] for a, b_ in zip(served, served[1:]))
+    bad = ty.clone()
+    bad[17] = 7  # C = 7 classes: label 7 is out of range
+    with pytest.raises(hb.HogbatchError):
+        hb.hogbatch_run(ws, pol, tX, bad, epochs=1)
+
+
+_TWO_PROC = r"""
+import os, sys, json
+sys.path.insert(0, os.getcwd())
+import numpy as np, torch
+import paper_conf_ipps_marws21_b200 as hb
+from tests.helpers import dataset, init_params, params_to_flat, to_device
+rank, name = int(sys.argv[1]), sys.argv[2]
+dims, N = [54, 128, 128, 7], 20000
+X, y = dataset("covtype", N, seed=0)
+m = hb.MLP(dims)
+m.set_params(params_to_flat(init_params(dims, seed=2)))
+tX, ty = to_device(X, y)
+specs = [hb.WorkerSpec(512, 2048, 2048), hb.WorkerSpec(32, 512, 32)]   # GPU0 large, GPU1 small (C3 split)
+w = hb.Worker(m, specs[rank].max_b)
+pol = hb.Policy(kind=hb.HB_ADAPTIVE, workers=specs, eta0=0.02, b0=32, first_worker=rank)
+pol.coord = hb.Coord(name, pol, N, 2, rank)
+st = hb.hogbatch_run([w], pol, tX, ty, epochs=3, trace_cap=100000)
+print(json.dumps({"trace": [list(r) for r in st["trace"]], "epochs": st["epochs_done"]}))
+pol.coord.close()
+"""
+
+
+def test_two_processes_share_one_coordinator_on_one_gpu():
+    # the multi-GPU process model (one process per GPU, one coordinator for the node) exercised with
+    # two processes on the one GPU of the test box: together they serve ONE set 𝔹 per epoch, and
+    # Algorithm 2 compares their workers' update counts (the small-batch worker's batch grows)
+    import json
+    import subprocess
+    import sys
+    _gpu()
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    name = f"/hbtest_{uuid.uuid4().hex[:12]}"
+    procs = [subprocess.Popen([sys.executable, "-c", _TWO_PROC, str(r), name], cwd=root, stdout=subprocess.PIPE,
+                              stderr=subprocess.PIPE, text=True) for r in range(2)]
+    outs = [p.communicate(timeout=600) for p in procs]
+    for p, (o, e) in zip(procs, outs):
+        assert p.returncode == 0, e[-3000:]
+    res = [json.loads(o.strip().splitlines()[-1]) for o, _ in outs]
+    assert all(r["epochs"] == 3 for r in res)
+    trace = sorted([tuple(t) for r in res for t in r["trace"]], key=lambda t: t[0])
+    assert [t[0] for t in trace] == list(range(len(trace)))  # one message sequence for both
+    assert {t[2] for t in res[0]["trace"]} == {0} and {t[2] for t in res[1]["trace"]} == {1}
+    for e in range(3):
+        served = sorted((t[10], t[7]) for t in trace if t[1] == e and t[9])
+        assert served[0][0] == 0 and all(a[0] + a[1] == b_[0] for a, b_ in zip(served, served[1:]))
+        assert {t[2] for t in trace if t[1] == e and t[9]} == {0, 1}
+    assert any(t[6] in ("double", "halve") for t in trace)  # the adaptive rule acted across processes

@@ -16,7 +16,7 @@ pytestmark = pytest.mark.gpu
 
 import paper_conf_ipps_marws21_b200 as hb  # noqa: E402
 from oracle import mlp64  # noqa: E402
-from tests.helpers import dataset, init_params, params_to_flat, rel_err, split_flat, to_device  # noqa: E402
+from tests.helpers import dataset, grad_errors, init_params, params_to_flat, rel_err, split_flat, to_device  # noqa: E402
 
 TOL = 1e-2
 
@@ -111,43 +111,26 @@ def test_fused_saturated_init():
         assert rel_err(got[l][1], db[l]) <= TOL, l
 
 
-_FORCED_CS_SCRIPT = r"""
-import os, sys, json
-sys.path.insert(0, os.getcwd())
-import numpy as np
-import paper_conf_ipps_marws21_b200 as hb
-from oracle import mlp64
-from tests.helpers import dataset, init_params, params_to_flat, rel_err, split_flat, to_device
-dims, b = [54, 256, 256, 7], 300
-X, y = dataset("covtype", b, seed=13)
-m = hb.MLP(dims, precision="bf16", seed=0)
-m.set_fused_min_batch(1)
-params = init_params(dims, seed=2)
-m.set_params(params_to_flat(params))
-w = hb.Worker(m, b)
-tX, ty = to_device(X, y)
-g, loss = w.step_grads(tX, ty, b)
-dW, db, l_ref = mlp64.grads(params, X.astype(np.float64), y)
-got = split_flat(g, dims)
-err = max(max(rel_err(got[l][0], dW[l]), rel_err(got[l][1], db[l])) for l in range(len(dims) - 1))
-print(json.dumps({"cs": m.fused_path(b), "err": err, "lerr": abs(loss - l_ref) / l_ref}))
-"""
-
-
 @pytest.mark.parametrize("cs", [1, 2, 4, 8])
 def test_every_cluster_size_matches_oracle(cs):
-    # the same 256-wide net at every cluster size (HB_RC_CS), each in a fresh process; at CS = 8
-    # the last four CTAs of every cluster own no valid column (n = 256 < 8 x 64 chunks)
-    import json, os, subprocess, sys
+    # the same 256-wide net at every cluster size (HB_OPT_RC_CLUSTER); at CS = 8 the last four CTAs
+    # of every cluster own no valid column (n = 256 < 8 x 64 chunks)
     _need_gpu()
-    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
-    env = dict(os.environ, HB_RC_CS=str(cs))
-    out = subprocess.run([sys.executable, "-c", _FORCED_CS_SCRIPT], cwd=root, env=env, capture_output=True,
-                         text=True, timeout=300)
-    assert out.returncode == 0, out.stderr[-2000:]
-    r = json.loads(out.stdout.strip().splitlines()[-1])
-    assert r["cs"] == cs
-    assert r["err"] <= TOL and r["lerr"] <= TOL, r
+    dims, b = [54, 256, 256, 7], 300
+    X, y = dataset("covtype", b, seed=13)
+    m = hb.MLP(dims, precision="bf16", seed=0)
+    m.set_fused_min_batch(1)
+    m.set_option("rc_cluster", cs)
+    params = init_params(dims, seed=2)
+    m.set_params(params_to_flat(params))
+    w = hb.Worker(m, b)
+    tX, ty = to_device(X, y)
+    g, loss = w.step_grads(tX, ty, b)
+    dW, db, l_ref = mlp64.grads(params, X.astype(np.float64), y)
+    assert m.fused_path(b) == cs
+    norm, elem = grad_errors(g, dims, dW, db)
+    assert max(norm) <= TOL and max(elem) <= TOL, (norm, elem)
+    assert abs(loss - l_ref) / l_ref <= TOL
 
 
 def test_unfused_shapes_report_layer_chain():
