@@ -14,8 +14,33 @@ namespace hb {
 // softmax cross-entropy: one warp per row.
 //   lse_i = m_i + log sum_c exp(z_ic - m_i),  loss_i = lse_i - z_{i,y_i}
 //   dZ_ic = (exp(z_ic - lse_i) - [c == y_i]) * inv_b        (gradient of the batch MEAN loss)
-// dZ may be null (loss only, mlp_loss).  C is arbitrary (loops over 32-wide column chunks).
+// dZ may be null (loss only, mlp_loss).  C <= 1024 with 16-byte aligned rows (ldl % 4 == 0): the
+// row is read ONCE into registers (float4 per lane, <= 8 per lane), so the kernel streams
+// b*C*4 bytes of logits in and b*C*sizeof(TDZ) bytes of dZ out (HBM-bound); larger C loops.
 // ---------------------------------------------------------------------------------------
+template <typename TDZ>
+__device__ __forceinline__ void store4(TDZ* d, int c, int C, float a, float b, float e, float f) {
+  const float v[4] = {a, b, e, f};
+#pragma unroll
+  for (int j = 0; j < 4; ++j)
+    if (c + j < C) d[c + j] = to_act<TDZ>(v[j]);
+}
+template <>
+__device__ __forceinline__ void store4<__nv_bfloat16>(__nv_bfloat16* d, int c, int C, float a, float b, float e, float f) {
+  if (c + 4 <= C && ((reinterpret_cast<uintptr_t>(d + c) & 7) == 0)) {
+    __nv_bfloat162 lo = __floats2bfloat162_rn(a, b), hi = __floats2bfloat162_rn(e, f);
+    uint2 u;
+    u.x = *reinterpret_cast<uint32_t*>(&lo);
+    u.y = *reinterpret_cast<uint32_t*>(&hi);
+    *reinterpret_cast<uint2*>(d + c) = u;
+    return;
+  }
+  const float v[4] = {a, b, e, f};
+#pragma unroll
+  for (int j = 0; j < 4; ++j)
+    if (c + j < C) d[c + j] = __float2bfloat16_rn(v[j]);
+}
+
 template <typename TDZ>
 __global__ void softmax_xent_kernel(const float* __restrict__ logits, int64_t ldl,
                                     const int32_t* __restrict__ y, const int* __restrict__ yoff, int b, int C, TDZ* dZ,
@@ -24,6 +49,62 @@ __global__ void softmax_xent_kernel(const float* __restrict__ logits, int64_t ld
   const int lane = threadIdx.x & 31;
   if (warp >= b) return;
   const float* z = logits + (int64_t)warp * ldl;
+  const int yi = y[(yoff ? *yoff : 0) + warp];
+  if (C <= 1024 && (ldl & 3) == 0) {
+    // one exp per element (kept in registers: p = exp(z - m)), dZ = p / s - onehot, scaled by 1/b
+    constexpr int V = 8;
+    constexpr float LOG2E = 1.4426950408889634f;
+    float4 v[V];
+    float m = -INFINITY;
+#pragma unroll
+    for (int i = 0; i < V; ++i) {
+      const int c = (i * 32 + lane) * 4;
+      v[i] = make_float4(-INFINITY, -INFINITY, -INFINITY, -INFINITY);
+      if (c < C) {
+        const float4 t = __ldg(reinterpret_cast<const float4*>(z + c));
+        v[i].x = t.x;
+        v[i].y = c + 1 < C ? t.y : -INFINITY;
+        v[i].z = c + 2 < C ? t.z : -INFINITY;
+        v[i].w = c + 3 < C ? t.w : -INFINITY;
+      }
+      m = fmaxf(m, fmaxf(fmaxf(v[i].x, v[i].y), fmaxf(v[i].z, v[i].w)));
+    }
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) m = fmaxf(m, __shfl_xor_sync(0xffffffffu, m, o));
+    const float mb = m * LOG2E;
+    float s = 0.f;
+#pragma unroll
+    for (int i = 0; i < V; ++i) {  // exp2(z*log2e - m*log2e); exp2(-inf) = 0 for the masked tail
+      v[i].x = exp2f(fmaf(v[i].x, LOG2E, -mb));
+      v[i].y = exp2f(fmaf(v[i].y, LOG2E, -mb));
+      v[i].z = exp2f(fmaf(v[i].z, LOG2E, -mb));
+      v[i].w = exp2f(fmaf(v[i].w, LOG2E, -mb));
+      s += (v[i].x + v[i].y) + (v[i].z + v[i].w);
+    }
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) s += __shfl_xor_sync(0xffffffffu, s, o);
+    if (lane == 0) row_loss[warp] = m + logf(s) - __ldg(z + yi);
+    if (dZ) {
+      TDZ* d = dZ + (int64_t)warp * ldz;
+      const float sc = inv_b / s;
+#pragma unroll
+      for (int i = 0; i < V; ++i) {
+        const int c = (i * 32 + lane) * 4;
+        if (c < C) {
+          float4 g = make_float4(v[i].x * sc, v[i].y * sc, v[i].z * sc, v[i].w * sc);
+          if (yi >= c && yi < c + 4) {  // the label's column: - 1/b
+            const int j = yi - c;
+            if (j == 0) g.x -= inv_b;
+            if (j == 1) g.y -= inv_b;
+            if (j == 2) g.z -= inv_b;
+            if (j == 3) g.w -= inv_b;
+          }
+          store4<TDZ>(d, c, C, g.x, g.y, g.z, g.w);
+        }
+      }
+    }
+    return;
+  }
   float m = -INFINITY;
   for (int c = lane; c < C; c += 32) m = fmaxf(m, z[c]);
 #pragma unroll
@@ -33,7 +114,6 @@ __global__ void softmax_xent_kernel(const float* __restrict__ logits, int64_t ld
 #pragma unroll
   for (int o = 16; o > 0; o >>= 1) s += __shfl_xor_sync(0xffffffffu, s, o);
   const float lse = m + logf(s);
-  const int yi = y[(yoff ? *yoff : 0) + warp];
   if (lane == 0) row_loss[warp] = lse - z[yi];
   if (dZ) {
     TDZ* d = dZ + (int64_t)warp * ldz;

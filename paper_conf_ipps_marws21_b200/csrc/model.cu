@@ -868,18 +868,22 @@ static int forward_tc(hb_worker* w, const void* X, int64_t ldx, int64_t x_rows, 
       ep.ld0 = w->ldc;
       rc = gemm_tc_p(EPI_FWD_LOGITS, false, false, b, Ly.n_out, Ly.n_in, A, B, ep, s);
       if (rc) return rc;
-      Prof pr(HB_PROF_SOFTMAX, s);
-      softmax_xent_kernel<__nv_bfloat16><<<(b * 32 + 255) / 256, 256, 0, s>>>(
-          w->logits, w->ldc, y, d_off, b, Ly.n_out, want_grad ? static_cast<__nv_bfloat16*>(w->dZ[l]) : nullptr,
-          w->ld_dzL, w->row_loss, 1.0f / (float)b);
-      int nl = 1;
-      if (want_grad) {
+      {
+        // algorithmic bytes: fp32 logits read once, bf16 dZ written once, labels and row losses
+        Prof pr(HB_PROF_SOFTMAX, s);
+        softmax_xent_kernel<__nv_bfloat16><<<(b * 32 + 255) / 256, 256, 0, s>>>(
+            w->logits, w->ldc, y, d_off, b, Ly.n_out, want_grad ? static_cast<__nv_bfloat16*>(w->dZ[l]) : nullptr,
+            w->ld_dzL, w->row_loss, 1.0f / (float)b);
+        HB_CUDA_TRY(cudaGetLastError());
+        pr.done(1, 0.0, (double)b * Ly.n_out * (want_grad ? 6.0 : 4.0) + 8.0 * b);
+      }
+      if (want_grad) {  // bias-gradient partials of dZ_L (reduced by the head's dW GEMM)
+        Prof pr(HB_PROF_BIAS, s);
         colsum_partial_kernel<__nv_bfloat16><<<dim3((Ly.n_out + 63) / 64, (b + 127) / 128), dim3(64, 4), 0, s>>>(
             static_cast<const __nv_bfloat16*>(w->dZ[l]), w->ld_dzL, b, Ly.n_out, 128, w->bpart[l]);
-        nl = 2;
+        HB_CUDA_TRY(cudaGetLastError());
+        pr.done(1, 0.0, (double)b * Ly.n_out * 2.0 + 4.0 * ((b + 127) / 128) * Ly.n_out);
       }
-      HB_CUDA_TRY(cudaGetLastError());
-      pr.done(nl, 0.0, (double)b * Ly.n_out * 8.0 + 8.0 * b);
     }
   }
   return HB_OK;

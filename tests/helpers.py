@@ -51,6 +51,10 @@ def dataset(kind: str, N: int, d: int | None = None, seed: int = 0):
     if kind == "realsim":
         csr, y = sparse_like(N, d or 20958, 51.5, 0.31, False, seed=seed)
         return csr_to_dense(csr, d or 20958), y
+    if kind == "delicious":  # 500 binary features, one of 983 Zipf-distributed labels
+        from synth import delicious_like
+        csr, y = delicious_like(N, seed=seed)
+        return csr_to_dense(csr, 500), y
     if kind == "gauss":  # generic dense inputs for odd shapes
         rng = np.random.default_rng(seed)
         X = bf16_round(rng.standard_normal((N, d)))

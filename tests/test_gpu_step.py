@@ -154,6 +154,15 @@ def test_many_classes_uses_warp_shuffle_softmax(prec):
     assert abs(loss - l_ref) / l_ref <= TOL[prec]
 
 
+@pytest.mark.parametrize("prec", ["bf16", "fp32"])
+def test_delicious_shaped_983_class_head(prec):
+    # the paper's delicious shape (983 labels) as a single-label softmax head:
+    # logits GEMM + the standalone warp-per-row softmax-xent kernel (C > 16), ragged batch
+    e, le, errs = grads_case([500, 256, 983], "delicious", 300, prec)
+    assert e <= TOL[prec], errs
+    assert le <= TOL[prec]
+
+
 def test_batch_equal_to_max_batch_and_ragged_tiles():
     # b = max_batch with a ragged last row tile (b % 128 != 0) and ragged widths
     e, le, errs = grads_case([100, 136, 72, 3], "gauss", 1000, "bf16", d=100)
