@@ -61,7 +61,8 @@ struct TcCfg {
   static constexpr int OUT_BYTES = TmaOut<BN, EPI>::BYTES;
   static constexpr int STAGES_RAW = (192 * 1024 - OUT_BYTES) / STAGE_BYTES;
   static constexpr int STAGES = STAGES_RAW > 8 ? 8 : STAGES_RAW;
-  static constexpr int TMEM_COLS = 2 * BN < 32 ? 32 : 2 * BN;          // two accumulators (double buffer)
+  // two accumulators (double buffer); TMEM is allocated in powers of two >= 32 columns
+  static constexpr int TMEM_COLS = 2 * BN <= 32 ? 32 : 2 * BN <= 64 ? 64 : 2 * BN <= 128 ? 128 : 2 * BN <= 256 ? 256 : 512;
   static constexpr int SMEM_BYTES = STAGES * STAGE_BYTES + OUT_BYTES + 1024 /*align*/ + 256 /*barriers*/;
 };
 
