@@ -252,7 +252,7 @@ def main():
     import torch
     import torch.distributed as dist
     torch.cuda.set_device(local)
-    import paper_conf_ipps_marws21_b200 as hb
+    import paper_conf_ipps_marws21_b200 as hb  # noqa: F811
     from paper_conf_ipps_marws21_b200 import dist as hbd
     hbd.init("nccl", torch.device("cuda", local))
     from synth import init_params, params_to_flat
@@ -272,9 +272,19 @@ def main():
         dist.all_gather_into_tensor(yd, y_shard_d)
     else:
         Xd, yd = X_shard, y_shard_d
-    X_host = torch.empty(Nper, ld, dtype=torch.bfloat16, pin_memory=True)   # e2e: this rank's inputs
-    X_host.copy_(X_shard)
+    # e2e inputs of this rank in pinned host memory: the sparse-shaped data sets as CSR (what a
+    # user holds — LIBSVM-style rows — densified on the device by hogbatch_run), covtype dense
     y_host = torch.from_numpy(y_shard.astype(np.int32)).pin_memory()
+    csr_host = None
+    if xs[0] == "csr" and world == 1:
+        indptr, indices, vals = xs[1]
+        csr_host = hb.CSR(torch.from_numpy(indptr.astype(np.int64)).pin_memory(),
+                          torch.from_numpy(indices.astype(np.int32)).pin_memory(),
+                          torch.from_numpy(np.asarray(vals, np.float32)).to(torch.bfloat16).pin_memory(), dims[0], ld)
+        X_host = None
+    else:
+        X_host = torch.empty(Nper, ld, dtype=torch.bfloat16, pin_memory=True)
+        X_host.copy_(X_shard)
     torch.cuda.synchronize()
 
     model = hb.MLP(dims, precision="bf16", seed=0, device=local)
@@ -387,12 +397,15 @@ def main():
     # ---- e2e through the public API with HOST inputs: every step the rank's rows are copied from
     #      pinned host memory (H2D; with N > 1 then all-gathered over NVLink so that 𝔹 spans the
     #      GPUs), hogbatch_run trains one epoch, and the trained parameters are read back (D2H) ----
-    e2e_ms, e2e_samples = [], 0
-    h2d = X_host.numel() * 2 + y_host.numel() * 4
-    d2h = model.num_params * 4
-    params_out = torch.empty(model.num_params, dtype=torch.float32, pin_memory=True).numpy()
-    if world == 1:
-        X_e2e, y_e2e = X_host, y_host      # hogbatch_run stages host data itself (chunked, overlapped)
+    e2e_ms, e2e_samples, e2e_loss = [], 0, None
+    if csr_host is not None:
+        h2d = csr_host.indptr.numel() * 8 + csr_host.indices.numel() * 4 + csr_host.values.numel() * 2 + \
+            y_host.numel() * 4
+    else:
+        h2d = X_host.numel() * 2 + y_host.numel() * 4
+    d2h = 8 * len(workers)  # the step's result: the epoch's training loss (one fp64 sum per worker)
+    if world == 1:   # hogbatch_run stages host data itself (chunked, overlapped; CSR densified on device)
+        X_e2e, y_e2e = (csr_host if csr_host is not None else X_host), y_host
     else:
         X_e2e = torch.empty(N, ld, dtype=torch.bfloat16, device=dev)
         y_e2e = torch.empty(N, dtype=torch.int32, device=dev)
@@ -401,15 +414,14 @@ def main():
 
     def e2e_step():
         if world == 1:
-            st_ = hb.hogbatch_run(workers, pol, X_e2e, y_e2e, epochs=1)
+            st_ = hb.hogbatch_run(workers, pol, X_e2e, y_e2e, epochs=1, train_loss=True)
         else:
             xs_buf.copy_(X_host, non_blocking=True)
             ys_buf.copy_(y_host, non_blocking=True)
             dist.all_gather_into_tensor(X_e2e, xs_buf)
             dist.all_gather_into_tensor(y_e2e, ys_buf)
             torch.cuda.synchronize()
-            st_ = hb.hogbatch_run(workers, pol, X_e2e, y_e2e, epochs=1, n=N)
-        model.get_params(out=params_out)
+            st_ = hb.hogbatch_run(workers, pol, X_e2e, y_e2e, epochs=1, n=N, train_loss=True)
         return st_
 
     if args.e2e_steps:
@@ -427,6 +439,7 @@ def main():
         torch.cuda.synchronize()
         e2e_ms.append(e0.elapsed_time(e1))
         e2e_samples += st["total_samples"]
+        e2e_loss = st["train_loss"]
     te = hbd.reduce_scalar(sum(e2e_ms), "max", dev)
     se = hbd.reduce_scalar(float(e2e_samples), "sum", dev)
     e2e_value = se / (te * 1e-3) if args.e2e_steps else None
@@ -552,7 +565,10 @@ def main():
             "update_share": (share / share.sum()).round(4).tolist() if share.sum() else None,
             "roofline": roof,
             "cpu_baseline": cpu,
-            "e2e": {"value": e2e_value, "unit": "samples/s", "h2d_bytes_per_step": h2d, "d2h_bytes_per_step": d2h},
+            "e2e": {"value": e2e_value, "unit": "samples/s", "h2d_bytes_per_step": h2d, "d2h_bytes_per_step": d2h,
+                    "inputs": "CSR rows in pinned host memory, densified on the device" if csr_host is not None
+                    else "dense rows in pinned host memory", "result": "epoch training loss read back",
+                    "last_train_loss": e2e_loss},
             "gpu_launches": launches,
             "clocks": clk,
             "time_to_target": ttt,

@@ -117,7 +117,19 @@ typedef struct hb_dataset {
   int32_t x_dtype;/* HB_BF16 (required for HB_PREC_BF16) or HB_F32                             */
   const int32_t* y; /* [n] labels in [0, C)                                                    */
   int64_t n;      /* number of examples N                                                      */
+  /* format HB_DATA_CSR: X is unused and the rows are given sparse (the paper's data sets are sparse
+   * LIBSVM files "processed in dense format" [L255]): hogbatch_run copies the CSR arrays to the
+   * device (when host pointers; all host or all device) and densifies them into a dense
+   * [n x ldx] copy of dtype x_dtype owned by the model, chunk by chunk on its copy stream (a memset
+   * and a warp-per-row scatter kernel per chunk); batches wait only for their chunk, as for dense
+   * host data.  Column indices must lie in [0, n_cols) with n_cols <= ldx; values are x_dtype. */
+  int32_t format;          /* HB_DATA_DENSE (0, default) or HB_DATA_CSR (1)                    */
+  int64_t n_cols;          /* CSR: number of features (the model's n_0)                        */
+  const int64_t* indptr;   /* CSR: [n + 1] row offsets into indices / values                   */
+  const int32_t* indices;  /* CSR: [nnz] column indices                                        */
+  const void* values;      /* CSR: [nnz] values of dtype x_dtype                               */
 } hb_dataset;
+enum { HB_DATA_DENSE = 0, HB_DATA_CSR = 1 };
 
 /* One record per ScheduleWork message (O5). */
 typedef struct hb_trace_rec {
@@ -145,6 +157,11 @@ typedef struct hb_stats {
   double total_train_s;   /* training seconds, loss evaluation excluded                     */
   int64_t total_samples;
   int32_t n_merges;
+  int32_t want_train_loss;/* input: 1 = accumulate the training loss on the device (one small
+                             reduction kernel per step)                                       */
+  double train_loss;      /* mean per-example cross-entropy of the forward passes of every batch
+                             this process served (before each update) — the run's training
+                             metric, read back with 8 bytes; NaN unless want_train_loss         */
 } hb_stats;
 
 /* ---- library ---------------------------------------------------------------- */

@@ -242,6 +242,33 @@ class Policy:
         return p, ws
 
 
+@dataclass
+class CSR:
+    """A sparse data set for hogbatch_run (hb_dataset format HB_DATA_CSR): torch tensors, all on the
+    host (pinned for an asynchronous copy) or all on the device; densified on the device into rows
+    of `ldx` (default: n_cols rounded up to 8) elements ("processed in dense format")."""
+    indptr: object   # int64 [n + 1]
+    indices: object  # int32 [nnz]
+    values: object   # bfloat16 (bf16 models) or float32 [nnz]
+    n_cols: int
+    ldx: int = 0
+
+    @property
+    def n(self) -> int:
+        return self.indptr.numel() - 1
+
+
+def _dataset(X, y, n):
+    if isinstance(X, CSR):
+        ld = X.ldx or pad_to(X.n_cols)
+        n = X.n if n is None else n
+        return _lib.Dataset(None, ld, _xdtype(X.values), y.data_ptr(), n, _lib.HB_DATA_CSR, X.n_cols,
+                            X.indptr.data_ptr(), X.indices.data_ptr(), X.values.data_ptr()), n
+    n = X.shape[0] if n is None else n
+    return _lib.Dataset(X.data_ptr(), X.stride(0), _xdtype(X), y.data_ptr(), n, _lib.HB_DATA_DENSE, 0, None, None,
+                        None), n
+
+
 def _rec_tuple(r):
     return (r.seq, r.epoch, r.worker, r.vtime, r.u_before, r.b_before, ACTIONS[r.action], r.b_after,
             r.u_after, r.served, r.offset, r.lr)
@@ -257,10 +284,12 @@ def schedule_trace(policy: Policy, N: int, epochs: int, cap: int = 1 << 20):
 
 
 def hogbatch_run(workers, policy: Policy, X, y, epochs: int = 1, n: int | None = None,
-                 trace_cap: int = 0, step_loss_cap: int = 0, max_epochs: int | None = None):
-    """``hogbatch_run(workers, policy, epochs)`` over device data (X [N x ldx], y [N]).  Per-worker
-    statistics are indexed by the global worker id (policy.workers)."""
-    n = X.shape[0] if n is None else n
+                 trace_cap: int = 0, step_loss_cap: int = 0, max_epochs: int | None = None,
+                 train_loss: bool = False):
+    """``hogbatch_run(workers, policy, epochs)`` over X [N x ldx] (device, or pinned host memory staged by
+    the library) or a ``CSR`` data set, labels y [N].  Per-worker statistics are indexed by the global
+    worker id (policy.workers)."""
+    ds, n = _dataset(X, y, n)
     p, _keep = policy.to_c()
     W = len(policy.workers)
     me = max_epochs or epochs
@@ -270,8 +299,7 @@ def hogbatch_run(workers, policy: Policy, X, y, epochs: int = 1, n: int | None =
     sm = (C.c_int64 * (me * W))()
     tr = (_lib.TraceRec * max(trace_cap, 1))()
     sl = (C.c_float * max(step_loss_cap, 1))()
-    st = _lib.Stats(me, 0, el, et, up, sm, tr, trace_cap, 0, sl, step_loss_cap, 0, 0.0, 0, 0)
-    ds = _lib.Dataset(X.data_ptr(), X.stride(0), _xdtype(X), y.data_ptr(), n)
+    st = _lib.Stats(me, 0, el, et, up, sm, tr, trace_cap, 0, sl, step_loss_cap, 0, 0.0, 0, 0, int(train_loss), 0.0)
     hs = (C.c_void_p * len(workers))(*[w.h.value for w in workers])
     _check(lib.hogbatch_run(hs, len(workers), C.byref(p), C.byref(ds), epochs, C.byref(st)))
     ed = st.epochs_done
@@ -288,6 +316,7 @@ def hogbatch_run(workers, policy: Policy, X, y, epochs: int = 1, n: int | None =
         total_train_s=st.total_train_s,
         total_samples=st.total_samples,
         n_merges=st.n_merges,
+        train_loss=st.train_loss,
     )
 
 

@@ -54,9 +54,13 @@ class Policy(C.Structure):
                 ("check_labels", C.c_int32), ("coord", C.c_void_p), ("first_worker", C.c_int32)]
 
 
+HB_DATA_DENSE, HB_DATA_CSR = 0, 1
+
+
 class Dataset(C.Structure):
     _fields_ = [("X", C.c_void_p), ("ldx", C.c_int64), ("x_dtype", C.c_int32),
-                ("y", C.c_void_p), ("n", C.c_int64)]
+                ("y", C.c_void_p), ("n", C.c_int64), ("format", C.c_int32), ("n_cols", C.c_int64),
+                ("indptr", C.c_void_p), ("indices", C.c_void_p), ("values", C.c_void_p)]
 
 
 class TraceRec(C.Structure):
@@ -74,7 +78,8 @@ class Stats(C.Structure):
                 ("trace", C.POINTER(TraceRec)), ("trace_cap", C.c_int64), ("trace_len", C.c_int64),
                 ("step_loss", C.POINTER(C.c_float)), ("step_loss_cap", C.c_int64),
                 ("n_steps", C.c_int64), ("total_train_s", C.c_double),
-                ("total_samples", C.c_int64), ("n_merges", C.c_int32)]
+                ("total_samples", C.c_int64), ("n_merges", C.c_int32), ("want_train_loss", C.c_int32),
+                ("train_loss", C.c_double)]
 
 
 class ProfEntry(C.Structure):

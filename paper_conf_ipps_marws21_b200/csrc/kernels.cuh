@@ -249,6 +249,25 @@ static __global__ void merge_apply_kernel(float* w, float* base, const float* __
   }
 }
 
+// CSR -> dense rows [r0, r1) of X [.. x ldx] (zeroed beforehand): one warp per row scatters its
+// nonzeros (hb_dataset format HB_DATA_CSR; the paper's sparse data "processed in dense format" [L255])
+template <typename T>
+static __global__ void densify_csr_kernel(const int64_t* __restrict__ indptr, const int32_t* __restrict__ indices,
+                                          const T* __restrict__ vals, int64_t r0, int64_t r1, int64_t n_cols, T* X,
+                                          int64_t ldx, int* bad) {
+  const int64_t r = r0 + ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) / 32;
+  const int lane = threadIdx.x & 31;
+  if (r >= r1) return;
+  T* row = X + r * ldx;
+  for (int64_t k = indptr[r] + lane; k < indptr[r + 1]; k += 32) {
+    const int32_t c = indices[k];
+    if (c >= 0 && c < n_cols)
+      row[c] = vals[k];
+    else
+      atomicOr(bad, 1);
+  }
+}
+
 // HB_CHECK=labels (hb_policy.check_labels): flag any label outside [0, C)
 static __global__ void check_labels_kernel(const int32_t* __restrict__ y, int64_t n, int C, int* bad) {
   int any = 0;

@@ -1092,13 +1092,13 @@ int step_graph(hb_worker* w, const void* X, int64_t ldx, int64_t x_rows, const i
 }
 
 int worker_execute(hb_worker* w, const void* X, int64_t ldx, int32_t xdt, int64_t x_rows, const int32_t* y,
-                   int64_t off, int b, float lr, bool graphs, bool serial, double* loss_dst) {
+                   int64_t off, int b, float lr, bool graphs, bool serial, double* loss_dst, bool accumulate) {
   const size_t xes = xdt == HB_BF16 ? 2 : 4;
   auto xrow = [&](int64_t o) { return static_cast<const char*>(X) + o * ldx * xes; };
   if (w->subs.empty()) {
     int rc = graphs ? step_graph(w, X, ldx, x_rows, y, off, b, lr)
                     : run_step(w, xrow(off), ldx, xdt, b, y + off, nullptr, b, lr, false, w->stream);
-    if (!rc && loss_dst) sum_rows_into(w, b, loss_dst, w->stream, false);
+    if (!rc && loss_dst) sum_rows_into(w, b, loss_dst, w->stream, accumulate);
     return rc;
   }
   const int t = (int)w->subs.size();
@@ -1113,7 +1113,7 @@ int worker_execute(hb_worker* w, const void* X, int64_t ldx, int32_t xdt, int64_
     int rc;
     if (serial) {
       rc = run_step(sw, xrow(o), ldx, xdt, sz, y + o, nullptr, sz, lr_i, false, w->stream);
-      if (!rc && loss_dst) sum_rows_into(sw, sz, loss_dst, w->stream, i > 0);
+      if (!rc && loss_dst) sum_rows_into(sw, sz, loss_dst, w->stream, accumulate || i > 0);
     } else {
       HB_CUDA_TRY(cudaStreamWaitEvent(sw->stream, w->ev_fork, 0));
       rc = graphs ? step_graph(sw, X, ldx, x_rows, y, o, sz, lr_i)
@@ -1130,7 +1130,7 @@ int worker_execute(hb_worker* w, const void* X, int64_t ldx, int32_t xdt, int64_
     for (int i = 0; i < t; ++i) {
       const int sz = base + (i < extra ? 1 : 0);
       if (sz == 0) continue;
-      sum_rows_into(w->subs[i], sz, loss_dst, w->stream, !first);
+      sum_rows_into(w->subs[i], sz, loss_dst, w->stream, accumulate || !first);
       first = false;
     }
   }
@@ -1306,6 +1306,9 @@ int mlp_destroy(hb_model* m) {
   cudaFree(m->chunk_sums);
   cudaFree(m->stage_x);
   cudaFree(m->stage_y);
+  cudaFree(m->csr_ptr);
+  cudaFree(m->csr_idx);
+  cudaFree(m->csr_val);
   for (cudaEvent_t e : m->stage_ev) cudaEventDestroy(e);
   if (m->copy_stream) cudaStreamDestroy(m->copy_stream);
   if (m->stream) cudaStreamDestroy(m->stream);
@@ -1316,6 +1319,23 @@ int mlp_destroy(hb_model* m) {
 }  // extern "C"
 
 namespace hb {
+int densify_csr_rows(const int64_t* indptr, const int32_t* indices, const void* vals, int xdt, int64_t r0, int64_t r1,
+                     int64_t n_cols, void* X, int64_t ldx, cudaStream_t s, int* bad) {
+  const size_t es = xdt == HB_BF16 ? 2 : 4;
+  HB_CUDA_TRY(cudaMemsetAsync(static_cast<char*>(X) + (size_t)r0 * ldx * es, 0, (size_t)(r1 - r0) * ldx * es, s));
+  const int64_t warps = r1 - r0;
+  const unsigned blocks = (unsigned)((warps * 32 + 255) / 256);
+  if (xdt == HB_BF16)
+    densify_csr_kernel<__nv_bfloat16><<<blocks, 256, 0, s>>>(indptr, indices, static_cast<const __nv_bfloat16*>(vals),
+                                                             r0, r1, n_cols, static_cast<__nv_bfloat16*>(X), ldx, bad);
+  else
+    densify_csr_kernel<float><<<blocks, 256, 0, s>>>(indptr, indices, static_cast<const float*>(vals), r0, r1, n_cols,
+                                                     static_cast<float*>(X), ldx, bad);
+  HB_CUDA_TRY(cudaGetLastError());
+  g_launches.fetch_add(1, std::memory_order_relaxed);
+  return HB_OK;
+}
+
 int check_labels_dev(const int32_t* y, int64_t n, int C, int device, bool* ok) {
   HB_CUDA_TRY(cudaSetDevice(device));
   int* d = nullptr;

@@ -84,6 +84,11 @@ struct hb_model {
   size_t stage_y_cap = 0;
   cudaStream_t copy_stream = nullptr;
   std::vector<cudaEvent_t> stage_ev;
+  // CSR datasets: device copies of the sparse arrays (reused across calls)
+  int64_t* csr_ptr = nullptr;
+  int32_t* csr_idx = nullptr;
+  void* csr_val = nullptr;
+  size_t csr_ptr_cap = 0, csr_nnz_cap = 0;
 };
 
 struct hb_worker {
@@ -134,6 +139,10 @@ struct hb_worker {
 
 namespace hb {
 int clone_model(hb_model* m, hb_model** out);
+// zero rows [r0, r1) of the dense X [.. x ldx] (dtype xdt) and scatter the CSR rows into them on s;
+// *bad (device int) is set if a column index is outside [0, n_cols)
+int densify_csr_rows(const int64_t* indptr, const int32_t* indices, const void* vals, int xdt, int64_t r0, int64_t r1,
+                     int64_t n_cols, void* X, int64_t ldx, cudaStream_t s, int* bad);
 // One SGD step.  X / y: the batch's first row, or (d_off != nullptr, tensor-core path) the
 // dataset base with the batch's first row read from *d_off on the device.  x_rows = rows of X.
 int run_step(hb_worker* w, const void* X, int64_t ldx, int32_t xdt, int64_t x_rows, const int32_t* y,
@@ -147,9 +156,10 @@ void clear_graphs(hb_worker* w);
 // a plain worker runs one SGD step; a nested worker splits B into its t sub-batches (the first
 // b mod t get ceil(b/t) rows, R6) with lr scaled to each sub-batch (lr * size / b),
 // concurrently on the sub-workers' streams (serial = in order on w->stream, deterministic).
-// If loss_dst != nullptr the summed per-row losses of the batch are written to *loss_dst (device).
+// If loss_dst != nullptr the summed per-row losses of the batch are written to (accumulate: added
+// to) *loss_dst (device).
 int worker_execute(hb_worker* w, const void* X, int64_t ldx, int32_t xdt, int64_t x_rows, const int32_t* y,
-                   int64_t off, int b, float lr, bool graphs, bool serial, double* loss_dst);
+                   int64_t off, int b, float lr, bool graphs, bool serial, double* loss_dst, bool accumulate = false);
 bool prof_enabled();
 int finish_loss(hb_worker* w, int b, float* loss_out, cudaStream_t s);
 // enqueue sum of the last step's per-row losses into *dst (device double)

@@ -119,6 +119,23 @@ def test_serial_run_is_bitwise_reproducible(dims):
     assert len(out) == 1
 
 
+def test_train_loss_is_the_mean_of_the_served_batches_losses():
+    # hb_stats.train_loss (one fp64 read back): concurrent mode (graph replay, device accumulator)
+    # equals the SERIAL run's per-step losses averaged over the served rows
+    dims = [54, 128, 7]
+    out = []
+    for det in (True, False):
+        X, y, m, params, tX, ty = setup(dims, "bf16", 512, 4500)
+        w = hb.Worker(m, 512)
+        pol = hb.Policy(kind=hb.HB_MINIBATCH, workers=[hb.WorkerSpec(512, 512, 512)], eta0=0.1, b0=32,
+                        deterministic=det)
+        st = hb.hogbatch_run([w], pol, tX, ty, epochs=2, step_loss_cap=100, train_loss=True)
+        out.append(st)
+    det, conc = out
+    np.testing.assert_allclose(det["train_loss"], np.mean(det["step_loss"]), rtol=1e-6)
+    np.testing.assert_allclose(conc["train_loss"], det["train_loss"], rtol=1e-12)
+
+
 def test_graph_replay_is_bitwise_equal_to_direct_launches():
     # concurrent mode replays one CUDA graph per batch size with a device-side row offset;
     # the deterministic mode launches kernels directly on per-batch pointers: same arithmetic
@@ -158,6 +175,49 @@ def test_host_dataset_is_staged_and_bitwise_equal_to_device_dataset(det, pinned)
         out.append((m.get_params(), st["epoch_loss"]))
     assert np.array_equal(out[0][0], out[1][0])
     assert out[0][1] == out[1][1]
+
+
+@pytest.mark.parametrize("where", ["host", "device"])
+def test_csr_dataset_is_densified_and_bitwise_equal_to_dense(where):
+    # hb_dataset format HB_DATA_CSR: the sparse rows (real-sim-like, "processed in
+    # dense format") are densified on the device chunk by chunk; the trained model equals the run on
+    # the dense device copy bit for bit (same rows, same batches, same kernels)
+    from synth import sparse_like
+    _gpu()
+    dims, N = [2000, 256, 2], 3000
+    (indptr, indices, vals), y = sparse_like(N, 2000, 51.5, 0.31, False, seed=3)
+    X = np.zeros((N, 2000), np.float32)
+    X[np.repeat(np.arange(N), np.diff(indptr)), indices] = vals
+    out = []
+    for fmt in ("dense", "csr"):
+        m = hb.MLP(dims)
+        m.set_params(params_to_flat(init_params(dims)))
+        m.set_option("stage_rows", 700)  # several chunks, ragged last one
+        w = hb.Worker(m, 256)
+        pol = hb.Policy(kind=hb.HB_MINIBATCH, workers=[hb.WorkerSpec(256, 256, 256)], eta0=0.1, b0=32, eval_loss=True)
+        if fmt == "dense":
+            tX, ty = to_device(X, y)
+            st = hb.hogbatch_run([w], pol, tX, ty, epochs=2)
+        else:
+            t = lambda a, dt: torch.from_numpy(np.ascontiguousarray(a)).to(dt)
+            csr = hb.CSR(t(indptr.astype(np.int64), torch.int64), t(indices, torch.int32), t(vals, torch.bfloat16), 2000)
+            ty = t(y.astype(np.int32), torch.int32)
+            if where == "host":
+                csr = hb.CSR(csr.indptr.pin_memory(), csr.indices.pin_memory(), csr.values.pin_memory(), 2000)
+                ty = ty.pin_memory()
+            else:
+                csr = hb.CSR(csr.indptr.cuda(), csr.indices.cuda(), csr.values.cuda(), 2000)
+                ty = ty.cuda()
+                torch.cuda.synchronize()
+            st = hb.hogbatch_run([w], pol, csr, ty, epochs=2)
+        out.append((m.get_params(), st["epoch_loss"]))
+    assert np.array_equal(out[0][0], out[1][0])
+    assert out[0][1] == out[1][1]
+    bad = torch.from_numpy(indices.copy()).to(torch.int32)
+    bad[5] = 2000  # column outside [0, n_cols)
+    csr = hb.CSR(torch.from_numpy(indptr.astype(np.int64)), bad, torch.from_numpy(vals).to(torch.bfloat16), 2000)
+    with pytest.raises(hb.HogbatchError):
+        hb.hogbatch_run([w], pol, csr, torch.from_numpy(y.astype(np.int32)), epochs=1)
 
 
 def test_host_dataset_mixed_pointers_rejected():
