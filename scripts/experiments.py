@@ -50,7 +50,9 @@ def main():
     ap.add_argument("--epochs", type=int, default=10)
     ap.add_argument("--eta-grid", default="0.001,0.01,0.1,1")
     ap.add_argument("--b0", type=int, default=32)
-    ap.add_argument("--out", default=os.path.join(ROOT, "profiles", "r01_experiments.json"))
+    ap.add_argument("--init-scale", type=float, default=1.0,
+                    help="W ~ N(0, (scale/sqrt(fan_in))^2) (R11: 1; 4 = the Glorot factor for sigmoid units)")
+    ap.add_argument("--out", default=os.path.join(ROOT, "profiles", "r02_experiments.json"))
     args = ap.parse_args()
 
     import torch
@@ -79,7 +81,7 @@ def main():
         yd = torch.from_numpy(y.astype(np.int32)).cuda()
         gen_s = time.time() - t0
         model = hb.MLP(dims, precision="bf16", seed=0)
-        p0 = params_to_flat(init_params(dims, seed=2))
+        p0 = params_to_flat(init_params(dims, seed=2, scale=args.init_scale))
         big = hb.Worker(model, 8192)
         small = hb.Worker(model, 2048)
         algos = {
@@ -108,6 +110,8 @@ def main():
         lmin = best(eta_star)
         target = 1.1 * lmin
         out = {"dims": dims, "N": N, "classes": C, "eta0": eta_star, "b0": args.b0, "epochs": args.epochs,
+               "init_scale": args.init_scale, "prior_loss": float(-(np.bincount(y, minlength=C) / N
+                                                                   * np.log(np.maximum(np.bincount(y, minlength=C) / N, 1e-300))).sum()),
                "min_loss": lmin, "target_loss": target, "data_gen_s": round(gen_s, 1),
                "grid_best_loss": {str(e): best(e) for e in etas}, "algorithms": {}}
         for a in algos:
