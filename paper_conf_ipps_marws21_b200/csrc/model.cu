@@ -1741,7 +1741,7 @@ static int bench_gemm_impl(int32_t kind, int32_t M, int32_t N, int32_t K, int32_
   cudaStream_t s;
   cudaStreamCreate(&s);
   EpiArgs ep{};
-    ep.no_pdl = !m->opt_pdl;
+    ep.no_pdl = 0;
   ep.M = M;
   ep.N = N;
   int epi;
