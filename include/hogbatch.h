@@ -208,11 +208,16 @@ int mlp_fused_path(const hb_model* m, int32_t batch, int32_t* cluster_size);
  *   HB_OPT_UPDATE           HB_UPDATE_HOGWILD (plain read-modify-write of the shared model, Hogwild
  *                           [L128, L170]; default) or HB_UPDATE_ATOMIC (the dW epilogue adds -lr*dW
  *                           with atomic adds: no concurrent update is lost)
+ *   HB_OPT_STEP_KERNEL_MAX_B steps of at most this many rows (and below the fused chain's threshold)
+ *                           run as ONE persistent launch: the step's 3L - 1 GEMMs as stages
+ *                           separated by grid barriers (narrow nets: widths <= 1024, C <= 16,
+ *                           L <= 8; plain workers); 0 = per-layer launches (default: measured
+ *                           slower on B200 — 86 vs 58 us per C2 step at b = 32)
  * Unknown key or out-of-range value -> HB_EINVAL. */
 enum {
   HB_OPT_FUSED_MIN_BATCH = 0, HB_OPT_ROWCHAIN = 1, HB_OPT_RC_CLUSTER = 2, HB_OPT_BWD_OVERLAP = 3,
   HB_OPT_HEAD_FUSE = 4, HB_OPT_DW_PAIR = 5, HB_OPT_PDL = 6, HB_OPT_GRAPHS = 7, HB_OPT_INFLIGHT = 8,
-  HB_OPT_STAGE_ROWS = 9, HB_OPT_UPDATE = 10
+  HB_OPT_STAGE_ROWS = 9, HB_OPT_UPDATE = 10, HB_OPT_STEP_KERNEL_MAX_B = 11
 };
 enum { HB_UPDATE_HOGWILD = 0, HB_UPDATE_ATOMIC = 1 };
 int mlp_set_option(hb_model* m, int32_t key, int64_t value);
@@ -324,7 +329,8 @@ enum {
   HB_PROF_BIAS = 5,       /* bias gradient + bias SGD                                   */
   HB_PROF_OTHER = 6,      /* loss reduction, shadow refresh, merge kernels              */
   HB_PROF_ROWCHAIN = 7,   /* fused per-row-block forward + softmax-xent + dX chain (narrow nets) */
-  HB_PROF_N = 8,
+  HB_PROF_STEPK = 8,      /* persistent small-batch step kernel (all GEMMs of a step in one launch) */
+  HB_PROF_N = 9,
   HB_PROF_LAYERS = 16     /* per-layer breakdown: entry HB_PROF_N + cls * HB_PROF_LAYERS + layer (0-based) */
 };
 typedef struct hb_prof_entry {

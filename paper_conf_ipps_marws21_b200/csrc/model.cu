@@ -21,6 +21,7 @@
 #include "model.h"
 #include "tc_gemm.cuh"
 #include "rowchain.cuh"
+#include "step_kernel.cuh"
 
 namespace hb {
 
@@ -367,9 +368,26 @@ static int prof_class(int epi) {
                                 : HB_PROF_WGRAD_GEMM;
 }
 
+// Planning mode of the persistent small-batch step (step_kernel.cuh): while g_plan is set, the
+// step's GEMMs are RECORDED (arguments + the layer they belong to) instead of launched, so the
+// persistent kernel runs exactly the GEMMs, operands and fused epilogues of the per-layer path.
+struct SkPlanEntry {
+  int epi;
+  bool a_mn, b_mn;
+  int M, N, K;
+  TcOp A, B;
+  EpiArgs ep;
+  int layer;
+};
+static thread_local std::vector<SkPlanEntry>* g_plan = nullptr;
+
 static int gemm_tc_p(int epi, bool a_mn, bool b_mn, int M, int N, int K, TcOp A, TcOp B, const EpiArgs& ep,
                      cudaStream_t s) {
   if (M <= 0 || N <= 0 || K <= 0) return HB_OK;
+  if (g_plan) {
+    g_plan->push_back(SkPlanEntry{epi, a_mn, b_mn, M, N, K, A, B, ep, g_prof_layer});
+    return HB_OK;
+  }
   Prof pr(prof_class(epi), s);
   int rc = gemm_tc(epi, a_mn, b_mn, M, N, K, A, B, ep, s);
   if (!rc) pr.done(1, 2.0 * M * N * (double)K, gemm_bytes(epi, M, N, K, 2.0, true));
@@ -569,6 +587,18 @@ static int64_t ld_dz(const hb_worker* w, int l) {
 static int act_dt(const hb_model* m) { return m->prec == HB_PREC_BF16 ? HB_BF16 : HB_F32; }
 static size_t act_size(const hb_model* m) { return m->prec == HB_PREC_BF16 ? 2 : 4; }
 
+// grid of a worker's persistent step kernel: fixed per worker (the stage barriers count launches of
+// one grid size), enough CTAs for the widest stage at max_batch, at most one per SM
+static int step_kernel_grid(const hb_model* m, int max_b) {
+  int mx = 1;
+  for (const Layer& Ly : m->layers) mx = std::max(mx, std::max(Ly.n_out, Ly.n_in));
+  const long t = (long)((max_b + TC_BM - 1) / TC_BM) * ((mx + 31) / 32) + (long)((mx + TC_BM - 1) / TC_BM) * ((mx + 31) / 32);
+  int nsm = 148, dev = 0;
+  cudaGetDevice(&dev);
+  cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, dev);
+  return (int)std::max<long>(1, std::min<long>(t, nsm > 0 ? nsm : 148));
+}
+
 static void free_worker_buffers(hb_worker* w) {
   for (void* p : w->H) cudaFree(p);
   for (void* p : w->S) cudaFree(p);
@@ -599,6 +629,8 @@ static void free_worker_buffers(hb_worker* w) {
   w->ws_l.clear();
   if (w->s2) cudaStreamDestroy(w->s2);
   w->s2 = nullptr;
+  cudaFree(w->sk_bar);
+  w->sk_bar = nullptr;
   cudaFree(w->logits);
   cudaFree(w->row_loss);
   cudaFree(w->dsum);
@@ -683,6 +715,12 @@ static int alloc_worker(hb_model* m, int max_b, cudaStream_t stream, bool own, h
       w->ws_l.push_back(p);
     }
     cudaEventCreateWithFlags(&w->ev_chain, cudaEventDisableTiming);
+  }
+  if (train && m->prec == HB_PREC_BF16) {  // persistent small-batch step: stage barriers + generation word
+    if (cudaMalloc(&w->sk_bar, (SK_MAX_S + 1) * sizeof(unsigned)) != cudaSuccess)
+      return fail_free(fail(HB_ENOMEM, "step-kernel barrier alloc"));
+    cudaMemset(w->sk_bar, 0, (SK_MAX_S + 1) * sizeof(unsigned));
+    w->sk_grid = step_kernel_grid(m, max_b);
   }
   if (cudaMalloc(&w->logits, (size_t)max_b * w->ldc * 4) != cudaSuccess ||
       cudaMalloc(&w->row_loss, (size_t)max_b * 4) != cudaSuccess ||
@@ -983,6 +1021,102 @@ static int run_step_rowchain(hb_worker* w, const RcCfg& c, const void* X, int64_
   return HB_OK;
 }
 
+static int step_gemms(hb_worker* w, const void* X, int64_t ldx, int64_t x_rows, const int32_t* y, const int* d_off,
+                      int b, float lr, bool grads_only, cudaStream_t s, bool overlap);
+
+// ---- persistent small-batch step (step_kernel.cuh) -------------------------------------------
+// Eligible: bf16 plain worker with its stage-barrier buffer, b <= HB_OPT_STEP_KERNEL_MAX_B, a
+// fused softmax-xent head (C <= 16, not fused with its dX), every width <= 1024, L <= 8 layers.
+static bool step_kernel_ok(const hb_worker* w, int b) {
+  const hb_model* m = w->m;
+  if (!w->sk_bar || m->opt_step_kernel_max_b <= 0 || b > m->opt_step_kernel_max_b) return false;
+  const int L = (int)m->layers.size();
+  if (L > SK_MAX_S / 2 || 3 * L - 1 > SK_MAX_G || m->layers.back().n_out > 16 || head_dx_fused(m)) return false;
+  for (const Layer& Ly : m->layers)
+    if (Ly.n_out > 1024 || Ly.n_in > 1024) return false;
+  return true;
+}
+
+static int run_step_persistent(hb_worker* w, const void* X, int64_t ldx, int64_t x_rows, const int32_t* y,
+                               const int* d_off, int b, float lr, bool grads_only, cudaStream_t s) {
+  hb_model* m = w->m;
+  const int L = (int)m->layers.size();
+  std::vector<SkPlanEntry> plan;
+  g_plan = &plan;
+  int rc = step_gemms(w, X, ldx, x_rows, y, d_off, b, lr, grads_only, s, false);
+  g_plan = nullptr;
+  if (rc) return rc;
+  if ((int)plan.size() > SK_MAX_G) return fail(HB_EUNSUPPORTED, "persistent step: too many GEMMs");
+  static SkParams P;  // ~15 KB: built on the host thread, copied into the launch's parameters
+  static std::mutex pmu;
+  std::lock_guard<std::mutex> g(pmu);
+  std::memset(&P, 0, sizeof(P));
+  double flops = 0.0, bytes = 0.0;
+  int nst = 0;
+  for (size_t k = 0; k < plan.size(); ++k) {
+    const SkPlanEntry& e = plan[k];
+    SkGemm& Q = P.g[k];
+    const int l = e.layer;
+    switch (e.epi) {
+      case EPI_FWD_SIG: Q.kind = SK_FWD; Q.stage = l; break;
+      case EPI_HEAD_XENT: Q.kind = SK_HEAD; Q.stage = L - 1; break;
+      case EPI_DGRAD_SIG: Q.kind = SK_DGRAD; Q.stage = 2 * L - 1 - l; break;
+      case EPI_WGRAD_SGD:
+      case EPI_WGRAD_STORE:
+        Q.kind = e.epi == EPI_WGRAD_SGD ? SK_WGRAD : SK_WGRAD_STORE;
+        Q.stage = std::min(2 * L - l, 2 * L - 1);
+        break;
+      default: return fail(HB_EUNSUPPORTED, "persistent step: unsupported epilogue");
+    }
+    const int bn = Q.kind == SK_HEAD ? 16 : 32;
+    const int64_t ar = e.A.rows ? e.A.rows : (e.a_mn ? e.K : e.M);
+    const int64_t br = e.B.rows ? e.B.rows : (e.b_mn ? e.K : e.N);
+    rc = e.a_mn ? make_map(&Q.ma, e.A.p, e.M, ar, e.A.ld * 2, 64, 64) : make_map(&Q.ma, e.A.p, e.K, ar, e.A.ld * 2, 64, TC_BM);
+    if (!rc) rc = e.b_mn ? make_map(&Q.mb, e.B.p, e.N, br, e.B.ld * 2, 64, 64) : make_map(&Q.mb, e.B.p, e.K, br, e.B.ld * 2, 64, bn);
+    if (rc) return rc;
+    Q.ep = e.ep;
+    Q.offA = e.A.off;
+    Q.offB = e.B.off;
+    Q.M = e.M;
+    Q.N = e.N;
+    Q.K = e.K;
+    Q.tiles_m = (e.M + TC_BM - 1) / TC_BM;
+    Q.tiles_n = (e.N + bn - 1) / bn;
+    nst = std::max(nst, Q.stage + 1);
+    flops += 2.0 * e.M * e.N * (double)e.K;
+    bytes += gemm_bytes(e.epi, e.M, e.N, e.K, 2.0, true);
+  }
+  P.ng = (int)plan.size();
+  P.nstages = nst;
+  P.bar = w->sk_bar;
+  P.dbg = g_rc_trace;
+  int dev = 0;
+  cudaGetDevice(&dev);
+  {
+    std::lock_guard<std::mutex> ga(g_attr_mu);
+    auto key = std::make_pair((const void*)step_kernel, dev);
+    if (!g_attr_done.count(key)) {
+      HB_CUDA_TRY(cudaFuncSetAttribute(step_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, SK_SMEM_BYTES));
+      g_attr_done.insert(key);
+    }
+  }
+  Prof pr(HB_PROF_STEPK, s);
+  cudaLaunchConfig_t cfg{};
+  cfg.gridDim = dim3(w->sk_grid, 1, 1);
+  cfg.blockDim = dim3(TC_THREADS);
+  cfg.dynamicSmemBytes = SK_SMEM_BYTES;
+  cfg.stream = s;
+  cudaLaunchAttribute attr[1];
+  attr[0].id = cudaLaunchAttributeCooperative;  // all CTAs co-resident (grid barriers)
+  attr[0].val.cooperative = 1;
+  cfg.attrs = attr;
+  cfg.numAttrs = 1;
+  HB_CUDA_TRY(cudaLaunchKernelEx(&cfg, step_kernel, P));
+  HB_CUDA_TRY(cudaGetLastError());
+  pr.done(1, flops, bytes);
+  return HB_OK;
+}
+
 // One SGD step of the bf16 tensor-core path: forward + fused head, then for l = L..1
 // dgrad (reads W_l before it is updated) and wgrad with the fused in-place SGD of W_l and b_l.
 // 3L - 1 kernel launches for C <= 16 (L fwd incl. head, L-1 dgrad, L wgrad).  Narrow nets take
@@ -990,16 +1124,25 @@ static int run_step_rowchain(hb_worker* w, const RcCfg& c, const void* X, int64_
 static int run_step_tc(hb_worker* w, const void* X, int64_t ldx, int64_t x_rows, const int32_t* y, const int* d_off,
                        int b, float lr, bool grads_only, cudaStream_t s) {
   hb_model* m = w->m;
-  const int L = (int)m->layers.size();
   {
     const RcCfg c = rowchain_cfg(m, b);
     if (c.ok && !w->sdw.empty()) return run_step_rowchain(w, c, X, ldx, x_rows, y, d_off, b, lr, grads_only, s);
   }
+  if (step_kernel_ok(w, b)) return run_step_persistent(w, X, ldx, x_rows, y, d_off, b, lr, grads_only, s);
+  return step_gemms(w, X, ldx, x_rows, y, d_off, b, lr, grads_only, s, m->opt_bwd_overlap && w->s2);
+}
+
+// The 3L - 1 tcgen05 GEMMs of one step in dependency order: forward + fused head, then for
+// l = L..1 the dX GEMM (reads W_l) and the dW GEMM with the fused SGD of W_l.
+static int step_gemms(hb_worker* w, const void* X, int64_t ldx, int64_t x_rows, const int32_t* y, const int* d_off,
+                      int b, float lr, bool grads_only, cudaStream_t s, bool overlap) {
+  hb_model* m = w->m;
+  const int L = (int)m->layers.size();
   int rc = forward_tc(w, X, ldx, x_rows, y, d_off, b, true, s);
   if (rc) return rc;
   // dW_l only has to follow dX_l (the last reader of W_l): it runs on the worker's second stream,
-  // overlapping dX_{l-1} (HB_NO_BWD_OVERLAP=1 keeps everything on one stream)
-  cudaStream_t s2 = m->opt_bwd_overlap && w->s2 ? w->s2 : s;
+  // overlapping dX_{l-1} (HB_OPT_BWD_OVERLAP = 0 keeps everything on one stream)
+  cudaStream_t s2 = overlap ? w->s2 : s;
   for (int l = L - 1; l >= 0; --l) {
     const Layer& Ly = m->layers[l];
     TcOp dZl{w->dZ[l], ld_dz(w, l), b, nullptr};
@@ -1367,6 +1510,7 @@ int clone_model(hb_model* m, hb_model** out) {
   r->opt_inflight = m->opt_inflight;
   r->opt_stage_rows = m->opt_stage_rows;
   r->opt_update = m->opt_update;
+  r->opt_step_kernel_max_b = m->opt_step_kernel_max_b;
   if (cudaDeviceSynchronize() != cudaSuccess ||
       cudaMemcpy(r->master, m->master, m->total * 4, cudaMemcpyDeviceToDevice) != cudaSuccess ||
       (m->shadow && cudaMemcpy(r->shadow, m->shadow, m->total * 2, cudaMemcpyDeviceToDevice) != cudaSuccess)) {
@@ -1490,6 +1634,10 @@ int mlp_set_option(hb_model* m, int32_t key, int64_t v) {
       HB_CHECK_ARG(v == HB_UPDATE_HOGWILD || v == HB_UPDATE_ATOMIC, "update must be HB_UPDATE_HOGWILD or _ATOMIC");
       m->opt_update = (int)v;
       return HB_OK;
+    case HB_OPT_STEP_KERNEL_MAX_B:
+      HB_CHECK_ARG(v >= 0 && v <= (1 << 20), "step-kernel max batch must be >= 0");
+      m->opt_step_kernel_max_b = (int)v;
+      return HB_OK;
     default: return fail(HB_EINVAL, "unknown option key");
   }
 }
@@ -1508,6 +1656,7 @@ int mlp_get_option(const hb_model* m, int32_t key, int64_t* v) {
     case HB_OPT_INFLIGHT: *v = m->opt_inflight; return HB_OK;
     case HB_OPT_STAGE_ROWS: *v = m->opt_stage_rows; return HB_OK;
     case HB_OPT_UPDATE: *v = m->opt_update; return HB_OK;
+    case HB_OPT_STEP_KERNEL_MAX_B: *v = m->opt_step_kernel_max_b; return HB_OK;
     default: return fail(HB_EINVAL, "unknown option key");
   }
 }
@@ -1638,6 +1787,8 @@ int mlp_worker_create_nested(hb_model* m, int32_t max_batch, int32_t t, void* cu
       mlp_worker_destroy(w);
       return rc;
     }
+    cudaFree(sw->sk_bar);  // t concurrent sub-steps: per-layer launches, no cooperative grids
+    sw->sk_bar = nullptr;
     w->subs.push_back(sw);
     cudaEvent_t e;
     cudaEventCreateWithFlags(&e, cudaEventDisableTiming);

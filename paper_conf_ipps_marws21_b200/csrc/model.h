@@ -65,6 +65,8 @@ struct hb_model {
   int opt_inflight = 0;             // HB_OPT_INFLIGHT: steps a worker may enqueue ahead (0 = auto)
   int64_t opt_stage_rows = 0;       // HB_OPT_STAGE_ROWS: host-dataset staging chunk rows (0 = auto)
   int opt_update = 0;               // HB_OPT_UPDATE: HB_UPDATE_HOGWILD or HB_UPDATE_ATOMIC
+  int opt_step_kernel_max_b = 0;    // HB_OPT_STEP_KERNEL_MAX_B: persistent one-launch step up to this b
+                                    // (off by default: measured slower than the per-layer launches)
   std::vector<hb::Layer> layers;
   size_t total = 0;                 // floats in the flat parameter buffer (incl. padding)
   float* master = nullptr;          // fp32 master weights + biases (the shared global model)
@@ -100,6 +102,8 @@ struct hb_worker {
   bool own_stream = false;
   std::vector<void*> H, S, dZ;  // per-layer activations, sigma' stash, output gradients
   int ld_dzL = 0;               // row stride of dZ_L (32 with the split-precision head, R24)
+  unsigned* sk_bar = nullptr;   // persistent small-batch step: stage arrival counters + generation
+  int sk_grid = 0;              // its fixed grid size
   bool hilo = false;            // dZ_L stored as bf16 hi / lo planes (C <= 16, bf16 model)
   float* logits = nullptr;      // [max_b x ldc] fp32
   int ldc = 0;

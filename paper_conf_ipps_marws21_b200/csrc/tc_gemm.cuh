@@ -166,195 +166,58 @@ __device__ __forceinline__ void stage16(uint8_t* sout, int o, int rl, int c, con
   *reinterpret_cast<uint4*>(row + (((j0 + 1) ^ (rl & 7)) << 4)) = make_uint4(p[4], p[5], p[6], p[7]);
 }
 
-template <int BN, bool A_MN, bool B_MN, int EPI, bool PAIR = false>
-__global__ void __launch_bounds__(TC_THREADS, 1)
-    tc_gemm_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUtensorMap tmB,
-                   const __grid_constant__ CUtensorMap tmO0, const __grid_constant__ CUtensorMap tmO1,
-                   int K, const int* __restrict__ offA, const int* __restrict__ offB, EpiArgs ep) {
-  using Cfg = TcCfg<BN, B_MN, EPI, PAIR>;
+// The fused epilogue of ONE output tile (m_tile, n_tile) whose accumulator is TMEM buffer `acc` of
+// the CTA's i-th tile: bias staging / sigma' prefetch, wait for the MMAs, TMEM -> registers ->
+// EPI-specific epilogue (epilogue.cuh) -> global (or the split-K park), then release the
+// accumulator to the MMA warp.  Executed by the TC_EPI_WARPS epilogue warps; shared by
+// tc_gemm_kernel and the persistent small-batch step kernel (step_kernel.cuh).
+struct EpiTileCtx {
+  uint32_t tmem_base;
+  uint64_t* tmem_full_bar;
+  uint64_t* tmem_empty_bar;
+  float* sbias;         // [2][BN]
+  float* red;           // [4 * BN]
+  float* dzs;           // [TC_BM * 16] (HEAD_XENT fused dX)
+  uint8_t* sout;        // TMA-store staging
+  uint8_t* smem;        // stage ring base (split-K park)
+  const CUtensorMap* tmO0;
+  const CUtensorMap* tmO1;
+  int splits, num_kb;
+  int warp, lane;
+  unsigned long long* dbg;
+};
+
+template <int BN, int EPI>
+__device__ __forceinline__ void tc_epilogue_tile(const EpiArgs& ep, const EpiTileCtx& x, int m_tile, int n_tile,
+                                                 int acc, int i, int acc_stride = BN) {
   using TO = TmaOut<BN, EPI>;
-  constexpr int STAGES = Cfg::STAGES;
-  static_assert(!PAIR || (A_MN && B_MN && BN >= 128 && !TO::on), "CTA pairs: split-K dW GEMMs only");
-  extern __shared__ uint8_t smem_raw[];
-  uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
-  uint8_t* sout = smem + STAGES * Cfg::STAGE_BYTES;  // TMA-store staging [NOUT][NBOX][128 rows x 128 B]
-  uint64_t* full_bar = reinterpret_cast<uint64_t*>(sout + Cfg::OUT_BYTES);
-  uint64_t* empty_bar = full_bar + STAGES;
-  uint64_t* tmem_full_bar = empty_bar + STAGES;   // [2]: accumulator a ready (MMA -> epilogue)
-  uint64_t* tmem_empty_bar = tmem_full_bar + 2;    // [2]: accumulator a drained (epilogue -> MMA)
-  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(tmem_empty_bar + 2);
-  __shared__ float red[4 * BN];    // per-quadrant column sums (bias-gradient partials)
-  __shared__ float sbias[2][BN];   // bias of the tile, double-buffered across tiles
-  __shared__ __align__(16) float dzs[EPI == EPI_HEAD_XENT ? TC_BM * 16 : 4];  // dZ_L rows (fused head dX)
-
-  const int warp = threadIdx.x >> 5;
-  const int lane = threadIdx.x & 31;
-  unsigned long long* dbg = ep.dbg ? ep.dbg + 12 * ((size_t)(blockIdx.z * gridDim.y + blockIdx.y) * gridDim.x + blockIdx.x) : nullptr;
-  HB_STAMP(dbg && threadIdx.x == 0, dbg[0]);
-  // Tiles: persistent CTAs walk tiles t = blockIdx.x, +gridDim.x, ... (n fastest, so CTAs running
-  // together share the A row panel in L2).  Split-K launches (gridDim.z > 1) are one tile per CTA.
-  const int tiles_n = (ep.N + BN - 1) / BN;
-  const int tiles_m = (ep.M + TC_BM - 1) / TC_BM;
-  const int num_tiles = tiles_n * tiles_m;
-  // split-K (dW GEMMs with K = batch): the gridDim.z CTAs of one output tile form a cluster,
-  // each accumulates k-blocks [kb_lo, kb_hi) in its own TMEM
-  const int splits = gridDim.z;
-  const int t_first = splits == 1 ? (int)blockIdx.x : (int)(blockIdx.y * gridDim.x + blockIdx.x);
-  const int t_step = splits == 1 ? (int)gridDim.x : num_tiles;
-  const int kz = blockIdx.z;
-  // CTA pair (grid x = M tiles, y = N tiles, z = splits; cluster (2, 1, S) — pairs must be along
-  // the cluster's x): half = blockIdx.x & 1; cluster rank of split sp's CTA with the same half =
-  // half + 2 sp; the pair's leader (half 0) has rank 2 kz
-  const uint32_t half = PAIR ? (blockIdx.x & 1) : 0;
-  const uint16_t pair_mask = (uint16_t)(3u << (2 * kz));
-  const int num_kb_all = (K + TC_BK - 1) / TC_BK;
-  const int kpb = (num_kb_all + splits - 1) / splits;
-  const int kb_lo = min(num_kb_all, kz * kpb);
-  const int num_kb = min(num_kb_all, kb_lo + kpb) - kb_lo;
-
-  if (warp == 0 && lane == 0) {
-    tma_prefetch_desc(&tmA);
-    tma_prefetch_desc(&tmB);
-    for (int s = 0; s < STAGES; ++s) {
-      mbar_init(&full_bar[s], 1);
-      mbar_init(&empty_bar[s], 1);
-    }
-    for (int a = 0; a < 2; ++a) {
-      mbar_init(&tmem_full_bar[a], 1);
-      mbar_init(&tmem_empty_bar[a], TC_EPI_WARPS);  // one arrive per epilogue warp
-    }
-    fence_barrier_init();
-  }
-  if (warp == 2) {
-    if (PAIR)
-      tmem_alloc_pair<Cfg::TMEM_COLS>(tmem_slot);
-    else
-      tmem_alloc<Cfg::TMEM_COLS>(tmem_slot);
-  }
-  tc_fence_before();
-  __syncthreads();
-  if (PAIR) cluster_sync_all();  // the leader's barriers are initialised before the peer's loads signal them
-  tc_fence_after();
-  const uint32_t tmem_base = *tmem_slot;
-  // programmatic dependent launch: everything above overlapped the previous kernel's tail;
-  // no global memory produced by it is touched before this point
-  asm volatile("griddepcontrol.wait;" ::: "memory");
-  asm volatile("griddepcontrol.launch_dependents;" ::: "memory");
-  HB_STAMP(dbg && threadIdx.x == 0, dbg[1]);
-
-  if (warp == 0 && lane == 0) {
-    // ===== TMA producer =====
-    const int oa = offA ? __ldg(offA) : 0;
-    const int ob = offB ? __ldg(offB) : 0;
-    int it = 0;  // k-blocks issued by this CTA (ring position across tiles)
-    for (int t = t_first; t < num_tiles; t += t_step) {
-    int mt_, nt_;
-    tile_coords(t, tiles_m, tiles_n, mt_, nt_);
-    if (PAIR) {  // one tile per CTA: this CTA's own M tile, the pair's N tile (its half of it)
-      mt_ = blockIdx.x;
-      nt_ = blockIdx.y;
-    }
-    const int m0 = mt_ * TC_BM, n0 = nt_ * BN + (int)half * Cfg::B_TILE;
-    const uint32_t lead_full = PAIR ? mapa_shared(smem_u32(full_bar), 2 * kz) : 0;
-    for (int kb = 0; kb < num_kb; ++kb, ++it) {
-      const int s = it % STAGES;
-      const uint32_t ph = (it / STAGES) & 1;
-      mbar_wait(&empty_bar[s], ph ^ 1);
-      uint8_t* sA = smem + s * Cfg::STAGE_BYTES;
-      uint8_t* sB = sA + Cfg::A_BYTES;
-      const int k0 = (kb_lo + kb) * TC_BK;
-      if (PAIR) {  // both CTAs' loads complete on the leader's barrier, which expects both
-        const uint32_t fb = lead_full + (uint32_t)(s * 8);
-        if (half == 0) mbar_arrive_expect_tx(&full_bar[s], 2 * Cfg::STAGE_BYTES);
-        tma_load_2d_pair(sA, &tmA, fb, m0, k0 + oa);
-        tma_load_2d_pair(sA + 8192, &tmA, fb, m0 + 64, k0 + oa);
-#pragma unroll
-        for (int j = 0; j < Cfg::B_ROWS / 64; ++j) tma_load_2d_pair(sB + j * 8192, &tmB, fb, n0 + 64 * j, k0 + ob);
-        continue;
-      }
-      mbar_arrive_expect_tx(&full_bar[s], Cfg::STAGE_BYTES);
-      if (!A_MN) {
-        tma_load_2d(sA, &tmA, &full_bar[s], k0, m0 + oa);
-      } else {
-        tma_load_2d(sA, &tmA, &full_bar[s], m0, k0 + oa);
-        tma_load_2d(sA + 8192, &tmA, &full_bar[s], m0 + 64, k0 + oa);
-      }
-      if (!B_MN) {
-        tma_load_2d(sB, &tmB, &full_bar[s], k0, n0 + ob);
-      } else {
-#pragma unroll
-        for (int j = 0; j < Cfg::B_ROWS / 64; ++j)
-          tma_load_2d(sB + j * 8192, &tmB, &full_bar[s], n0 + 64 * j, k0 + ob);
-      }
-    }
-    }
-  } else if (warp == 1 && lane == 0 && half == 0) {
-    // ===== MMA issuer (single thread; in a pair the leader issues for both CTAs) =====
-    constexpr uint32_t idesc = make_idesc_bf16(PAIR ? 2 * TC_BM : TC_BM, BN, A_MN, B_MN);
-    int it = 0, i = 0;
-    for (int t = t_first; t < num_tiles; t += t_step, ++i) {
-    const int acc = i & 1;
-    mbar_wait(&tmem_empty_bar[acc], ((i >> 1) & 1) ^ 1);  // epilogue has drained this accumulator
-    tc_fence_after();
-    const uint32_t tacc = tmem_base + (uint32_t)(acc * BN);
-    for (int kb = 0; kb < num_kb; ++kb, ++it) {
-      const int s = it % STAGES;
-      const uint32_t ph = (it / STAGES) & 1;
-      mbar_wait(&full_bar[s], ph);
-      tc_fence_after();
-      HB_STAMP(dbg && it == 0, dbg[2]);
-      const uint32_t a_base = smem_u32(smem + s * Cfg::STAGE_BYTES);
-      const uint32_t b_base = a_base + Cfg::A_BYTES;
-#pragma unroll
-      for (int kk = 0; kk < TC_BK / 16; ++kk) {
-        // K-major SW128: rows of 128 B, 8-row groups 1024 B apart (SBO); +32 B per UMMA_K = 16.
-        // MN-major SW128: 64-element MN chunks 8192 B apart (LBO), 8-row K groups 1024 B apart
-        // (SBO); +16 rows * 128 B = 2048 B per UMMA_K.
-        const uint64_t ad = A_MN ? make_sw128_desc(a_base + kk * 2048, 8192, 1024)
-                                 : make_sw128_desc(a_base + kk * 32, 16, 1024);
-        const uint64_t bd = B_MN ? make_sw128_desc(b_base + kk * 2048, 8192, 1024)
-                                 : make_sw128_desc(b_base + kk * 32, 16, 1024);
-        if (PAIR)
-          umma_bf16_pair(tacc, ad, bd, idesc, (kb | kk) != 0);
-        else
-          umma_bf16(tacc, ad, bd, idesc, (kb | kk) != 0);
-      }
-      if (PAIR)
-        umma_commit_pair(&empty_bar[s], pair_mask);  // both CTAs' slots
-      else
-        umma_commit(&empty_bar[s]);  // frees the smem slot when these MMAs complete
-    }
-    if (PAIR)
-      umma_commit_pair(&tmem_full_bar[acc], pair_mask);
-    else
-      umma_commit(&tmem_full_bar[acc]);  // accumulator ready (arrives even if num_kb == 0)
-    HB_STAMP(dbg && i == 0, dbg[3]);
-    }
-  } else if (warp >= 4) {
-    // ===== epilogue (8 warps): TMEM -> registers -> fused epilogue -> global =====
-    // warp w reads TMEM lanes 32*(w%4).. (tile rows) and handles column half h = (w-4)/4
-    const int q = warp & 3;
-    const int h = (warp - 4) >> 2;  // column part 0..TC_EPI_PARTS-1
-    const int et = threadIdx.x - 128;  // 0..255
-    const int rl = q * 32 + lane;      // row within the tile
-    constexpr int NP = BN / 16 < TC_EPI_PARTS ? BN / 16 : TC_EPI_PARTS;  // parts with columns
-    constexpr int HALF = BN / NP;                                        // columns per warp
-    const bool active = h < NP;
-    const int c_lo = active ? h * HALF : 0;
-    int i = 0;
-    for (int t = t_first; t < num_tiles; t += t_step, ++i) {
-    const int acc = i & 1;
-    int m_tile, n_tile;
-    tile_coords(t, tiles_m, tiles_n, m_tile, n_tile);
-    if (PAIR) {
-      m_tile = blockIdx.x;
-      n_tile = blockIdx.y;
-    }
+  const int warp = x.warp, lane = x.lane;
+  const int q = warp & 3;
+  const int h = (warp - 4) >> 2;  // column part 0..TC_EPI_PARTS-1
+  const int et = threadIdx.x - 128;  // 0..TC_EPI_THREADS-1
+  const int rl = q * 32 + lane;      // row within the tile
+  constexpr int NP = BN / 16 < TC_EPI_PARTS ? BN / 16 : TC_EPI_PARTS;  // parts with columns
+  constexpr int HALF = BN / NP;                                        // columns per warp
+  const bool active = h < NP;
+  const int c_lo = active ? h * HALF : 0;
+  const int splits = x.splits, num_kb = x.num_kb;
+  uint8_t* sout = x.sout;
+  uint8_t* smem = x.smem;
+  float* red = x.red;
+  float* dzs = x.dzs;
+  uint64_t* tmem_full_bar = x.tmem_full_bar;
+  uint64_t* tmem_empty_bar = x.tmem_empty_bar;
+  const uint32_t tmem_base = x.tmem_base;
+  unsigned long long* dbg = x.dbg;
+  (void)dbg;
+  (void)dzs;
+  (void)sout;
+  (void)smem;
     const int m0 = m_tile * TC_BM, n0 = n_tile * BN;
     const int r = m0 + rl;
     const bool row_ok = r < ep.M;
-    const uint32_t tbase = tmem_base + (uint32_t)(acc * BN) + ((uint32_t)(q * 32) << 16);
-    float* sb = sbias[acc];
+    const uint32_t tbase = tmem_base + (uint32_t)(acc * acc_stride) + ((uint32_t)(q * 32) << 16);
+    float* sb = x.sbias + acc * BN;
 
     // stage the bias of the tile's columns in shared memory while the mainloop runs
     if (EPI == EPI_FWD_SIG || EPI == EPI_FWD_LOGITS || EPI == EPI_HEAD_XENT) {
@@ -648,7 +511,7 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
             if (o == 1 && !ep.out1) continue;
 #pragma unroll
             for (int bx = 0; bx < TO::NBOX; ++bx)
-              tma_store_2d(o == 0 ? &tmO0 : &tmO1, sout + (size_t)(o * TO::NBOX + bx) * TC_BM * 128, n0 + bx * 64, m0);
+              tma_store_2d(o == 0 ? x.tmO0 : x.tmO1, sout + (size_t)(o * TO::NBOX + bx) * TC_BM * 128, n0 + bx * 64, m0);
           }
           tma_store_commit();
         }
@@ -673,7 +536,187 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
     tc_fence_before();
     __syncwarp();
     if (lane == 0) mbar_arrive(&tmem_empty_bar[acc]);
-    }  // tile loop
+}
+
+template <int BN, bool A_MN, bool B_MN, int EPI, bool PAIR = false>
+__global__ void __launch_bounds__(TC_THREADS, 1)
+    tc_gemm_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUtensorMap tmB,
+                   const __grid_constant__ CUtensorMap tmO0, const __grid_constant__ CUtensorMap tmO1,
+                   int K, const int* __restrict__ offA, const int* __restrict__ offB, EpiArgs ep) {
+  using Cfg = TcCfg<BN, B_MN, EPI, PAIR>;
+  using TO = TmaOut<BN, EPI>;
+  constexpr int STAGES = Cfg::STAGES;
+  static_assert(!PAIR || (A_MN && B_MN && BN >= 128 && !TO::on), "CTA pairs: split-K dW GEMMs only");
+  extern __shared__ uint8_t smem_raw[];
+  uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
+  uint8_t* sout = smem + STAGES * Cfg::STAGE_BYTES;  // TMA-store staging [NOUT][NBOX][128 rows x 128 B]
+  uint64_t* full_bar = reinterpret_cast<uint64_t*>(sout + Cfg::OUT_BYTES);
+  uint64_t* empty_bar = full_bar + STAGES;
+  uint64_t* tmem_full_bar = empty_bar + STAGES;   // [2]: accumulator a ready (MMA -> epilogue)
+  uint64_t* tmem_empty_bar = tmem_full_bar + 2;    // [2]: accumulator a drained (epilogue -> MMA)
+  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(tmem_empty_bar + 2);
+  __shared__ float red[4 * BN];    // per-quadrant column sums (bias-gradient partials)
+  __shared__ float sbias[2][BN];   // bias of the tile, double-buffered across tiles
+  __shared__ __align__(16) float dzs[EPI == EPI_HEAD_XENT ? TC_BM * 16 : 4];  // dZ_L rows (fused head dX)
+
+  const int warp = threadIdx.x >> 5;
+  const int lane = threadIdx.x & 31;
+  unsigned long long* dbg = ep.dbg ? ep.dbg + 12 * ((size_t)(blockIdx.z * gridDim.y + blockIdx.y) * gridDim.x + blockIdx.x) : nullptr;
+  HB_STAMP(dbg && threadIdx.x == 0, dbg[0]);
+  // Tiles: persistent CTAs walk tiles t = blockIdx.x, +gridDim.x, ... (n fastest, so CTAs running
+  // together share the A row panel in L2).  Split-K launches (gridDim.z > 1) are one tile per CTA.
+  const int tiles_n = (ep.N + BN - 1) / BN;
+  const int tiles_m = (ep.M + TC_BM - 1) / TC_BM;
+  const int num_tiles = tiles_n * tiles_m;
+  // split-K (dW GEMMs with K = batch): the gridDim.z CTAs of one output tile form a cluster,
+  // each accumulates k-blocks [kb_lo, kb_hi) in its own TMEM
+  const int splits = gridDim.z;
+  const int t_first = splits == 1 ? (int)blockIdx.x : (int)(blockIdx.y * gridDim.x + blockIdx.x);
+  const int t_step = splits == 1 ? (int)gridDim.x : num_tiles;
+  const int kz = blockIdx.z;
+  // CTA pair (grid x = M tiles, y = N tiles, z = splits; cluster (2, 1, S) — pairs must be along
+  // the cluster's x): half = blockIdx.x & 1; cluster rank of split sp's CTA with the same half =
+  // half + 2 sp; the pair's leader (half 0) has rank 2 kz
+  const uint32_t half = PAIR ? (blockIdx.x & 1) : 0;
+  const uint16_t pair_mask = (uint16_t)(3u << (2 * kz));
+  const int num_kb_all = (K + TC_BK - 1) / TC_BK;
+  const int kpb = (num_kb_all + splits - 1) / splits;
+  const int kb_lo = min(num_kb_all, kz * kpb);
+  const int num_kb = min(num_kb_all, kb_lo + kpb) - kb_lo;
+
+  if (warp == 0 && lane == 0) {
+    tma_prefetch_desc(&tmA);
+    tma_prefetch_desc(&tmB);
+    for (int s = 0; s < STAGES; ++s) {
+      mbar_init(&full_bar[s], 1);
+      mbar_init(&empty_bar[s], 1);
+    }
+    for (int a = 0; a < 2; ++a) {
+      mbar_init(&tmem_full_bar[a], 1);
+      mbar_init(&tmem_empty_bar[a], TC_EPI_WARPS);  // one arrive per epilogue warp
+    }
+    fence_barrier_init();
+  }
+  if (warp == 2) {
+    if (PAIR)
+      tmem_alloc_pair<Cfg::TMEM_COLS>(tmem_slot);
+    else
+      tmem_alloc<Cfg::TMEM_COLS>(tmem_slot);
+  }
+  tc_fence_before();
+  __syncthreads();
+  if (PAIR) cluster_sync_all();  // the leader's barriers are initialised before the peer's loads signal them
+  tc_fence_after();
+  const uint32_t tmem_base = *tmem_slot;
+  // programmatic dependent launch: everything above overlapped the previous kernel's tail;
+  // no global memory produced by it is touched before this point
+  asm volatile("griddepcontrol.wait;" ::: "memory");
+  asm volatile("griddepcontrol.launch_dependents;" ::: "memory");
+  HB_STAMP(dbg && threadIdx.x == 0, dbg[1]);
+
+  if (warp == 0 && lane == 0) {
+    // ===== TMA producer =====
+    const int oa = offA ? __ldg(offA) : 0;
+    const int ob = offB ? __ldg(offB) : 0;
+    int it = 0;  // k-blocks issued by this CTA (ring position across tiles)
+    for (int t = t_first; t < num_tiles; t += t_step) {
+    int mt_, nt_;
+    tile_coords(t, tiles_m, tiles_n, mt_, nt_);
+    if (PAIR) {  // one tile per CTA: this CTA's own M tile, the pair's N tile (its half of it)
+      mt_ = blockIdx.x;
+      nt_ = blockIdx.y;
+    }
+    const int m0 = mt_ * TC_BM, n0 = nt_ * BN + (int)half * Cfg::B_TILE;
+    const uint32_t lead_full = PAIR ? mapa_shared(smem_u32(full_bar), 2 * kz) : 0;
+    for (int kb = 0; kb < num_kb; ++kb, ++it) {
+      const int s = it % STAGES;
+      const uint32_t ph = (it / STAGES) & 1;
+      mbar_wait(&empty_bar[s], ph ^ 1);
+      uint8_t* sA = smem + s * Cfg::STAGE_BYTES;
+      uint8_t* sB = sA + Cfg::A_BYTES;
+      const int k0 = (kb_lo + kb) * TC_BK;
+      if (PAIR) {  // both CTAs' loads complete on the leader's barrier, which expects both
+        const uint32_t fb = lead_full + (uint32_t)(s * 8);
+        if (half == 0) mbar_arrive_expect_tx(&full_bar[s], 2 * Cfg::STAGE_BYTES);
+        tma_load_2d_pair(sA, &tmA, fb, m0, k0 + oa);
+        tma_load_2d_pair(sA + 8192, &tmA, fb, m0 + 64, k0 + oa);
+#pragma unroll
+        for (int j = 0; j < Cfg::B_ROWS / 64; ++j) tma_load_2d_pair(sB + j * 8192, &tmB, fb, n0 + 64 * j, k0 + ob);
+        continue;
+      }
+      mbar_arrive_expect_tx(&full_bar[s], Cfg::STAGE_BYTES);
+      if (!A_MN) {
+        tma_load_2d(sA, &tmA, &full_bar[s], k0, m0 + oa);
+      } else {
+        tma_load_2d(sA, &tmA, &full_bar[s], m0, k0 + oa);
+        tma_load_2d(sA + 8192, &tmA, &full_bar[s], m0 + 64, k0 + oa);
+      }
+      if (!B_MN) {
+        tma_load_2d(sB, &tmB, &full_bar[s], k0, n0 + ob);
+      } else {
+#pragma unroll
+        for (int j = 0; j < Cfg::B_ROWS / 64; ++j)
+          tma_load_2d(sB + j * 8192, &tmB, &full_bar[s], n0 + 64 * j, k0 + ob);
+      }
+    }
+    }
+  } else if (warp == 1 && lane == 0 && half == 0) {
+    // ===== MMA issuer (single thread; in a pair the leader issues for both CTAs) =====
+    constexpr uint32_t idesc = make_idesc_bf16(PAIR ? 2 * TC_BM : TC_BM, BN, A_MN, B_MN);
+    int it = 0, i = 0;
+    for (int t = t_first; t < num_tiles; t += t_step, ++i) {
+    const int acc = i & 1;
+    mbar_wait(&tmem_empty_bar[acc], ((i >> 1) & 1) ^ 1);  // epilogue has drained this accumulator
+    tc_fence_after();
+    const uint32_t tacc = tmem_base + (uint32_t)(acc * BN);
+    for (int kb = 0; kb < num_kb; ++kb, ++it) {
+      const int s = it % STAGES;
+      const uint32_t ph = (it / STAGES) & 1;
+      mbar_wait(&full_bar[s], ph);
+      tc_fence_after();
+      HB_STAMP(dbg && it == 0, dbg[2]);
+      const uint32_t a_base = smem_u32(smem + s * Cfg::STAGE_BYTES);
+      const uint32_t b_base = a_base + Cfg::A_BYTES;
+#pragma unroll
+      for (int kk = 0; kk < TC_BK / 16; ++kk) {
+        // K-major SW128: rows of 128 B, 8-row groups 1024 B apart (SBO); +32 B per UMMA_K = 16.
+        // MN-major SW128: 64-element MN chunks 8192 B apart (LBO), 8-row K groups 1024 B apart
+        // (SBO); +16 rows * 128 B = 2048 B per UMMA_K.
+        const uint64_t ad = A_MN ? make_sw128_desc(a_base + kk * 2048, 8192, 1024)
+                                 : make_sw128_desc(a_base + kk * 32, 16, 1024);
+        const uint64_t bd = B_MN ? make_sw128_desc(b_base + kk * 2048, 8192, 1024)
+                                 : make_sw128_desc(b_base + kk * 32, 16, 1024);
+        if (PAIR)
+          umma_bf16_pair(tacc, ad, bd, idesc, (kb | kk) != 0);
+        else
+          umma_bf16(tacc, ad, bd, idesc, (kb | kk) != 0);
+      }
+      if (PAIR)
+        umma_commit_pair(&empty_bar[s], pair_mask);  // both CTAs' slots
+      else
+        umma_commit(&empty_bar[s]);  // frees the smem slot when these MMAs complete
+    }
+    if (PAIR)
+      umma_commit_pair(&tmem_full_bar[acc], pair_mask);
+    else
+      umma_commit(&tmem_full_bar[acc]);  // accumulator ready (arrives even if num_kb == 0)
+    HB_STAMP(dbg && i == 0, dbg[3]);
+    }
+  } else if (warp >= 4) {
+    // ===== epilogue (8 warps): TMEM -> registers -> fused epilogue -> global =====
+    // warp w reads TMEM lanes 32*(w%4).. (tile rows) and handles column half h = (w-4)/4
+    const EpiTileCtx ectx{tmem_base, tmem_full_bar, tmem_empty_bar, &sbias[0][0], red, dzs, sout, smem, &tmO0,
+                          &tmO1, splits, num_kb, warp, lane, dbg};
+    int i = 0;
+    for (int t = t_first; t < num_tiles; t += t_step, ++i) {
+      int m_tile, n_tile;
+      tile_coords(t, tiles_m, tiles_n, m_tile, n_tile);
+      if (PAIR) {
+        m_tile = blockIdx.x;
+        n_tile = blockIdx.y;
+      }
+      tc_epilogue_tile<BN, EPI>(ep, ectx, m_tile, n_tile, i & 1, i);
+    }
   }
 
   if ((EPI == EPI_WGRAD_SGD || EPI == EPI_WGRAD_STORE) && splits > 1) {

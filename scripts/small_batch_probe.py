@@ -14,8 +14,9 @@ X, y = dataset("covtype", max(bs) * 64, seed=0)
 tX, ty = to_device(X, y)
 m = hb.MLP(dims)
 m.set_params(params_to_flat(init_params(dims)))
-w = hb.Worker(m, max(bs))
+m.set_option("step_kernel_max_b", int(os.environ.get("SKB", "0")))
 for b in bs:
+    w = hb.Worker(m, b)  # per-b worker: the persistent kernel's grid follows its max_batch
     n = b * steps
     reps = max(1, (n + tX.shape[0] - 1) // tX.shape[0])
     Xb, yb = (tX.repeat(reps, 1)[:n].contiguous(), ty.repeat(reps)[:n].contiguous()) if reps > 1 else (tX[:n], ty[:n])

@@ -163,6 +163,41 @@ def test_delicious_shaped_983_class_head(prec):
     assert le <= TOL[prec]
 
 
+@pytest.mark.parametrize("b", [32, 256, 1000, 2048])
+def test_persistent_step_kernel_matches_oracle_and_per_layer_path(b):
+    # small batches of narrow nets run as ONE persistent launch (step_kernel.cuh): the same GEMMs,
+    # operands and epilogues as the per-layer launches, as stages between grid barriers
+    dims = [54, 512, 512, 512, 512, 7]
+    X, y = dataset("covtype", b, seed=21)
+    params = init_params(dims, seed=2)
+    tX, ty = to_device(X, y)
+    out = {}
+    for mode in ("persistent", "per_layer"):
+        m = hb.MLP(dims)
+        m.set_params(params_to_flat(params))
+        m.set_option("step_kernel_max_b", 2048 if mode == "persistent" else 0)
+        w = hb.Worker(m, b)
+        l0 = hb.kernel_launches()
+        g, loss = w.step_grads(tX, ty, b)
+        out[mode] = (g, loss, hb.kernel_launches() - l0)
+    assert out["persistent"][2] == 2 and out["per_layer"][2] == 15  # + the batch-loss reduction
+    dW, db, l_ref = mlp64.grads(params, X.astype(np.float64), y)
+    norm, elem = grad_errors(out["persistent"][0], dims, dW, db)
+    assert max(norm) <= TOL["bf16"] and max(elem) <= TOL["bf16"], (norm, elem)
+    assert abs(out["persistent"][1] - l_ref) / l_ref <= TOL["bf16"]
+    assert rel_err(out["persistent"][0], out["per_layer"][0]) <= 1e-3
+    # and one in-place SGD step through it
+    m = hb.MLP(dims)
+    m.set_params(params_to_flat(params))
+    m.set_option("step_kernel_max_b", 2048)
+    w = hb.Worker(m, b)
+    w.step(tX, ty, b, 0.5)
+    new, _ = mlp64.sgd_step(params, X.astype(np.float64), y, 0.5)
+    got = split_flat(m.get_params(), dims)
+    for l in range(len(dims) - 1):
+        assert rel_err(got[l][0] - params[l][0], new[l][0] - params[l][0]) <= TOL["bf16"], l
+
+
 def test_batch_equal_to_max_batch_and_ragged_tiles():
     # b = max_batch with a ragged last row tile (b % 128 != 0) and ragged widths
     e, le, errs = grads_case([100, 136, 72, 3], "gauss", 1000, "bf16", d=100)
