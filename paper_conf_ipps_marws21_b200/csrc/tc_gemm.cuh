@@ -40,13 +40,23 @@ constexpr int TC_EPI_PARTS = TC_EPI_WARPS / 4;
 constexpr int TC_THREADS = 128 + TC_EPI_THREADS;   // 4 control warps + the epilogue warps
 
 // Epilogues whose bf16 outputs are staged in swizzled shared memory and written with TMA bulk
-// stores (full 128-byte lines instead of one 16-byte piece of 32 different rows per warp store)
+// stores (full 128-byte lines instead of one 16-byte piece of 32 different rows per warp store).
+// The tile is written in 64-column chunks through TWO staging buffers: chunk j is staged while the
+// bulk stores of chunk j-1 drain, so the staging costs 2 x NOUT x 16 KB whatever BN (B200, C3
+// 8192x1024x1024: 256-wide tiles with a whole-tile staged epilogue were epilogue-bound).
 template <int BN, int EPI>
 struct TmaOut {
-  static constexpr bool on = (EPI == EPI_FWD_SIG || EPI == EPI_DGRAD_SIG) && (BN == 64 || BN == 128);
-  static constexpr int NBOX = BN / 64;                     // 64-column boxes per output
-  static constexpr int NOUT = EPI == EPI_FWD_SIG ? 2 : 1;  // H and S, or dZ
-  static constexpr int BYTES = on ? NOUT * NBOX * TC_BM * 128 : 0;
+#ifndef HB_TMA_OUT_MAX_BN
+#define HB_TMA_OUT_MAX_BN 256
+#endif
+  static constexpr bool on = (EPI == EPI_FWD_SIG || EPI == EPI_DGRAD_SIG) && (BN == 64 || BN == 128 || BN == 256) &&
+                             BN <= HB_TMA_OUT_MAX_BN;
+  static constexpr int NCHUNK = BN / 64;                   // 64-column chunks per tile
+  // 256-wide tiles keep a 4-deep operand ring: one staging buffer, and the forward's sigma' stash
+  // is written directly (only H goes through TMA); narrower tiles double-buffer H and S
+  static constexpr int NBUF = BN == 128 ? 2 : 1;
+  static constexpr int NOUT = EPI == EPI_FWD_SIG && BN <= 128 ? 2 : 1;  // staged outputs
+  static constexpr int BYTES = on ? NBUF * NOUT * TC_BM * 128 : 0;
 };
 
 // PAIR: a CTA pair (cluster x = 2) computes a 256 x BN tile with tcgen05.mma.cta_group::2 — each
@@ -59,7 +69,10 @@ struct TcCfg {
   static constexpr int B_BYTES = B_ROWS * TC_BK * 2;
   static constexpr int STAGE_BYTES = A_BYTES + B_BYTES;
   static constexpr int OUT_BYTES = TmaOut<BN, EPI>::BYTES;
-  static constexpr int STAGES_RAW = (192 * 1024 - OUT_BYTES) / STAGE_BYTES;
+#ifndef HB_RING_BYTES
+#define HB_RING_BYTES (210 * 1024)
+#endif
+  static constexpr int STAGES_RAW = (HB_RING_BYTES - OUT_BYTES) / STAGE_BYTES;
   static constexpr int STAGES = STAGES_RAW > 8 ? 8 : STAGES_RAW;
   // two accumulators (double buffer); TMEM is allocated in powers of two >= 32 columns
   static constexpr int TMEM_COLS = 2 * BN <= 32 ? 32 : 2 * BN <= 64 ? 64 : 2 * BN <= 128 ? 128 : 2 * BN <= 256 ? 256 : 512;
@@ -158,6 +171,15 @@ __device__ __forceinline__ void tile_coords(int t, int tiles_m, int tiles_n, int
 // Write 16 bf16 values (8 packed words) of tile row rl, tile columns c..c+15 into staging output o
 // (boxes of 128 rows x 64 columns, 128-byte rows, 16-byte chunks XOR-swizzled by row % 8 — the
 // TMA SWIZZLE_128B layout, which also makes these per-row writes bank-conflict free).
+// 16 bf16 values (8 packed words) of tile row rl, chunk columns c..c+15 (c < 64) into a 128-row x
+// 128-byte staging box (TMA SWIZZLE_128B layout)
+__device__ __forceinline__ void stage16_box(uint8_t* box, int rl, int c, const uint32_t* p) {
+  const int j0 = c >> 3;
+  uint8_t* row = box + (size_t)rl * 128;
+  *reinterpret_cast<uint4*>(row + ((j0 ^ (rl & 7)) << 4)) = make_uint4(p[0], p[1], p[2], p[3]);
+  *reinterpret_cast<uint4*>(row + (((j0 + 1) ^ (rl & 7)) << 4)) = make_uint4(p[4], p[5], p[6], p[7]);
+}
+
 template <int NBOX>
 __device__ __forceinline__ void stage16(uint8_t* sout, int o, int rl, int c, const uint32_t* p) {
   const int box = c >> 6, j0 = (c & 63) >> 3;
@@ -229,7 +251,10 @@ __device__ __forceinline__ void tc_epilogue_tile(const EpiArgs& ep, const EpiTil
     if (EPI == EPI_DGRAD_SIG && active && row_ok) {
 #pragma unroll
       for (int i = 0; i < NCH; ++i) {
-        const int nc = n0 + c_lo + 16 * i;
+        // group i of this warp: whole-tile layout [c_lo + 16 i], or chunked (TMA store) layout
+        // chunk i / (CW/16), columns h * CW + 16 (i % (CW/16)) of it
+        constexpr int G16 = (64 / TC_EPI_PARTS) / 16 > 0 ? (64 / TC_EPI_PARTS) / 16 : 1;
+        const int nc = TO::on ? n0 + 64 * (i / G16) + h * (64 / TC_EPI_PARTS) + 16 * (i % G16) : n0 + c_lo + 16 * i;
         if (nc + 16 <= ep.N) {
           const uint4* S = reinterpret_cast<const uint4*>(static_cast<const __nv_bfloat16*>(ep.aux) +
                                                           (int64_t)r * ep.ldaux + nc);
@@ -357,6 +382,110 @@ __device__ __forceinline__ void tc_epilogue_tile(const EpiArgs& ep, const EpiTil
                 epi_elem<EPI, __nv_bfloat16, false>(ep, r, j, __uint_as_float(r0[j]) + __uint_as_float(r1[j]));
           }
         }
+      } else if (TO::on) {
+        // ---- 64-column chunks through two staging buffers, one bulk-store group per chunk ----
+        constexpr int CW = 64 / TC_EPI_PARTS;  // columns of a chunk per warp
+        static_assert(CW % 16 == 0, "chunk columns per warp");
+        int pi = 0;  // index into this warp's prefetched sigma' groups (dgrad)
+#pragma unroll
+        for (int j = 0; j < TO::NCHUNK; ++j) {
+          uint8_t* sbuf = sout + (size_t)(j % TO::NBUF) * TO::NOUT * TC_BM * 128;
+          if (j >= TO::NBUF) {  // the bulk stores of chunk j - NBUF have read this buffer
+            if (et == 0) {
+              if (TO::NBUF == 2)
+                tma_store_wait_read_1();
+              else
+                tma_store_wait_read();
+            }
+            epi_bar_sync();
+          }
+#pragma unroll
+          for (int g = 0; g < CW / 16; ++g, ++pi) {
+            const int cc = h * CW + 16 * g;  // column within the chunk
+            const int c = 64 * j + cc;       // column within the tile
+            const int nc = n0 + c;
+            float v[16];
+            if (nc < ep.N) {  // warp-uniform
+              uint32_t raw[16];
+              tmem_ld_32x32b_x16(tbase + (uint32_t)c, raw);
+              tmem_ld_wait();
+#pragma unroll
+              for (int k = 0; k < 16; ++k) v[k] = __uint_as_float(raw[k]);
+            } else {
+#pragma unroll
+              for (int k = 0; k < 16; ++k) v[k] = 0.f;
+            }
+            if (EPI == EPI_FWD_SIG) {
+              // all rows / columns staged; rows >= M and columns >= N are clipped by the TMA store
+              uint32_t hp[8], sp[8];
+#pragma unroll
+              for (int qq = 0; qq < 8; ++qq) {
+                float h0, d0, h1, d1;
+                sigmoid_d_fast(v[2 * qq] + sb[c + 2 * qq], h0, d0);
+                sigmoid_d_fast(v[2 * qq + 1] + sb[c + 2 * qq + 1], h1, d1);
+                hp[qq] = pack_bf16x2(h0, h1);
+                sp[qq] = pack_bf16x2(d0, d1);
+              }
+              stage16_box(sbuf, rl, cc, hp);
+              if (ep.out1) {
+                if (TO::NOUT == 2) {
+                  stage16_box(sbuf + TC_BM * 128, rl, cc, sp);
+                } else if (row_ok) {  // sigma' stash written directly (256-wide tiles)
+                  __nv_bfloat16* S = static_cast<__nv_bfloat16*>(ep.out1) + (int64_t)r * ep.ld1 + nc;
+                  if (nc + 16 <= ep.N) {
+                    reinterpret_cast<uint4*>(S)[0] = make_uint4(sp[0], sp[1], sp[2], sp[3]);
+                    reinterpret_cast<uint4*>(S)[1] = make_uint4(sp[4], sp[5], sp[6], sp[7]);
+                  } else {
+#pragma unroll
+                    for (int k = 0; k < 16; ++k)
+                      if (nc + k < ep.N) S[k] = __ushort_as_bfloat16((unsigned short)(sp[k >> 1] >> (16 * (k & 1))));
+                  }
+                }
+              }
+            } else {  // DGRAD: dZ = acc * sigma'(Z) (prefetched S), fp32 values feed the bias partials
+              if (row_ok && nc < ep.N) {
+                if (nc + 16 <= ep.N) {
+                  const uint4 s0 = spre[pi][0], s1 = spre[pi][1];
+                  const __nv_bfloat162* sv0 = reinterpret_cast<const __nv_bfloat162*>(&s0);
+                  const __nv_bfloat162* sv1 = reinterpret_cast<const __nv_bfloat162*>(&s1);
+#pragma unroll
+                  for (int qq = 0; qq < 4; ++qq) {
+                    const float2 a = __bfloat1622float2(sv0[qq]);
+                    v[2 * qq] *= a.x;
+                    v[2 * qq + 1] *= a.y;
+                    const float2 b2 = __bfloat1622float2(sv1[qq]);
+                    v[8 + 2 * qq] *= b2.x;
+                    v[8 + 2 * qq + 1] *= b2.y;
+                  }
+                } else {
+                  const __nv_bfloat16* S = static_cast<const __nv_bfloat16*>(ep.aux) + (int64_t)r * ep.ldaux;
+#pragma unroll
+                  for (int k = 0; k < 16; ++k) v[k] = nc + k < ep.N ? v[k] * __bfloat162float(S[nc + k]) : 0.f;
+                }
+              } else {
+#pragma unroll
+                for (int k = 0; k < 16; ++k) v[k] = 0.f;
+              }
+              uint32_t pk[8];
+#pragma unroll
+              for (int qq = 0; qq < 8; ++qq) pk[qq] = pack_bf16x2(v[2 * qq], v[2 * qq + 1]);
+              stage16_box(sbuf, rl, cc, pk);
+              if (ep.bpart_out) {
+                const float t = warp_colsum16(v, lane);
+                if (!(lane & 1)) red[q * BN + c + colsum16_col(lane)] = t;
+              }
+            }
+          }
+          fence_proxy_async();
+          epi_bar_sync();  // the chunk is staged
+          if (et == 0) {
+            if (n0 + 64 * j < ep.N) {
+              tma_store_2d(x.tmO0, sbuf, n0 + 64 * j, m0);
+              if (TO::NOUT == 2 && ep.out1) tma_store_2d(x.tmO1, sbuf + TC_BM * 128, n0 + 64 * j, m0);
+            }
+            tma_store_commit();  // one group per chunk (empty groups keep the count)
+          }
+        }
       } else if (active) {
 #pragma unroll
         for (int cc = 0; cc < HALF; cc += 16) {
@@ -389,13 +518,9 @@ __device__ __forceinline__ void tc_epilogue_tile(const EpiArgs& ep, const EpiTil
                 uint32_t pk[8];
 #pragma unroll
                 for (int qq = 0; qq < 8; ++qq) pk[qq] = pack_bf16x2(v[2 * qq], v[2 * qq + 1]);
-                if (TO::on) {
-                  stage16<TO::NBOX>(sout, 0, rl, c, pk);
-                } else {
-                  uint4* D = reinterpret_cast<uint4*>(static_cast<__nv_bfloat16*>(ep.out0) + (int64_t)r * ep.ld0 + nc);
-                  D[0] = make_uint4(pk[0], pk[1], pk[2], pk[3]);
-                  D[1] = make_uint4(pk[4], pk[5], pk[6], pk[7]);
-                }
+                uint4* D = reinterpret_cast<uint4*>(static_cast<__nv_bfloat16*>(ep.out0) + (int64_t)r * ep.ld0 + nc);
+                D[0] = make_uint4(pk[0], pk[1], pk[2], pk[3]);
+                D[1] = make_uint4(pk[4], pk[5], pk[6], pk[7]);
               } else {
                 const __nv_bfloat16* S = static_cast<const __nv_bfloat16*>(ep.aux) + (int64_t)r * ep.ldaux;
                 __nv_bfloat16* D = static_cast<__nv_bfloat16*>(ep.out0) + (int64_t)r * ep.ld0;
@@ -403,16 +528,10 @@ __device__ __forceinline__ void tc_epilogue_tile(const EpiArgs& ep, const EpiTil
                 for (int j = 0; j < 16; ++j) {
                   if (nc + j < ep.N) {
                     v[j] *= __bfloat162float(S[nc + j]);
-                    if (!TO::on) D[nc + j] = __float2bfloat16_rn(v[j]);
+                    D[nc + j] = __float2bfloat16_rn(v[j]);
                   } else {
                     v[j] = 0.f;
                   }
-                }
-                if (TO::on) {  // columns >= N are clipped by the TMA store
-                  uint32_t pk[8];
-#pragma unroll
-                  for (int qq = 0; qq < 8; ++qq) pk[qq] = pack_bf16x2(v[2 * qq], v[2 * qq + 1]);
-                  stage16<TO::NBOX>(sout, 0, rl, c, pk);
                 }
               }
             } else {
@@ -441,19 +560,6 @@ __device__ __forceinline__ void tc_epilogue_tile(const EpiArgs& ep, const EpiTil
             for (int qq = 0; qq < 4; ++qq)
               sts128(pa + qq * 16, __float_as_uint(v[4 * qq]), __float_as_uint(v[4 * qq + 1]),
                      __float_as_uint(v[4 * qq + 2]), __float_as_uint(v[4 * qq + 3]));
-          } else if (TO::on && EPI == EPI_FWD_SIG) {
-            // all rows / columns staged; rows >= M and columns >= N are clipped by the TMA store
-            uint32_t hp[8], sp[8];
-#pragma unroll
-            for (int qq = 0; qq < 8; ++qq) {
-              float h0, d0, h1, d1;
-              sigmoid_d_fast(v[2 * qq] + sb[c + 2 * qq], h0, d0);
-              sigmoid_d_fast(v[2 * qq + 1] + sb[c + 2 * qq + 1], h1, d1);
-              hp[qq] = pack_bf16x2(h0, h1);
-              sp[qq] = pack_bf16x2(d0, d1);
-            }
-            stage16<TO::NBOX>(sout, 0, rl, c, hp);
-            if (ep.out1) stage16<TO::NBOX>(sout, 1, rl, c, sp);
           } else if (row_ok) {
             if (EPI == EPI_FWD_SIG && full) {
               uint32_t hp[8], sp[8];
@@ -502,20 +608,6 @@ __device__ __forceinline__ void tc_epilogue_tile(const EpiArgs& ep, const EpiTil
           }
         }
       }
-      if (TO::on) {  // staged tile complete -> one thread issues the bulk stores
-        fence_proxy_async();
-        epi_bar_sync();
-        if (et == 0) {
-#pragma unroll
-          for (int o = 0; o < TO::NOUT; ++o) {
-            if (o == 1 && !ep.out1) continue;
-#pragma unroll
-            for (int bx = 0; bx < TO::NBOX; ++bx)
-              tma_store_2d(o == 0 ? x.tmO0 : x.tmO1, sout + (size_t)(o * TO::NBOX + bx) * TC_BM * 128, n0 + bx * 64, m0);
-          }
-          tma_store_commit();
-        }
-      }
       if (EPI == EPI_DGRAD_SIG && ep.bpart_out) {
         if (!TO::on) epi_bar_sync();
         for (int cc = et; cc < BN && n0 + cc < ep.N; cc += TC_EPI_THREADS)
@@ -555,13 +647,13 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
   uint64_t* tmem_full_bar = empty_bar + STAGES;   // [2]: accumulator a ready (MMA -> epilogue)
   uint64_t* tmem_empty_bar = tmem_full_bar + 2;    // [2]: accumulator a drained (epilogue -> MMA)
   uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(tmem_empty_bar + 2);
-  __shared__ float red[4 * BN];    // per-quadrant column sums (bias-gradient partials)
+  __shared__ float red[EPI == EPI_DGRAD_SIG || EPI == EPI_HEAD_XENT ? 4 * BN : 4];  // bias-gradient partials
   __shared__ float sbias[2][BN];   // bias of the tile, double-buffered across tiles
   __shared__ __align__(16) float dzs[EPI == EPI_HEAD_XENT ? TC_BM * 16 : 4];  // dZ_L rows (fused head dX)
 
   const int warp = threadIdx.x >> 5;
   const int lane = threadIdx.x & 31;
-  unsigned long long* dbg = ep.dbg ? ep.dbg + 12 * ((size_t)(blockIdx.z * gridDim.y + blockIdx.y) * gridDim.x + blockIdx.x) : nullptr;
+  unsigned long long* dbg = ep.dbg ? ep.dbg + 32 * ((size_t)(blockIdx.z * gridDim.y + blockIdx.y) * gridDim.x + blockIdx.x) : nullptr;
   HB_STAMP(dbg && threadIdx.x == 0, dbg[0]);
   // Tiles: persistent CTAs walk tiles t = blockIdx.x, +gridDim.x, ... (n fastest, so CTAs running
   // together share the A row panel in L2).  Split-K launches (gridDim.z > 1) are one tile per CTA.
@@ -701,6 +793,7 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
     else
       umma_commit(&tmem_full_bar[acc]);  // accumulator ready (arrives even if num_kb == 0)
     HB_STAMP(dbg && i == 0, dbg[3]);
+    HB_STAMP(dbg && i < 5, dbg[12 + i]);  // tuning: MMAs of tile i issued
     }
   } else if (warp >= 4) {
     // ===== epilogue (8 warps): TMEM -> registers -> fused epilogue -> global =====
@@ -715,7 +808,9 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
         m_tile = blockIdx.x;
         n_tile = blockIdx.y;
       }
+      HB_STAMP(dbg && threadIdx.x == 128 && i < 5, dbg[17 + i]);  // tuning: epilogue of tile i starts
       tc_epilogue_tile<BN, EPI>(ep, ectx, m_tile, n_tile, i & 1, i);
+      HB_STAMP(dbg && threadIdx.x == 128 && i < 5, dbg[22 + i]);  // tuning: epilogue of tile i done
     }
   }
 
