@@ -1215,8 +1215,15 @@ int step_graph(hb_worker* w, const void* X, int64_t ldx, int64_t x_rows, const i
     int rc = run_step(w, X, ldx, HB_BF16, x_rows, y, w->d_off, b, lr, false, s);
     cudaGraph_t graph = nullptr;
     cudaError_t ce = cudaStreamEndCapture(s, &graph);
+    cudaStreamCaptureStatus cs = cudaStreamCaptureStatusNone;
+    if (cudaStreamIsCapturing(s, &cs) == cudaSuccess && cs != cudaStreamCaptureStatusNone) {
+      cudaGraph_t g2 = nullptr;  // an invalidated capture: end it so the stream is usable again
+      cudaStreamEndCapture(s, &g2);
+      if (g2) cudaGraphDestroy(g2);
+    }
     if (rc) {
       if (graph) cudaGraphDestroy(graph);
+      cudaGetLastError();
       return rc;
     }
     if (ce != cudaSuccess) return fail(HB_ECUDA, std::string("graph capture: ") + cudaGetErrorString(ce));
