@@ -213,7 +213,11 @@ def main():
     ap.add_argument("--policy", default="adaptive", choices=["adaptive", "minibatch"])
     ap.add_argument("--eta0", type=float, default=None, help="lr at b0 (default: 0.01 for C4, 0.05 otherwise)")
     ap.add_argument("--b0", type=int, default=32)
-    ap.add_argument("--merges", type=int, default=1, help="replica merges per epoch (N > 1)")
+    ap.add_argument("--merges", type=int, default=1, help="replica merges per epoch (N > 1, --sync merge)")
+    ap.add_argument("--sync", default="merge", choices=["merge", "async"],
+                    help="N > 1: NCCL replica merges at the coordinator's merge points, or NEXT f2: every "
+                         "update also lands on every peer replica (CUDA IPC peer memory, atomic adds)")
+    ap.add_argument("--async-scale", type=float, default=1.0, help="f2: stale-update damping of peer updates")
     ap.add_argument("--n", type=int, default=0, help="rows per GPU (default: the config's N)")
     ap.add_argument("--e2e-steps", type=int, default=3)
     ap.add_argument("--no-cpu-baseline", action="store_true")
@@ -355,10 +359,17 @@ def main():
         dist.barrier()
         if rank != 0:
             coord = hb.Coord(name, pol, N, world, rank)
-        uid = hbd.share_bytes(hb.Comm.unique_id() if rank == 0 else None)
-        comm = hb.Comm(uid, world, rank, local)
-        model.merge_begin()
-        pol.coord, pol.comm, pol.merges_per_epoch = coord, comm, args.merges
+        pol.coord = coord
+        if args.sync == "merge":
+            uid = hbd.share_bytes(hb.Comm.unique_id() if rank == 0 else None)
+            comm = hb.Comm(uid, world, rank, local)
+            model.merge_begin()
+            pol.comm, pol.merges_per_epoch = comm, args.merges
+        else:  # f2: asynchronous cross-GPU updates through peer memory (atomic, no merge round)
+            handles = [None] * world
+            dist.all_gather_object(handles, model.ipc_handle())
+            model.set_option("update", hb.HB_UPDATE_ATOMIC)
+            model.attach_ipc_peers([h for r, h in enumerate(handles) if r != rank], scale=args.async_scale)
 
     flush = torch.empty(256 << 20, dtype=torch.uint8, device=dev)
 
@@ -558,6 +569,7 @@ def main():
             "config": {"workload": cfg["workload"], "workers": desc, "rows_per_gpu": Nper, "rows_global": N,
                        "step": "one hogbatch_run epoch over the global data set (one coordinator for all GPUs)",
                        "eta0_at_b0": [eta0, args.b0], "merges_per_epoch": args.merges if world > 1 else 0,
+                       "sync": args.sync if world > 1 else None,
                        "l2": "flushed between timed steps (256 MiB write); the data set (3 GB per 72,309 rows) "
                              "exceeds the 126 MB L2"},
             "tc_peak_frac": value * F / (world * peaks["bf16_sus"] * 1e12),
@@ -578,6 +590,9 @@ def main():
         comm.close()
     if world > 1:
         dist.barrier()
+        if args.sync == "async":
+            model.attach_ipc_peers([])
+            dist.barrier()
         if coord is not None:
             coord.close()
         dist.destroy_process_group()

@@ -353,6 +353,24 @@ int hb_merge_replicas(hb_model* m, hb_worker* const* workers, int32_t n, float g
 int hb_merge_schedule(int64_t N, int32_t merges_per_epoch, const int32_t* batches, int64_t n_batches,
                       int32_t* mid_epoch_out, int32_t* total_out);
 
+/* ---- asynchronous cross-replica Hogbatch (NEXT f2; "reference replicas",
+ * L175 "the learning rate can be decreased" for stale replicas) ---------------------------
+ * After mlp_attach_peers / mlp_attach_ipc_peers, every SGD update this model applies (the dW
+ * epilogue's W -= lr * dW and the bias update) is ALSO added, scaled by `scale` (stale-gradient
+ * damping, 0 <= scale; 1 = none), to each peer replica's fp32 master with an atomic add —
+ * peer-to-peer over NVLink, no round barrier — and the peer's bf16 shadow element is rewritten
+ * from the value that add produced.  Peers are models of identical shape: in this process
+ * (mlp_attach_peers: another model on this GPU, or on a peer-accessible GPU) or in another
+ * process (mlp_ipc_handle exports a model's 128-byte handle pair; mlp_attach_ipc_peers maps up to
+ * 7 of them).  Updates made while the peers are detached are not propagated; n = 0 detaches.
+ * bf16 models only.  Concurrent updates of one replica race as in Hogwild [L128, L170]; under
+ * HB_UPDATE_ATOMIC only the shadow refresh is racy.  (NVLink multicast — one multimem.red per
+ * update for all replicas — is the intended transport; it needs a multicast domain, which the
+ * development pool's one-GPU leases do not have.) */
+int mlp_attach_peers(hb_model* m, hb_model* const* peers, int32_t n, float scale);
+int mlp_ipc_handle(const hb_model* m, uint8_t out[128]);
+int mlp_attach_ipc_peers(hb_model* m, const uint8_t* handles, int32_t n, float scale);
+
 /* ---- multi-GPU replica merge over NCCL (future work L277) -------- */
 int hb_nccl_unique_id(uint8_t out[128]);
 int hb_comm_create(const uint8_t id[128], int32_t nranks, int32_t rank, int32_t device,

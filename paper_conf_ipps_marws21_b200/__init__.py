@@ -79,6 +79,22 @@ class MLP:
         Call before creating workers."""
         self.set_option("fused_min_batch", min_batch)
 
+    def attach_peers(self, peers, scale: float = 1.0) -> None:
+        """``mlp_attach_peers``: every update of this model also goes to each peer replica (NEXT f2)."""
+        hs = (C.c_void_p * max(1, len(peers)))(*[p.h.value for p in peers])
+        _check(lib.mlp_attach_peers(self.h, hs, len(peers), scale))
+
+    def ipc_handle(self) -> bytes:
+        """``mlp_ipc_handle``: 128 bytes another process passes to ``attach_ipc_peers``."""
+        buf = (C.c_uint8 * 128)()
+        _check(lib.mlp_ipc_handle(self.h, buf))
+        return bytes(buf)
+
+    def attach_ipc_peers(self, handles, scale: float = 1.0) -> None:
+        blob = b"".join(handles)
+        buf = (C.c_uint8 * max(1, len(blob)))(*blob)
+        _check(lib.mlp_attach_ipc_peers(self.h, buf, len(handles), scale))
+
     def merge_replicas(self, workers, gamma: float = 1.0) -> None:
         """``hb_merge_replicas``: integrate the deep replicas among `workers` into this model."""
         hs = (C.c_void_p * len(workers))(*[w.h.value for w in workers])

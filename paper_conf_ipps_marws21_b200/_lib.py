@@ -32,7 +32,7 @@ EXPORTS = ("hb_last_error", "hb_abi_version", "hb_device_ok", "mlp_create", "mlp
            "hb_nccl_unique_id", "hb_comm_create", "hb_comm_destroy", "hb_merge_begin", "hb_merge",
            "hb_merge_replicas", "hb_kernel_launches", "hb_prof_enable", "hb_prof_read", "hb_merge_schedule",
            "mlp_worker_create_nested", "hb_coord_create", "hb_coord_destroy", "hb_coord_reset",
-           "hb_coord_schedule", "hb_coord_idle")
+           "hb_coord_schedule", "hb_coord_idle", "mlp_attach_peers", "mlp_ipc_handle", "mlp_attach_ipc_peers")
 # tuning build only (include/hogbatch_tuning.h): not exported by the product library
 TUNING_EXPORTS = ("hb_bench_gemm", "hb_bench_gemm_phases", "hb_rc_trace", "hb_bench_step")
 PROF_LAYERS = 16
@@ -121,6 +121,9 @@ def load():
         "hb_merge_begin": ([VP], C.c_int),
         "hb_merge": ([VP, VP, F, VP], C.c_int),
         "hb_merge_replicas": ([VP, P(VP), I32, F], C.c_int),
+        "mlp_attach_peers": ([VP, P(VP), I32, F], C.c_int),
+        "mlp_ipc_handle": ([VP, P(C.c_uint8)], C.c_int),
+        "mlp_attach_ipc_peers": ([VP, P(C.c_uint8), I32, F], C.c_int),
         "hb_coord_create": ([C.c_char_p, P(Policy), I64, I32, I32, P(VP)], C.c_int),
         "hb_coord_destroy": ([VP], C.c_int),
         "hb_coord_reset": ([VP, P(Policy), I64], C.c_int),

@@ -13,6 +13,8 @@
 
 namespace hb {
 
+constexpr int HB_MAX_PEERS = 7;
+
 enum { EPI_FWD_SIG = 0, EPI_FWD_LOGITS = 1, EPI_DGRAD_SIG = 2, EPI_WGRAD_SGD = 3, EPI_WGRAD_STORE = 4,
        EPI_HEAD_XENT = 5 };
 
@@ -49,6 +51,13 @@ struct EpiArgs {
   int pair;                    // host-side: dW GEMM on CTA pairs (tcgen05 cta_group::2) when eligible
   int no_pdl;                  // host-side: launch without programmatic dependent launch
   int atomic;                  // WGRAD_SGD: W -= lr * dW with atomic adds (HB_UPDATE_ATOMIC)
+  // asynchronous cross-replica Hogbatch (NEXT f2, mlp_attach_peers): every update of W / b is also
+  // added, scaled by pscale (stale-gradient damping [L175]), to each peer replica's fp32 master
+  // with an atomic add (peer-to-peer over NVLink), and the peer's bf16 shadow element rewritten
+  int npeer;
+  float pscale;
+  int64_t pm_off[HB_MAX_PEERS];  // peer master - this master (elements)
+  int64_t ps_off[HB_MAX_PEERS];  // peer shadow - this shadow (elements)
   // softmax cross-entropy head fused into the output-layer GEMM (C <= 16):
   const int32_t* y;     // labels (dataset base when yoff != nullptr)
   const int* yoff;      // device row offset of the batch (graph replay), nullable
@@ -67,6 +76,15 @@ struct EpiArgs {
 __device__ __forceinline__ uint32_t pack_bf16x2(float a, float b) {
   __nv_bfloat162 t = __floats2bfloat162_rn(a, b);
   return *reinterpret_cast<uint32_t*>(&t);
+}
+
+// f2: add -lr * pscale * g to element idx of every peer replica (and rewrite its shadow element)
+__device__ __forceinline__ void peer_push1(const EpiArgs& ep, float* w_local, __nv_bfloat16* sh_local, float g) {
+  const float d = __fmul_rn(-ep.lr * ep.pscale, g);
+  for (int p = 0; p < ep.npeer; ++p) {
+    const float nv = atomicAdd(w_local + ep.pm_off[p], d) + d;
+    if (sh_local) sh_local[ep.ps_off[p]] = __float2bfloat16_rn(nv);
+  }
 }
 
 template <typename T>
@@ -112,6 +130,7 @@ __device__ __forceinline__ void epi_elem(const EpiArgs& ep, int r, int n, float 
       ep.master[idx] = w;
     }
     if (ep.shadow) ep.shadow[idx] = __float2bfloat16_rn(w);
+    if (ep.npeer) peer_push1(ep, ep.master + idx, ep.shadow ? ep.shadow + idx : nullptr, v);
   } else {  // EPI_WGRAD_STORE
     int64_t idx = ep.transposed ? (int64_t)n * ep.ldw + r : (int64_t)r * ep.ldw + n;
     static_cast<float*>(ep.out0)[idx] = v;
@@ -212,6 +231,10 @@ __device__ __forceinline__ void epi_row16_bf16(const EpiArgs& ep, int r, int n0,
     uint4* Sh = reinterpret_cast<uint4*>(ep.shadow + (int64_t)r * ep.ldw + n0);
     Sh[0] = make_uint4(sp[0], sp[1], sp[2], sp[3]);
     Sh[1] = make_uint4(sp[4], sp[5], sp[6], sp[7]);
+    if (ep.npeer) {
+#pragma unroll
+      for (int k = 0; k < 16; ++k) peer_push1(ep, ep.master + (int64_t)r * ep.ldw + n0 + k, ep.shadow + (int64_t)r * ep.ldw + n0 + k, v[k]);
+    }
   } else {
 #pragma unroll
     for (int j = 0; j < 16; ++j) epi_elem<EPI, __nv_bfloat16, false>(ep, r, n0 + j, v[j]);

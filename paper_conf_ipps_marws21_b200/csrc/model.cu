@@ -953,6 +953,14 @@ static int launch_wgrad(hb_worker* w, int l, const void* X, int64_t ldx, int64_t
   ep.pair = m->opt_dw_pair;
   ep.no_pdl = !m->opt_pdl;
   ep.atomic = m->opt_update == HB_UPDATE_ATOMIC;
+  if (!grads_only && !m->peers.empty()) {  // f2: the update also goes to every peer replica
+    ep.npeer = (int)m->peers.size();
+    ep.pscale = m->peer_scale;
+    for (int p = 0; p < ep.npeer; ++p) {
+      ep.pm_off[p] = m->peers[p].first - m->master;
+      ep.ps_off[p] = m->peers[p].second - m->shadow;
+    }
+  }
   ep.bias_upd = m->master + Ly.b_off;
   ep.bias_grad = grads_only ? w->grads + Ly.b_off : nullptr;
   ep.ws = ws;
@@ -1448,6 +1456,8 @@ int mlp_create(const int32_t* dims, int32_t n_dims, int32_t activation, int32_t 
 int mlp_destroy(hb_model* m) {
   if (!m) return HB_OK;
   cudaSetDevice(m->device);
+  cudaDeviceSynchronize();
+  for (void* p : m->ipc_opened) cudaIpcCloseMemHandle(p);
   if (m->eval) mlp_worker_destroy(m->eval);
   cudaFree(m->master);
   cudaFree(m->shadow);
@@ -1716,6 +1726,75 @@ int mlp_set_params(hb_model* m, const float* host_src, int64_t n) {
     HB_CUDA_TRY(cudaGetLastError());
   }
   HB_CUDA_TRY(cudaStreamSynchronize(m->stream));
+  return HB_OK;
+}
+
+static void detach_peers(hb_model* m) {
+  for (void* p : m->ipc_opened) cudaIpcCloseMemHandle(p);
+  m->ipc_opened.clear();
+  m->peers.clear();
+}
+
+int mlp_attach_peers(hb_model* m, hb_model* const* peers, int32_t n, float scale) {
+  HB_CHECK_ARG(m && n >= 0 && n <= HB_MAX_PEERS && (n == 0 || peers), "0 <= n <= 7 peers");
+  HB_CHECK_ARG(scale >= 0.f, "scale must be >= 0");
+  if (m->prec != HB_PREC_BF16) return fail(HB_EUNSUPPORTED, "peer replicas: bf16 models only");
+  for (int i = 0; i < n; ++i) {
+    HB_CHECK_ARG(peers[i] && peers[i] != m && peers[i]->dims == m->dims && peers[i]->prec == m->prec,
+                 "peers must be other models of identical shape");
+    if (peers[i]->device != m->device) {  // another GPU of this process: peer-to-peer access
+      int can = 0;
+      cudaDeviceCanAccessPeer(&can, m->device, peers[i]->device);
+      if (!can) return fail(HB_EUNSUPPORTED, "no peer-to-peer access between the models' devices");
+      HB_CUDA_TRY(cudaSetDevice(m->device));
+      cudaError_t e = cudaDeviceEnablePeerAccess(peers[i]->device, 0);
+      if (e != cudaSuccess && e != cudaErrorPeerAccessAlreadyEnabled) return fail(HB_ECUDA, "enable peer access");
+      cudaGetLastError();
+    }
+  }
+  detach_peers(m);
+  for (int i = 0; i < n; ++i) m->peers.push_back({peers[i]->master, peers[i]->shadow});
+  m->peer_scale = scale;
+  return HB_OK;
+}
+
+int mlp_ipc_handle(const hb_model* m, uint8_t out[128]) {
+  HB_CHECK_ARG(m && out, "null arg");
+  if (m->prec != HB_PREC_BF16) return fail(HB_EUNSUPPORTED, "peer replicas: bf16 models only");
+  HB_CUDA_TRY(cudaSetDevice(m->device));
+  cudaIpcMemHandle_t hm, hs;
+  static_assert(sizeof(cudaIpcMemHandle_t) == 64, "ipc handle size");
+  HB_CUDA_TRY(cudaIpcGetMemHandle(&hm, m->master));
+  HB_CUDA_TRY(cudaIpcGetMemHandle(&hs, m->shadow));
+  std::memcpy(out, &hm, 64);
+  std::memcpy(out + 64, &hs, 64);
+  return HB_OK;
+}
+
+int mlp_attach_ipc_peers(hb_model* m, const uint8_t* handles, int32_t n, float scale) {
+  HB_CHECK_ARG(m && n >= 0 && n <= HB_MAX_PEERS && (n == 0 || handles), "0 <= n <= 7 peers");
+  HB_CHECK_ARG(scale >= 0.f, "scale must be >= 0");
+  if (m->prec != HB_PREC_BF16) return fail(HB_EUNSUPPORTED, "peer replicas: bf16 models only");
+  HB_CUDA_TRY(cudaSetDevice(m->device));
+  HB_CUDA_TRY(cudaDeviceSynchronize());
+  detach_peers(m);
+  for (int i = 0; i < n; ++i) {
+    cudaIpcMemHandle_t hm, hs;
+    std::memcpy(&hm, handles + 128 * i, 64);
+    std::memcpy(&hs, handles + 128 * i + 64, 64);
+    void *pm = nullptr, *ps = nullptr;
+    if (cudaIpcOpenMemHandle(&pm, hm, cudaIpcMemLazyEnablePeerAccess) != cudaSuccess ||
+        cudaIpcOpenMemHandle(&ps, hs, cudaIpcMemLazyEnablePeerAccess) != cudaSuccess) {
+      cudaGetLastError();
+      if (pm) cudaIpcCloseMemHandle(pm);
+      detach_peers(m);
+      return fail(HB_ECUDA, "cudaIpcOpenMemHandle of a peer replica failed");
+    }
+    m->ipc_opened.push_back(pm);
+    m->ipc_opened.push_back(ps);
+    m->peers.push_back({static_cast<float*>(pm), static_cast<__nv_bfloat16*>(ps)});
+  }
+  m->peer_scale = scale;
   return HB_OK;
 }
 

@@ -86,6 +86,11 @@ struct hb_model {
   size_t stage_y_cap = 0;
   cudaStream_t copy_stream = nullptr;
   std::vector<cudaEvent_t> stage_ev;
+  // asynchronous cross-replica updates (NEXT f2): peer replicas' fp32 master / bf16 shadow
+  // (identical layout) that every update of this model is also added to, scaled by peer_scale
+  std::vector<std::pair<float*, __nv_bfloat16*>> peers;
+  std::vector<void*> ipc_opened;  // cudaIpcOpenMemHandle mappings to close
+  float peer_scale = 1.f;
   // CSR datasets: device copies of the sparse arrays (reused across calls)
   int64_t* csr_ptr = nullptr;
   int32_t* csr_idx = nullptr;

@@ -148,6 +148,7 @@ __device__ __forceinline__ void bias_reduce_update(const EpiArgs& ep, int lo, in
         atomicAdd(ep.bias_upd + bi, __fmul_rn(-ep.lr, acc));
       else
         ep.bias_upd[bi] += __fmul_rn(-ep.lr, acc);
+      if (ep.npeer) peer_push1(ep, ep.bias_upd + bi, nullptr, acc);  // biases have no shadow
     }
     else
       ep.bias_grad[bi] = acc;
@@ -927,6 +928,14 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
           }
           uint2 sh = make_uint2(pack_bf16x2(w.x, w.y), pack_bf16x2(w.z, w.w));
           *reinterpret_cast<uint2*>(ep.shadow + (int64_t)gm * ep.ldw + gn) = sh;
+          if (ep.npeer) {
+            float* wl = ep.master + (int64_t)gm * ep.ldw + gn;
+            __nv_bfloat16* sl = ep.shadow + (int64_t)gm * ep.ldw + gn;
+            peer_push1(ep, wl, sl, acc.x);
+            peer_push1(ep, wl + 1, sl + 1, acc.y);
+            peer_push1(ep, wl + 2, sl + 2, acc.z);
+            peer_push1(ep, wl + 3, sl + 3, acc.w);
+          }
         } else {
 #pragma unroll
           for (int j = 0; j < 4; ++j)

@@ -207,3 +207,105 @@ def test_two_processes_share_one_coordinator_on_one_gpu():
         assert served[0][0] == 0 and all(a[0] + a[1] == b_[0] for a, b_ in zip(served, served[1:]))
         assert {t[2] for t in trace if t[1] == e and t[9]} == {0, 1}
     assert any(t[6] in ("double", "halve") for t in trace)  # the adaptive rule acted across processes
+
+
+# ---- NEXT f2: asynchronous cross-replica Hogbatch (every update also lands on the peer replicas) ----
+
+@pytest.mark.parametrize("dims,b", [([54, 256, 128, 7], 256), ([54, 512, 512, 512, 7], 4096)])
+def test_peer_replicas_receive_every_update(dims, b):
+    # replicas A and B attached to each other: A's step lands on A (read-modify-write) and on B
+    # (atomic add), B's next step reads the updated B, ... — after alternating steps both equal, bit
+    # for bit, ONE model that took the same steps in the same order (the fused-chain shape at
+    # b = 4096 covers the split-K dW epilogue)
+    _gpu()
+    X, y = dataset("covtype", 4 * b, seed=3)
+    y = (y % dims[-1]).astype(np.int32)
+    tX, ty = to_device(X, y)
+    P0 = params_to_flat(init_params(dims, seed=2))
+    A, B, Cm = hb.MLP(dims), hb.MLP(dims), hb.MLP(dims)
+    for m in (A, B, Cm):
+        m.set_params(P0)
+    A.attach_peers([B])
+    B.attach_peers([A])
+    wa, wb, wc = hb.Worker(A, b), hb.Worker(B, b), hb.Worker(Cm, b)
+    for k in range(4):
+        (wa if k % 2 == 0 else wb).step(tX[k * b:], ty[k * b:], b, 0.3)
+        torch.cuda.synchronize()
+        wc.step(tX[k * b:], ty[k * b:], b, 0.3)
+        torch.cuda.synchronize()
+    pa, pb, pc = A.get_params(), B.get_params(), Cm.get_params()
+    assert np.array_equal(pa, pb)
+    assert np.array_equal(pa, pc)
+    # damping [L175]: with scale 1/2 the peer receives exactly half of every update (to fp32 rounding)
+    A.set_params(P0)
+    B.set_params(P0)
+    A.attach_peers([B], scale=0.5)
+    B.attach_peers([])
+    wa.step(tX, ty, b, 0.3)
+    torch.cuda.synchronize()
+    da, db_ = A.get_params().astype(np.float64) - P0, B.get_params().astype(np.float64) - P0
+    assert np.abs(db_ - 0.5 * da).max() <= 2.0 ** -22 * np.abs(P0).max() + 1e-12
+    assert np.abs(da).max() > 0
+
+
+_PEER_PROC = r"""
+import os, sys, time, json
+sys.path.insert(0, os.getcwd())
+import numpy as np, torch
+import paper_conf_ipps_marws21_b200 as hb
+from tests.helpers import dataset, init_params, params_to_flat, to_device
+rank, name, tmp = int(sys.argv[1]), sys.argv[2], sys.argv[3]
+def wait_for(path):
+    t0 = time.time()
+    while not os.path.exists(path):
+        if time.time() - t0 > 120: raise RuntimeError("peer did not show up: " + path)
+        time.sleep(0.01)
+dims, N = [54, 128, 128, 7], 16384
+X, y = dataset("covtype", N, seed=0)
+tX, ty = to_device(X, y)
+m = hb.MLP(dims)
+m.set_params(params_to_flat(init_params(dims, seed=2)))
+m.set_option("update", hb.HB_UPDATE_ATOMIC)
+open(f"{tmp}/h{rank}.tmp", "wb").write(m.ipc_handle()); os.rename(f"{tmp}/h{rank}.tmp", f"{tmp}/h{rank}")
+wait_for(f"{tmp}/h{1 - rank}")
+m.attach_ipc_peers([open(f"{tmp}/h{1 - rank}", "rb").read()])
+specs = [hb.WorkerSpec(256, 1024, 1024), hb.WorkerSpec(64, 512, 64)]
+w = hb.Worker(m, specs[rank].max_b)
+pol = hb.Policy(kind=hb.HB_ADAPTIVE, workers=specs, eta0=0.02, b0=32, first_worker=rank)
+pol.coord = hb.Coord(name, pol, N, 2, rank)
+st = hb.hogbatch_run([w], pol, tX, ty, epochs=2)
+torch.cuda.synchronize()
+open(f"{tmp}/done{rank}", "w").write("1")
+wait_for(f"{tmp}/done{1 - rank}")  # the peer's last updates into this replica have landed
+np.save(f"{tmp}/p{rank}.npy", m.get_params())
+open(f"{tmp}/saved{rank}", "w").write("1")
+wait_for(f"{tmp}/saved{1 - rank}")
+m.attach_ipc_peers([])
+pol.coord.close()
+print(json.dumps({"updates": int(st["updates"].sum()), "samples": int(st["total_samples"])}))
+"""
+
+
+def test_two_processes_update_each_others_replica_asynchronously(tmp_path):
+    # NEXT f2 across processes (one per GPU in production; two on the one test GPU here): each
+    # process trains its own replica under ONE shared coordinator, and every update also lands in
+    # the other replica through CUDA IPC peer memory — no merge round.  With atomic updates no
+    # update is lost, so both replicas end with the same sum of updates (up to fp32 add order)
+    import json
+    import subprocess
+    import sys
+    _gpu()
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    name = f"/hbtest_{uuid.uuid4().hex[:12]}"
+    procs = [subprocess.Popen([sys.executable, "-c", _PEER_PROC, str(r), name, str(tmp_path)], cwd=root,
+                              stdout=subprocess.PIPE, stderr=subprocess.PIPE, text=True) for r in range(2)]
+    outs = [p.communicate(timeout=600) for p in procs]
+    for p, (o, e) in zip(procs, outs):
+        assert p.returncode == 0, e[-3000:]
+    res = [json.loads(o.strip().splitlines()[-1]) for o, _ in outs]
+    assert sum(r["samples"] for r in res) > 0
+    pa, pb = np.load(tmp_path / "p0.npy"), np.load(tmp_path / "p1.npy")
+    P0 = params_to_flat(init_params([54, 128, 128, 7], seed=2))
+    moved = np.linalg.norm(pa.astype(np.float64) - P0)
+    assert moved > 0
+    assert np.linalg.norm(pa.astype(np.float64) - pb) <= 1e-4 * moved
