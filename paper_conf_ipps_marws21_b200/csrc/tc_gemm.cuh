@@ -157,8 +157,16 @@ __device__ __forceinline__ void bias_reduce_update(const EpiArgs& ep, int lo, in
 
 // Grouped tile rasterisation: consecutive tile indices walk down GROUP_M row tiles before moving
 // to the next column tile, so the ~148 tiles resident at once cover a compact block of the
-// output and share both their A row panels and their B column panels through L2.
-constexpr int TC_GROUP_M = 8;
+// output and share both their A row panels and their B column panels through L2.  With ~148
+// tiles in flight a group of m row tiles spans ~148/m column tiles, so per wave the A panels are
+// re-read tiles_n*m/148 times and the B panels tiles_m/m times; for the C4 layer-1 GEMMs (64 x 16
+// and 32 x 82 tiles) the traffic minimum is near m = 17.  GROUP_M = 16 measured 1.60 GB of DRAM
+// traffic per layer-1 wgrad+SGD launch against 2.08 GB at 8, and +1.1 % C4 samples/s
+// (profiles/r02_group_m.txt).
+#ifndef HB_GROUP_M
+#define HB_GROUP_M 16
+#endif
+constexpr int TC_GROUP_M = HB_GROUP_M;
 __device__ __forceinline__ void tile_coords(int t, int tiles_m, int tiles_n, int& m_tile, int& n_tile) {
   const int per_group = TC_GROUP_M * tiles_n;
   const int g = t / per_group;
