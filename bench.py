@@ -221,6 +221,7 @@ def main():
     ap.add_argument("--n", type=int, default=0, help="rows per GPU (default: the config's N)")
     ap.add_argument("--e2e-steps", type=int, default=3)
     ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--opt", action="append", default=[], help="model option key=value (HB_OPT_*, e.g. gemm_pair=1)")
     ap.add_argument("--no-prof", action="store_true")
     ap.add_argument("--ttt-epochs", type=int, default=None,
                     help="epochs per algorithm for time-to-target (0 disables; N=1 only)")
@@ -292,6 +293,9 @@ def main():
     torch.cuda.synchronize()
 
     model = hb.MLP(dims, precision="bf16", seed=0, device=local)
+    for kv in args.opt:  # per-model launch options (include/hogbatch.h HB_OPT_*)
+        k, v = kv.split("=")
+        model.set_option(k, int(v))
     params0 = params_to_flat(init_params(dims, seed=2))
     model.set_params(params0)
     big_max = 8192

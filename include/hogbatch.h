@@ -213,11 +213,16 @@ int mlp_fused_path(const hb_model* m, int32_t batch, int32_t* cluster_size);
  *                           separated by grid barriers (narrow nets: widths <= 1024, C <= 16,
  *                           L <= 8; plain workers); 0 = per-layer launches (default: measured
  *                           slower on B200 — 86 vs 58 us per C2 step at b = 32)
+ *   HB_OPT_GEMM_PAIR        1 = forward, dX and unsplit dW GEMMs with >= 256 output columns, an
+ *                           even number of 128-row tiles and >= 74 tile pairs (one wave) run as
+ *                           persistent CTA pairs (tcgen05 cta_group::2, 256 x 256 tiles; default);
+ *                           0 = one CTA per 128-row tile
  * Unknown key or out-of-range value -> HB_EINVAL. */
 enum {
   HB_OPT_FUSED_MIN_BATCH = 0, HB_OPT_ROWCHAIN = 1, HB_OPT_RC_CLUSTER = 2, HB_OPT_BWD_OVERLAP = 3,
   HB_OPT_HEAD_FUSE = 4, HB_OPT_DW_PAIR = 5, HB_OPT_PDL = 6, HB_OPT_GRAPHS = 7, HB_OPT_INFLIGHT = 8,
-  HB_OPT_STAGE_ROWS = 9, HB_OPT_UPDATE = 10, HB_OPT_STEP_KERNEL_MAX_B = 11
+  HB_OPT_STAGE_ROWS = 9, HB_OPT_UPDATE = 10, HB_OPT_STEP_KERNEL_MAX_B = 11,
+  HB_OPT_GEMM_PAIR = 12
 };
 enum { HB_UPDATE_HOGWILD = 0, HB_UPDATE_ATOMIC = 1 };
 int mlp_set_option(hb_model* m, int32_t key, int64_t value);

@@ -21,7 +21,8 @@ HB_CREDIT_DISPATCH, HB_CREDIT_COMPLETION = 0, 1
 HB_UPDATE_HOGWILD, HB_UPDATE_ATOMIC = 0, 1
 # mlp_set_option keys
 OPTIONS = {"fused_min_batch": 0, "rowchain": 1, "rc_cluster": 2, "bwd_overlap": 3, "head_fuse": 4, "dw_pair": 5,
-           "pdl": 6, "graphs": 7, "inflight": 8, "stage_rows": 9, "update": 10, "step_kernel_max_b": 11}
+           "pdl": 6, "graphs": 7, "inflight": 8, "stage_rows": 9, "update": 10, "step_kernel_max_b": 11,
+           "gemm_pair": 12}
 ACTIONS = ("none", "halve", "double", "clamp_lo", "clamp_hi")
 
 # every symbol include/hogbatch.h declares (checked by tests/test_abi.py)

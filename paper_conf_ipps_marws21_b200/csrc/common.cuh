@@ -289,6 +289,11 @@ __device__ __forceinline__ void mbar_arrive_expect_tx_remote(uint32_t cluster_ba
                "r"(bytes)
                : "memory");
 }
+// arrive on an mbarrier of a CTA of the cluster (shared::cluster address), releasing this thread's
+// prior memory operations (and, after tcgen05.fence::before_thread_sync, its TMEM reads) at cluster scope
+__device__ __forceinline__ void mbar_arrive_cluster(uint32_t cluster_bar) {
+  asm volatile("mbarrier.arrive.release.cluster.shared::cluster.b64 _, [%0];" ::"r"(cluster_bar) : "memory");
+}
 // bulk copy local shared memory -> shared memory of another CTA of the cluster, completion
 // (bytes) signalled on that CTA's mbarrier
 __device__ __forceinline__ void bulk_copy_s2cluster(uint32_t cluster_dst, const void* src, uint32_t bytes,
@@ -364,6 +369,31 @@ __device__ __forceinline__ void sigmoid_d_fast(float z, float& h, float& d) {
   const float es = e * s;
   h = z >= 0.f ? s : es;
   d = es * s;
+}
+
+// sigmoid_d_fast of two elements, z = acc + bias, on the packed fp32x2 pipe (FADD2 / FFMA2 / FMUL2,
+// sm_100): the same IEEE operations per element in the same order — the negations are exact and
+// fma(e, -1, -1) = -(1 + e) rounded — so the results are bitwise those of two sigmoid_d_fast
+// calls, at about half the FP instructions (the tile epilogues are issue-bound on them)
+__device__ __forceinline__ void sigmoid_d_fast2(float a0, float a1, float b0, float b1, float& h0, float& h1,
+                                                float& d0, float& d1) {
+  const float2 z = __fadd2_rn(make_float2(a0, a1), make_float2(b0, b1));
+#ifdef HB_FAKE_SIG  // tuning only (wrong numerics): the epilogue's cost without the sigmoid math
+  h0 = z.x; h1 = z.y; d0 = z.x * 0.25f; d1 = z.y * 0.25f;
+  return;
+#endif
+  const float2 e = make_float2(ex2_ftz(fabsf(z.x) * -1.4426950408889634f), ex2_ftz(fabsf(z.y) * -1.4426950408889634f));
+  const float2 ny = __ffma2_rn(e, make_float2(-1.0f, -1.0f), make_float2(-1.0f, -1.0f));
+  const float2 two = make_float2(2.0f, 2.0f);
+  float2 s = __ffma2_rn(make_float2(8.0f / 17.0f, 8.0f / 17.0f), ny, make_float2(24.0f / 17.0f, 24.0f / 17.0f));
+  s = __fmul2_rn(s, __ffma2_rn(ny, s, two));
+  s = __fmul2_rn(s, __ffma2_rn(ny, s, two));
+  const float2 es = __fmul2_rn(e, s);
+  const float2 dd = __fmul2_rn(es, s);
+  h0 = z.x >= 0.f ? s.x : es.x;
+  h1 = z.y >= 0.f ? s.y : es.y;
+  d0 = dd.x;
+  d1 = dd.y;
 }
 
 }  // namespace hb

@@ -49,6 +49,7 @@ struct EpiArgs {
   unsigned long long* dbg;  // tuning only: per-CTA phase timestamps (globaltimer ns), nullable
   int force_bn, force_splits;  // host-side launch choices for dW GEMMs (0 = heuristic)
   int pair;                    // host-side: dW GEMM on CTA pairs (tcgen05 cta_group::2) when eligible
+  int fwd_pair;                // host-side: forward / dX GEMM on persistent CTA pairs when eligible
   int no_pdl;                  // host-side: launch without programmatic dependent launch
   int atomic;                  // WGRAD_SGD: W -= lr * dW with atomic adds (HB_UPDATE_ATOMIC)
   // asynchronous cross-replica Hogbatch (NEXT f2, mlp_attach_peers): every update of W / b is also

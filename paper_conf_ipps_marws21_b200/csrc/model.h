@@ -60,6 +60,7 @@ struct hb_model {
   int opt_bwd_overlap = 1;          // HB_OPT_BWD_OVERLAP: dW_l on a second stream, overlapping dX_{l-1}
   int opt_head_fuse = 0;            // HB_OPT_HEAD_FUSE: output layer's dX in the head epilogue
   int opt_dw_pair = 0;              // HB_OPT_DW_PAIR: split-K dW GEMMs on CTA pairs (cta_group::2)
+  int opt_gemm_pair = 1;            // HB_OPT_GEMM_PAIR: forward / dX / unsplit dW GEMMs on persistent CTA pairs
   int opt_pdl = 1;                  // HB_OPT_PDL: programmatic dependent launch
   int opt_graphs = 1;               // HB_OPT_GRAPHS: hogbatch_run replays one CUDA graph per (b, lr)
   int opt_inflight = 0;             // HB_OPT_INFLIGHT: steps a worker may enqueue ahead (0 = auto)

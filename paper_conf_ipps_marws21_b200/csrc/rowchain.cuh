@@ -491,8 +491,8 @@ __global__ void __launch_bounds__(RC_THREADS, 1) rowchain_kernel(const __grid_co
                 d0 = h0 * 0.25f;
                 d1 = h1 * 0.25f;
 #else
-                sigmoid_d_fast(__uint_as_float(raw[g2 * 16 + 2 * k]) + bb[2 * k], h0, d0);
-                sigmoid_d_fast(__uint_as_float(raw[g2 * 16 + 2 * k + 1]) + bb[2 * k + 1], h1, d1);
+                sigmoid_d_fast2(__uint_as_float(raw[g2 * 16 + 2 * k]), __uint_as_float(raw[g2 * 16 + 2 * k + 1]),
+                                bb[2 * k], bb[2 * k + 1], h0, h1, d0, d1);
 #endif
                 pk[k] = pack_bf16x2(h0, h1);
                 sp[k] = pack_bf16x2(d0, d1);

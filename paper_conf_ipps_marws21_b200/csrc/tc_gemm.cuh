@@ -44,7 +44,13 @@ constexpr int TC_THREADS = 128 + TC_EPI_THREADS;   // 4 control warps + the epil
 // The tile is written in 64-column chunks through TWO staging buffers: chunk j is staged while the
 // bulk stores of chunk j-1 drain, so the staging costs 2 x NOUT x 16 KB whatever BN (B200, C3
 // 8192x1024x1024: 256-wide tiles with a whole-tile staged epilogue were epilogue-bound).
-template <int BN, int EPI>
+#ifndef HB_PAIR_NBUF
+#define HB_PAIR_NBUF 1
+#endif
+#ifndef HB_PAIR_NOUT
+#define HB_PAIR_NOUT 1
+#endif
+template <int BN, int EPI, bool PAIR = false>
 struct TmaOut {
 #ifndef HB_TMA_OUT_MAX_BN
 #define HB_TMA_OUT_MAX_BN 256
@@ -54,13 +60,17 @@ struct TmaOut {
   static constexpr int NCHUNK = BN / 64;                   // 64-column chunks per tile
   // 256-wide tiles keep a 4-deep operand ring: one staging buffer, and the forward's sigma' stash
   // is written directly (only H goes through TMA); narrower tiles double-buffer H and S
-  static constexpr int NBUF = BN == 128 ? 2 : 1;
-  static constexpr int NOUT = EPI == EPI_FWD_SIG && BN <= 128 ? 2 : 1;  // staged outputs
+  // (CTA pairs load half of B per stage, so their ring has room for more staging)
+  static constexpr int NBUF = BN == 128 || (PAIR && HB_PAIR_NBUF == 2) ? 2 : 1;
+  static constexpr int NOUT = EPI == EPI_FWD_SIG && (BN <= 128 || (PAIR && HB_PAIR_NOUT == 2)) ? 2 : 1;  // staged outputs
   static constexpr int BYTES = on ? NBUF * NOUT * TC_BM * 128 : 0;
 };
 
 // PAIR: a CTA pair (cluster x = 2) computes a 256 x BN tile with tcgen05.mma.cta_group::2 — each
 // CTA loads its own 128 A rows and HALF of the B tile (BN/2 rows), the leader issues the MMAs.
+// Two uses: split-K dW GEMMs (one tile per pair, clusters (2, 1, S)) and persistent forward / dX
+// GEMMs (clusters (2, 1, 1) walking 256 x 256 tiles): per SM the pair halves the B operand's shared-
+// memory fill and tensor-core read and the L2 traffic per flop against a 128 x 256 tile.
 template <int BN, bool B_MN, int EPI = EPI_WGRAD_SGD, bool PAIR = false>
 struct TcCfg {
   static constexpr int A_BYTES = TC_BM * TC_BK * 2;                     // 16 KB
@@ -68,7 +78,7 @@ struct TcCfg {
   static constexpr int B_ROWS = B_MN ? (B_TILE < 64 ? 64 : B_TILE) : B_TILE;  // MN-major loads 64-wide boxes
   static constexpr int B_BYTES = B_ROWS * TC_BK * 2;
   static constexpr int STAGE_BYTES = A_BYTES + B_BYTES;
-  static constexpr int OUT_BYTES = TmaOut<BN, EPI>::BYTES;
+  static constexpr int OUT_BYTES = TmaOut<BN, EPI, PAIR>::BYTES;
 #ifndef HB_RING_BYTES
 #define HB_RING_BYTES (210 * 1024)
 #endif
@@ -216,12 +226,13 @@ struct EpiTileCtx {
   int splits, num_kb;
   int warp, lane;
   unsigned long long* dbg;
+  uint32_t empty_remote;  // CTA pair: shared::cluster address of the leader's tmem_empty_bar (0: local)
 };
 
-template <int BN, int EPI>
+template <int BN, int EPI, bool PAIR = false>
 __device__ __forceinline__ void tc_epilogue_tile(const EpiArgs& ep, const EpiTileCtx& x, int m_tile, int n_tile,
                                                  int acc, int i, int acc_stride = BN) {
-  using TO = TmaOut<BN, EPI>;
+  using TO = TmaOut<BN, EPI, PAIR>;
   const int warp = x.warp, lane = x.lane;
   const int q = warp & 3;
   const int h = (warp - 4) >> 2;  // column part 0..TC_EPI_PARTS-1
@@ -408,30 +419,28 @@ __device__ __forceinline__ void tc_epilogue_tile(const EpiArgs& ep, const EpiTil
             }
             epi_bar_sync();
           }
+          // this warp's columns of the chunk: every TMEM load in flight before the one wait
+          uint32_t rawc[CW / 16][16];
+#pragma unroll
+          for (int g = 0; g < CW / 16; ++g)
+            if (n0 + 64 * j + h * CW + 16 * g < ep.N) tmem_ld_32x32b_x16(tbase + (uint32_t)(64 * j + h * CW + 16 * g), rawc[g]);
+          tmem_ld_wait();
+          HB_STAMP(dbg && et == 0 && i == 1 && j == 0, dbg[31]);  // tuning: first chunk loaded (tile 1)
 #pragma unroll
           for (int g = 0; g < CW / 16; ++g, ++pi) {
             const int cc = h * CW + 16 * g;  // column within the chunk
             const int c = 64 * j + cc;       // column within the tile
             const int nc = n0 + c;
             float v[16];
-            if (nc < ep.N) {  // warp-uniform
-              uint32_t raw[16];
-              tmem_ld_32x32b_x16(tbase + (uint32_t)c, raw);
-              tmem_ld_wait();
 #pragma unroll
-              for (int k = 0; k < 16; ++k) v[k] = __uint_as_float(raw[k]);
-            } else {
-#pragma unroll
-              for (int k = 0; k < 16; ++k) v[k] = 0.f;
-            }
+            for (int k = 0; k < 16; ++k) v[k] = nc < ep.N ? __uint_as_float(rawc[g][k]) : 0.f;
             if (EPI == EPI_FWD_SIG) {
               // all rows / columns staged; rows >= M and columns >= N are clipped by the TMA store
               uint32_t hp[8], sp[8];
 #pragma unroll
               for (int qq = 0; qq < 8; ++qq) {
                 float h0, d0, h1, d1;
-                sigmoid_d_fast(v[2 * qq] + sb[c + 2 * qq], h0, d0);
-                sigmoid_d_fast(v[2 * qq + 1] + sb[c + 2 * qq + 1], h1, d1);
+                sigmoid_d_fast2(v[2 * qq], v[2 * qq + 1], sb[c + 2 * qq], sb[c + 2 * qq + 1], h0, h1, d0, d1);
                 hp[qq] = pack_bf16x2(h0, h1);
                 sp[qq] = pack_bf16x2(d0, d1);
               }
@@ -485,6 +494,7 @@ __device__ __forceinline__ void tc_epilogue_tile(const EpiArgs& ep, const EpiTil
               }
             }
           }
+          HB_STAMP(dbg && et == 0 && i == 1 && j < 4, dbg[27 + j]);  // tuning: chunk j computed (tile 1)
           fence_proxy_async();
           epi_bar_sync();  // the chunk is staged
           if (et == 0) {
@@ -575,8 +585,7 @@ __device__ __forceinline__ void tc_epilogue_tile(const EpiArgs& ep, const EpiTil
 #pragma unroll
               for (int qq = 0; qq < 8; ++qq) {
                 float h0, d0, h1, d1;
-                sigmoid_d_fast(v[2 * qq] + sb[c + 2 * qq], h0, d0);
-                sigmoid_d_fast(v[2 * qq + 1] + sb[c + 2 * qq + 1], h1, d1);
+                sigmoid_d_fast2(v[2 * qq], v[2 * qq + 1], sb[c + 2 * qq], sb[c + 2 * qq + 1], h0, h1, d0, d1);
                 hp[qq] = pack_bf16x2(h0, h1);
                 sp[qq] = pack_bf16x2(d0, d1);
               }
@@ -636,7 +645,12 @@ __device__ __forceinline__ void tc_epilogue_tile(const EpiArgs& ep, const EpiTil
     // release this accumulator to the MMA warp (all TMEM reads of the tile have completed)
     tc_fence_before();
     __syncwarp();
-    if (lane == 0) mbar_arrive(&tmem_empty_bar[acc]);
+    if (lane == 0) {
+      if (x.empty_remote)  // CTA pair: the leader's MMAs write both CTAs' accumulators
+        mbar_arrive_cluster(x.empty_remote + (uint32_t)(acc * 8));
+      else
+        mbar_arrive(&tmem_empty_bar[acc]);
+    }
 }
 
 template <int BN, bool A_MN, bool B_MN, int EPI, bool PAIR = false>
@@ -645,9 +659,10 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
                    const __grid_constant__ CUtensorMap tmO0, const __grid_constant__ CUtensorMap tmO1,
                    int K, const int* __restrict__ offA, const int* __restrict__ offB, EpiArgs ep) {
   using Cfg = TcCfg<BN, B_MN, EPI, PAIR>;
-  using TO = TmaOut<BN, EPI>;
+  using TO = TmaOut<BN, EPI, PAIR>;
   constexpr int STAGES = Cfg::STAGES;
-  static_assert(!PAIR || (A_MN && B_MN && BN >= 128 && !TO::on), "CTA pairs: split-K dW GEMMs only");
+  static_assert(!PAIR || (A_MN && B_MN && BN >= 128 && !TO::on) || (!A_MN && BN == 256),
+                "CTA pairs: split-K dW GEMMs or persistent 256 x 256 forward / dX tiles");
   extern __shared__ uint8_t smem_raw[];
   uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
   uint8_t* sout = smem + STAGES * Cfg::STAGE_BYTES;  // TMA-store staging [NOUT][NBOX][128 rows x 128 B]
@@ -668,12 +683,15 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
   // together share the A row panel in L2).  Split-K launches (gridDim.z > 1) are one tile per CTA.
   const int tiles_n = (ep.N + BN - 1) / BN;
   const int tiles_m = (ep.M + TC_BM - 1) / TC_BM;
-  const int num_tiles = tiles_n * tiles_m;
   // split-K (dW GEMMs with K = batch): the gridDim.z CTAs of one output tile form a cluster,
   // each accumulates k-blocks [kb_lo, kb_hi) in its own TMEM
   const int splits = gridDim.z;
-  const int t_first = splits == 1 ? (int)blockIdx.x : (int)(blockIdx.y * gridDim.x + blockIdx.x);
-  const int t_step = splits == 1 ? (int)gridDim.x : num_tiles;
+  // persistent CTA pairs walk 256-row pair tiles; pair p is the cluster (2p, 2p+1) along x
+  const bool pair_persist = PAIR && splits == 1;
+  const int tiles_mp = pair_persist ? (tiles_m + 1) / 2 : tiles_m;
+  const int num_tiles = tiles_n * tiles_mp;
+  const int t_first = splits == 1 ? (int)(PAIR ? blockIdx.x >> 1 : blockIdx.x) : (int)(blockIdx.y * gridDim.x + blockIdx.x);
+  const int t_step = splits == 1 ? (int)(PAIR ? gridDim.x >> 1 : gridDim.x) : num_tiles;
   const int kz = blockIdx.z;
   // CTA pair (grid x = M tiles, y = N tiles, z = splits; cluster (2, 1, S) — pairs must be along
   // the cluster's x): half = blockIdx.x & 1; cluster rank of split sp's CTA with the same half =
@@ -684,6 +702,19 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
   const int kpb = (num_kb_all + splits - 1) / splits;
   const int kb_lo = min(num_kb_all, kz * kpb);
   const int num_kb = min(num_kb_all, kb_lo + kpb) - kb_lo;
+  // output tile (m_tile, n_tile) of the CTA's tile index t
+  auto tile_of = [&](int t, int& m_tile, int& n_tile) {
+    if (PAIR && splits > 1) {  // split-K pair: one tile per CTA, from the grid
+      m_tile = blockIdx.x;
+      n_tile = blockIdx.y;
+    } else if (PAIR) {
+      int mp;
+      tile_coords(t, tiles_mp, tiles_n, mp, n_tile);
+      m_tile = 2 * mp + (int)half;
+    } else {
+      tile_coords(t, tiles_m, tiles_n, m_tile, n_tile);
+    }
+  };
 
   if (warp == 0 && lane == 0) {
     tma_prefetch_desc(&tmA);
@@ -694,7 +725,7 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
     }
     for (int a = 0; a < 2; ++a) {
       mbar_init(&tmem_full_bar[a], 1);
-      mbar_init(&tmem_empty_bar[a], TC_EPI_WARPS);  // one arrive per epilogue warp
+      mbar_init(&tmem_empty_bar[a], (PAIR ? 2 : 1) * TC_EPI_WARPS);  // one arrive per epilogue warp (of the pair)
     }
     fence_barrier_init();
   }
@@ -722,11 +753,7 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
     int it = 0;  // k-blocks issued by this CTA (ring position across tiles)
     for (int t = t_first; t < num_tiles; t += t_step) {
     int mt_, nt_;
-    tile_coords(t, tiles_m, tiles_n, mt_, nt_);
-    if (PAIR) {  // one tile per CTA: this CTA's own M tile, the pair's N tile (its half of it)
-      mt_ = blockIdx.x;
-      nt_ = blockIdx.y;
-    }
+    tile_of(t, mt_, nt_);  // PAIR: this CTA's own M tile, the pair's N tile (its half of it)
     const int m0 = mt_ * TC_BM, n0 = nt_ * BN + (int)half * Cfg::B_TILE;
     const uint32_t lead_full = PAIR ? mapa_shared(smem_u32(full_bar), 2 * kz) : 0;
     for (int kb = 0; kb < num_kb; ++kb, ++it) {
@@ -739,10 +766,18 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
       if (PAIR) {  // both CTAs' loads complete on the leader's barrier, which expects both
         const uint32_t fb = lead_full + (uint32_t)(s * 8);
         if (half == 0) mbar_arrive_expect_tx(&full_bar[s], 2 * Cfg::STAGE_BYTES);
-        tma_load_2d_pair(sA, &tmA, fb, m0, k0 + oa);
-        tma_load_2d_pair(sA + 8192, &tmA, fb, m0 + 64, k0 + oa);
+        if (!A_MN) {
+          tma_load_2d_pair(sA, &tmA, fb, k0, m0 + oa);
+        } else {
+          tma_load_2d_pair(sA, &tmA, fb, m0, k0 + oa);
+          tma_load_2d_pair(sA + 8192, &tmA, fb, m0 + 64, k0 + oa);
+        }
+        if (!B_MN) {
+          tma_load_2d_pair(sB, &tmB, fb, k0, n0 + ob);
+        } else {
 #pragma unroll
-        for (int j = 0; j < Cfg::B_ROWS / 64; ++j) tma_load_2d_pair(sB + j * 8192, &tmB, fb, n0 + 64 * j, k0 + ob);
+          for (int j = 0; j < Cfg::B_ROWS / 64; ++j) tma_load_2d_pair(sB + j * 8192, &tmB, fb, n0 + 64 * j, k0 + ob);
+        }
         continue;
       }
       mbar_arrive_expect_tx(&full_bar[s], Cfg::STAGE_BYTES);
@@ -767,7 +802,10 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
     int it = 0, i = 0;
     for (int t = t_first; t < num_tiles; t += t_step, ++i) {
     const int acc = i & 1;
-    mbar_wait(&tmem_empty_bar[acc], ((i >> 1) & 1) ^ 1);  // epilogue has drained this accumulator
+    if (PAIR)  // both CTAs' epilogues have drained this accumulator (remote arrivals)
+      mbar_wait_cluster(&tmem_empty_bar[acc], ((i >> 1) & 1) ^ 1);
+    else
+      mbar_wait(&tmem_empty_bar[acc], ((i >> 1) & 1) ^ 1);  // epilogue has drained this accumulator
     tc_fence_after();
     const uint32_t tacc = tmem_base + (uint32_t)(acc * BN);
     for (int kb = 0; kb < num_kb; ++kb, ++it) {
@@ -808,17 +846,14 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
     // ===== epilogue (8 warps): TMEM -> registers -> fused epilogue -> global =====
     // warp w reads TMEM lanes 32*(w%4).. (tile rows) and handles column half h = (w-4)/4
     const EpiTileCtx ectx{tmem_base, tmem_full_bar, tmem_empty_bar, &sbias[0][0], red, dzs, sout, smem, &tmO0,
-                          &tmO1, splits, num_kb, warp, lane, dbg};
+                          &tmO1, splits, num_kb, warp, lane, dbg,
+                          PAIR ? mapa_shared(smem_u32(tmem_empty_bar), 2 * kz) : 0u};
     int i = 0;
     for (int t = t_first; t < num_tiles; t += t_step, ++i) {
       int m_tile, n_tile;
-      tile_coords(t, tiles_m, tiles_n, m_tile, n_tile);
-      if (PAIR) {
-        m_tile = blockIdx.x;
-        n_tile = blockIdx.y;
-      }
+      tile_of(t, m_tile, n_tile);
       HB_STAMP(dbg && threadIdx.x == 128 && i < 5, dbg[17 + i]);  // tuning: epilogue of tile i starts
-      tc_epilogue_tile<BN, EPI>(ep, ectx, m_tile, n_tile, i & 1, i);
+      tc_epilogue_tile<BN, EPI, PAIR>(ep, ectx, m_tile, n_tile, i & 1, i);
       HB_STAMP(dbg && threadIdx.x == 128 && i < 5, dbg[22 + i]);  // tuning: epilogue of tile i done
     }
   }
@@ -827,7 +862,8 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
     // ---- split-K reduce-scatter: CTA kz of the cluster reduces rows [kz*rps, (kz+1)*rps) of the
     //      tile over the `splits` partials (read from every CTA's shared memory, fixed order) and
     //      applies the fused SGD update ----
-    static_assert(TC_BM * (BN + 4) * 4 <= Cfg::STAGES * Cfg::STAGE_BYTES, "split-K tile must fit the ring");
+    static_assert(!(EPI == EPI_WGRAD_SGD || EPI == EPI_WGRAD_STORE) || TC_BM * (BN + 4) * 4 <= Cfg::STAGES * Cfg::STAGE_BYTES,
+                  "split-K tile must fit the ring");
     // the fp32 master rows of this CTA's slice do not depend on the partials: fetch them (up to 8
     // float4 per thread) before the cluster barrier so their latency hides behind it
     constexpr int RED_MAXIT = 8;
@@ -835,11 +871,7 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
     {
       const int t = t_first;
       int m_tile, n_tile;
-      tile_coords(t, tiles_m, tiles_n, m_tile, n_tile);
-      if (PAIR) {
-        m_tile = blockIdx.x;
-        n_tile = blockIdx.y;
-      }
+      tile_of(t, m_tile, n_tile);
       const int tid = threadIdx.x - 128;
       const int rps = TC_BM / splits;
 #pragma unroll
@@ -858,11 +890,7 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
     if (warp >= 4) {
       const int t = t_first;
       int m_tile, n_tile;
-      tile_coords(t, tiles_m, tiles_n, m_tile, n_tile);
-      if (PAIR) {
-        m_tile = blockIdx.x;
-        n_tile = blockIdx.y;
-      }
+      tile_of(t, m_tile, n_tile);
       const int m0 = m_tile * TC_BM, n0 = n_tile * BN;
       const int tid = threadIdx.x - 128;  // 0..255
       const int rps = TC_BM / splits;
@@ -971,6 +999,8 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
   }
 
   if (TO::on && threadIdx.x == 128) tma_store_wait_all();  // bulk stores complete before exit
+  // persistent pair: neither CTA leaves while the other may still arrive on its barriers
+  if (PAIR && splits == 1) cluster_sync_all();
   HB_STAMP(dbg && threadIdx.x == 128, dbg[6]);
   tc_fence_before();
   __syncthreads();

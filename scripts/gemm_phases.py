@@ -5,7 +5,8 @@ sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
 import paper_conf_ipps_marws21_b200 as hb
 names = ["start", "prologue", "first_full", "mma_done", "epi_ready", "tmem_full", "epi_done", "exit",
          "parked", "synced", "reduced", "bias_done"] + [f"mma_issued_t{i}" for i in range(5)] + \
-        [f"epi_start_t{i}" for i in range(5)] + [f"epi_done_t{i}" for i in range(5)]
+        [f"epi_start_t{i}" for i in range(5)] + [f"epi_done_t{i}" for i in range(5)] + \
+        [f"t1_chunk{j}_computed" for j in range(4)] + ["t1_chunk0_loaded"]
 for arg in sys.argv[1:]:
     kind, M, N, K = (int(x) for x in arg.split(','))
     cap = 32 * 4096

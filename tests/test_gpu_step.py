@@ -35,10 +35,12 @@ def make(dims, prec, max_batch, seed=2, scale=1.0):
     return m, w, params
 
 
-def grads_case(dims, kind, b, prec, scale=1.0, d=None):
+def grads_case(dims, kind, b, prec, scale=1.0, d=None, opts=None, elem_tol=None):
     X, y = dataset(kind, b, d=d or dims[0], seed=7)
     y = (y % dims[-1]).astype(np.int32)
     m, w, params = make(dims, prec, b, scale=scale)
+    for k, v in (opts or {}).items():
+        m.set_option(k, v)
     tX, ty = to_device(X, y, "bf16" if prec == "bf16" else "f32")
     g, loss = w.step_grads(tX, ty, b)
     rows = w.row_losses(b)
@@ -50,7 +52,7 @@ def grads_case(dims, kind, b, prec, scale=1.0, d=None):
     scale = np.maximum(1.0, np.abs(Z[-1]).max(axis=1))
     row_err = float((np.abs(rows - ref_rows) / scale).max())
     assert row_err <= TOL[prec], ("per-row loss", row_err)
-    assert max(elem) <= TOL[prec], ("element-wise", elem)
+    assert max(elem) <= (elem_tol or TOL[prec]), ("element-wise", elem)
     return max(norm), abs(loss - l_ref) / l_ref, norm
 
 
@@ -202,6 +204,34 @@ def test_batch_equal_to_max_batch_and_ragged_tiles():
     # b = max_batch with a ragged last row tile (b % 128 != 0) and ragged widths
     e, le, errs = grads_case([100, 136, 72, 3], "gauss", 1000, "bf16", d=100)
     assert e <= TOL["bf16"], errs
+
+
+@pytest.mark.parametrize("dims,kind,b,elem_tol", [
+    ([300, 1024, 1024, 1024, 2], "w8a", 5000, None),   # forward + dX pairs
+    # forward + unsplit dW pairs; a 4096-wide sigmoid layer on unit-norm realsim rows is in its
+    # near-linear regime, where bf16 rounding gives element-wise errors ~1.5e-2 (R25,
+    # the C4 bound 2.5e-2; normwise stays <= 1e-2)
+    ([4000, 4096, 2], "realsim", 2200, 2.5e-2)])
+def test_cta_pair_gemms(dims, kind, b, elem_tol):
+    # HB_OPT_GEMM_PAIR (default on): forward / dX / unsplit dW GEMMs run as persistent CTA pairs
+    # (cta_group::2, 256 x 256 tiles over two SMs, ragged last pair tile).  Same k order per output
+    # element as the one-CTA tiles, so the gradients must agree bitwise with the one-CTA path, and
+    # with the oracle
+    e, le, errs = grads_case(dims, kind, b, "bf16", opts={"gemm_pair": 1, "rowchain": 0}, elem_tol=elem_tol)
+    assert e <= TOL["bf16"], errs
+    assert le <= TOL["bf16"]
+    X, y = dataset(kind, b, d=dims[0], seed=7)
+    y = (y % dims[-1]).astype(np.int32)
+    tX, ty = to_device(X, y, "bf16")
+    out = []
+    for pair in (0, 1):
+        m, w, _ = make(dims, "bf16", b)
+        m.set_option("rowchain", 0)
+        m.set_option("gemm_pair", pair)
+        g, loss = w.step_grads(tX, ty, b)
+        out.append((np.array(g, copy=True), loss))
+    assert np.array_equal(out[0][0], out[1][0])
+    assert out[0][1] == out[1][1]
 
 
 def test_mlp_create_argument_errors():
