@@ -1997,14 +1997,14 @@ static int bench_gemm_impl(int32_t kind, int32_t M, int32_t N, int32_t K, int32_
   if (cudaMalloc(&A, arows * lda * 2) || cudaMalloc(&B, brows * ldb * 2) || cudaMalloc(&O, out_elems * 2) ||
       cudaMalloc(&S, out_elems * 2) || cudaMalloc(&W, out_elems * 4) || cudaMalloc(&Wsh, out_elems * 2) ||
       cudaMalloc(&bias, ldo * 4 + 64) || cudaMalloc(&ws, (size_t)148 * TC_BM * 256 * 4) ||
-      cudaMalloc(&bp, (size_t)((std::max(M, K) + 127) / 128) * ldo * 4 + 4096))
+      cudaMalloc(&bp, (size_t)((std::max(M, K) + 127) / 128) * std::max<int64_t>(ldo, M) * 4 + 4096))
     return fail(HB_ENOMEM, "bench alloc");
   cudaMemset(A, 0, arows * lda * 2);
   cudaMemset(B, 0, brows * ldb * 2);
   cudaMemset(W, 0, out_elems * 4);
   cudaMemset(bias, 0, ldo * 4 + 64);
   cudaMemset(S, 0, out_elems * 2);
-  cudaMemset(bp, 0, (size_t)((std::max(M, K) + 127) / 128) * ldo * 4 + 4096);
+  cudaMemset(bp, 0, (size_t)((std::max(M, K) + 127) / 128) * std::max<int64_t>(ldo, M) * 4 + 4096);  // wgrad: ldp = M
   cudaStream_t s;
   cudaStreamCreate(&s);
   EpiArgs ep{};
@@ -2082,7 +2082,8 @@ static int bench_gemm_impl(int32_t kind, int32_t M, int32_t N, int32_t K, int32_
   cudaStreamDestroy(s);
   cudaFree(A); cudaFree(B); cudaFree(O); cudaFree(S); cudaFree(W); cudaFree(Wsh); cudaFree(bias); cudaFree(ws);
   cudaFree(bp);
-  if (!rc && cudaGetLastError() != cudaSuccess) return fail(HB_ECUDA, "bench kernel failed");
+  const cudaError_t err = cudaGetLastError();
+  if (!rc && err != cudaSuccess) return fail(HB_ECUDA, cudaGetErrorString(err));
   return rc;
 }
 
