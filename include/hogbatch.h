@@ -217,12 +217,18 @@ int mlp_fused_path(const hb_model* m, int32_t batch, int32_t* cluster_size);
  *                           even number of 128-row tiles and >= 74 tile pairs (one wave) run as
  *                           persistent CTA pairs (tcgen05 cta_group::2, 256 x 256 tiles; default);
  *                           0 = one CTA per 128-row tile
+ *   HB_OPT_HEAD_KERNEL      1 = the output layer of a net with C <= 8 classes (and at least one
+ *                           hidden layer) runs on the per-layer path as ONE streaming CUDA-core pass
+ *                           over H_{L-1} / sigma'_{L-1}: logits, softmax cross-entropy, dZ_{L-1}
+ *                           (Eq. (2)) and dW_L / db_L from fp32 dZ_L, then a small reduction kernel
+ *                           applies Eq. (3) to W_L, b_L (default); 0 = tensor-core head GEMM,
+ *                           output-layer dX GEMM and dW GEMM (R24 split-precision dZ_L)
  * Unknown key or out-of-range value -> HB_EINVAL. */
 enum {
   HB_OPT_FUSED_MIN_BATCH = 0, HB_OPT_ROWCHAIN = 1, HB_OPT_RC_CLUSTER = 2, HB_OPT_BWD_OVERLAP = 3,
   HB_OPT_HEAD_FUSE = 4, HB_OPT_DW_PAIR = 5, HB_OPT_PDL = 6, HB_OPT_GRAPHS = 7, HB_OPT_INFLIGHT = 8,
   HB_OPT_STAGE_ROWS = 9, HB_OPT_UPDATE = 10, HB_OPT_STEP_KERNEL_MAX_B = 11,
-  HB_OPT_GEMM_PAIR = 12
+  HB_OPT_GEMM_PAIR = 12, HB_OPT_HEAD_KERNEL = 13
 };
 enum { HB_UPDATE_HOGWILD = 0, HB_UPDATE_ATOMIC = 1 };
 int mlp_set_option(hb_model* m, int32_t key, int64_t value);
@@ -335,7 +341,8 @@ enum {
   HB_PROF_OTHER = 6,      /* loss reduction, shadow refresh, merge kernels              */
   HB_PROF_ROWCHAIN = 7,   /* fused per-row-block forward + softmax-xent + dX chain (narrow nets) */
   HB_PROF_STEPK = 8,      /* persistent small-batch step kernel (all GEMMs of a step in one launch) */
-  HB_PROF_N = 9,
+  HB_PROF_HEAD = 9,       /* small-C output layer in one CUDA-core pass: logits + softmax-CE + dX + dW partials */
+  HB_PROF_N = 10,
   HB_PROF_LAYERS = 16     /* per-layer breakdown: entry HB_PROF_N + cls * HB_PROF_LAYERS + layer (0-based) */
 };
 typedef struct hb_prof_entry {

@@ -22,7 +22,7 @@ HB_UPDATE_HOGWILD, HB_UPDATE_ATOMIC = 0, 1
 # mlp_set_option keys
 OPTIONS = {"fused_min_batch": 0, "rowchain": 1, "rc_cluster": 2, "bwd_overlap": 3, "head_fuse": 4, "dw_pair": 5,
            "pdl": 6, "graphs": 7, "inflight": 8, "stage_rows": 9, "update": 10, "step_kernel_max_b": 11,
-           "gemm_pair": 12}
+           "gemm_pair": 12, "head_kernel": 13}
 ACTIONS = ("none", "halve", "double", "clamp_lo", "clamp_hi")
 
 # every symbol include/hogbatch.h declares (checked by tests/test_abi.py)
@@ -38,7 +38,7 @@ EXPORTS = ("hb_last_error", "hb_abi_version", "hb_device_ok", "mlp_create", "mlp
 TUNING_EXPORTS = ("hb_bench_gemm", "hb_bench_gemm_phases", "hb_rc_trace", "hb_bench_step")
 PROF_LAYERS = 16
 PROF_CLASSES = ("fwd_gemm", "head_gemm", "softmax_xent", "dgrad_gemm", "wgrad_sgd_gemm", "bias_sgd", "other",
-                "rowchain", "step_kernel")
+                "rowchain", "step_kernel", "head_kernel")
 
 
 class WorkerPolicy(C.Structure):

@@ -22,6 +22,7 @@
 #include "tc_gemm.cuh"
 #include "rowchain.cuh"
 #include "step_kernel.cuh"
+#include "head.cuh"
 
 namespace hb {
 
@@ -608,6 +609,52 @@ static int64_t ld_dz(const hb_worker* w, int l) {
   return l == (int)w->m->layers.size() - 1 ? w->ld_dzL : w->m->layers[l].ldo;
 }
 
+// ---- small-C output layer as one CUDA-core pass (head.cuh) ---------------------------------
+// Shape of the launch for a batch of b rows: CMAX classes (2/4/8), CPT 8-column chunks per
+// thread, T threads, RB rows per round; a contiguous range of `rows` rows per CTA, grid CTAs
+// (at most the resident capacity: one 256-thread CTA per SM, more for narrower rows).
+struct HeadCfg {
+  bool ok = false;
+  int cmax = 0, cw = 0, cpt = 0, T = 0, rb = 0, rows = 0, grid = 0;
+};
+static HeadCfg head_shape(const hb_model* m, int b) {
+  HeadCfg h;
+  const int L = (int)m->layers.size();
+  if (m->prec != HB_PREC_BF16 || L < 2 || b <= 0) return h;
+  const Layer& Ly = m->layers[L - 1];
+  const int C = Ly.n_out, n = Ly.n_in;
+  if (C > HEAD_MAX_C) return h;
+  h.cmax = C <= 2 ? 2 : C <= 4 ? 4 : 8;
+  const bool narrow = n <= 1024;  // HeadShape: 8-byte chunks, 32 / CMAX rows per round, one CTA per SM
+  h.cw = narrow ? 4 : 8;
+  const int maxt = narrow ? 256 : h.cmax <= 4 ? 512 : 256;  // HeadShape::MAXT
+  const int nc = (n + h.cw - 1) / h.cw;
+  h.T = std::min(maxt, (nc + 31) / 32 * 32);
+  h.cpt = (nc + h.T - 1) / h.T;
+  if (h.cmax * h.cpt > (h.cmax <= 4 ? 4 : 8)) return h;  // register budget (wider rows: tensor-core head)
+  h.rb = narrow ? 32 / h.cmax : std::max(1, std::min(16 / h.cmax, 4 / h.cpt));
+  static int nsm = 0;
+  if (!nsm) {
+    int dev = 0;
+    cudaGetDevice(&dev);
+    cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, dev);
+    if (nsm <= 0) nsm = 148;
+  }
+  const int rounds = (b + h.rb - 1) / h.rb;
+  const int cap = narrow ? nsm : nsm * std::max(1, maxt / h.T);
+  const int g = std::min(rounds, cap);
+  h.rows = (rounds + g - 1) / g * h.rb;
+  h.grid = (b + h.rows - 1) / h.rows;
+  h.ok = true;
+  return h;
+}
+// the per-layer step uses it unless disabled, the model is recorded for the persistent step
+// kernel (g_plan) or the worker has no partial buffer
+static HeadCfg head_cfg(const hb_worker* w, int b) {
+  if (!w->m->opt_head_kernel || !w->hws || g_plan) return HeadCfg{};
+  return head_shape(w->m, b);
+}
+
 static int act_dt(const hb_model* m) { return m->prec == HB_PREC_BF16 ? HB_BF16 : HB_F32; }
 static size_t act_size(const hb_model* m) { return m->prec == HB_PREC_BF16 ? 2 : 4; }
 
@@ -639,6 +686,8 @@ static void free_worker_buffers(hb_worker* w) {
   w->h_off = nullptr;
   cudaFree(w->ws);
   w->ws = nullptr;
+  cudaFree(w->hws);
+  w->hws = nullptr;
   for (cudaEvent_t e : w->ev_bwd) cudaEventDestroy(e);
   w->ev_bwd.clear();
   if (w->ev_join2) cudaEventDestroy(w->ev_join2);
@@ -706,12 +755,16 @@ static int alloc_worker(hb_model* m, int max_b, cudaStream_t stream, bool own, h
   const int C = m->layers.back().n_out;
   w->ldc = (int)round_up(C, 4);
   const int mt = (max_b + 127) / 128;
+  const HeadCfg hc = head_shape(m, max_b);  // the head kernel's grid grows with b: max_b bounds it
   for (int l = 0; l < L; ++l) {
     float* p = nullptr;
-    if (cudaMalloc(&p, (size_t)4 * mt * m->layers[l].n_out * 4) != cudaSuccess)  // x4: per-quadrant (fused path)
+    const size_t rows = std::max<size_t>((size_t)4 * mt, hc.ok ? (size_t)hc.grid : 0);  // x4: per-quadrant (fused path)
+    if (cudaMalloc(&p, rows * m->layers[l].n_out * 4) != cudaSuccess)
       return fail_free(fail(HB_ENOMEM, "bias partial alloc"));
     w->bpart.push_back(p);
   }
+  if (hc.ok && cudaMalloc(&w->hws, (size_t)hc.grid * C * (m->layers.back().n_in + 1) * 4) != cudaSuccess)
+    return fail_free(fail(HB_ENOMEM, "head partial alloc"));
   if (m->prec == HB_PREC_BF16 && cudaMalloc(&w->ws, (size_t)148 * TC_BM * 256 * 4) != cudaSuccess)
     return fail_free(fail(HB_ENOMEM, "split-K workspace alloc"));
   if (m->prec == HB_PREC_BF16) {  // second stream for the dW GEMMs (backward overlap)
@@ -874,11 +927,131 @@ static bool head_dx_fused(const hb_model* m) {
   return m->opt_head_fuse && m->layers.size() >= 2 && m->layers.back().n_out <= 16;
 }
 
+// The output layer in one pass (head.cuh): logits, softmax-CE row losses and, when training, dZ_{L-1}
+// with its bias partials (one row per CTA) and the per-CTA dW_L / db_L partials.
+template <int CMAX, int CPT, int RB, int CW>
+static int launch_head_t(const HeadCfg& hc, HeadArgs a, bool pdl, cudaStream_t s) {
+  auto kern = head_fused_kernel<CMAX, CPT, RB, CW>;
+  constexpr int kMaxSmem = 200 * 1024;
+  {
+    int dev = 0;
+    cudaGetDevice(&dev);
+    std::lock_guard<std::mutex> g(g_attr_mu);
+    auto key = std::make_pair((const void*)kern, dev);
+    if (!g_attr_done.count(key)) {
+      HB_CUDA_TRY(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, kMaxSmem));
+      g_attr_done.insert(key);
+    }
+  }
+  // ring of RB-row stages of H (and S): as deep as fits, at most HEAD_MAX_STAGES
+  const size_t stage = (size_t)RB * a.ld * 2 * (a.dz ? 2 : 1);
+  a.stages = (int)std::min<size_t>(HEAD_MAX_STAGES, kMaxSmem / stage);
+  if (a.stages < 2) return fail(HB_EUNSUPPORTED, "head kernel: rows too wide for the shared-memory ring");
+  cudaLaunchConfig_t cfg{};
+  cfg.gridDim = dim3(hc.grid);
+  cfg.blockDim = dim3(hc.T);
+  cfg.dynamicSmemBytes = stage * a.stages;
+  cfg.stream = s;
+  cudaLaunchAttribute attr[1];
+  attr[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+  attr[0].val.programmaticStreamSerializationAllowed = 1;
+  cfg.attrs = attr;
+  cfg.numAttrs = pdl ? 1 : 0;
+  HB_CUDA_TRY(cudaLaunchKernelEx(&cfg, kern, a));
+  HB_CUDA_TRY(cudaGetLastError());
+  return HB_OK;
+}
+
+static int launch_head(hb_worker* w, const HeadCfg& hc, const int32_t* y, const int* d_off, int b, bool train,
+                       cudaStream_t s) {
+  hb_model* m = w->m;
+  const int L = (int)m->layers.size();
+  const Layer& Ly = m->layers[L - 1];
+  const Layer& Lp = m->layers[L - 2];
+  HeadArgs a{};
+  a.H = static_cast<const __nv_bfloat16*>(w->H[L - 2]);
+  a.S = train ? static_cast<const __nv_bfloat16*>(w->S[L - 2]) : nullptr;
+  a.ld = Lp.ldo;
+  a.W = m->shadow + Ly.w_off;
+  a.ldw = Ly.ldw;
+  a.bias = m->master + Ly.b_off;
+  a.y = y;
+  a.yoff = d_off;
+  a.b = b;
+  a.n = Ly.n_in;
+  a.C = Ly.n_out;
+  a.rows_per_cta = hc.rows;
+  a.inv_b = 1.0f / (float)b;
+  a.row_loss = w->row_loss;
+  a.dz = train ? static_cast<__nv_bfloat16*>(w->dZ[L - 2]) : nullptr;
+  a.bpart = w->bpart[L - 2];
+  a.dwp = w->hws;
+  a.dbp = w->hws + (size_t)hc.grid * a.C * a.n;
+  ProfLayer pl(L - 1);
+  Prof pr(HB_PROF_HEAD, s);
+  const bool pdl = m->opt_pdl != 0;
+  int rc;
+  switch (hc.cw * 10000 + hc.cmax * 1000 + hc.cpt * 100 + hc.rb) {
+    case 82104: rc = launch_head_t<2, 1, 4, 8>(hc, a, pdl, s); break;
+    case 82202: rc = launch_head_t<2, 2, 2, 8>(hc, a, pdl, s); break;
+    case 84104: rc = launch_head_t<4, 1, 4, 8>(hc, a, pdl, s); break;
+    case 88102: rc = launch_head_t<8, 1, 2, 8>(hc, a, pdl, s); break;
+    case 42116: rc = launch_head_t<2, 1, 16, 4>(hc, a, pdl, s); break;
+    case 44108: rc = launch_head_t<4, 1, 8, 4>(hc, a, pdl, s); break;
+    case 48104: rc = launch_head_t<8, 1, 4, 4>(hc, a, pdl, s); break;
+    default: return fail(HB_EUNSUPPORTED, "head kernel shape");
+  }
+  if (rc) return rc;
+  // algorithmic: H read (+ S read, dZ_{L-1} written when training), labels, row losses
+  const double bn = (double)b * a.n;
+  pr.done(1, (train ? 6.0 : 2.0) * bn * a.C, bn * (train ? 6.0 : 2.0) + 8.0 * b);
+  return HB_OK;
+}
+
+// Eq. (3) for the output layer from the head kernel's partials: W_L -= lr dW_L, b_L -= lr db_L (or,
+// grads_only, the gradients stored), the same element update as the dW GEMM epilogue.
+static int launch_head_update(hb_worker* w, const HeadCfg& hc, float lr, bool grads_only, cudaStream_t s) {
+  hb_model* m = w->m;
+  const int L = (int)m->layers.size();
+  const Layer& Ly = m->layers[L - 1];
+  const int C = Ly.n_out, n = Ly.n_in;
+  EpiArgs ep{};
+  ep.master = m->master + Ly.w_off;
+  ep.shadow = m->shadow + Ly.w_off;
+  ep.ldw = Ly.ldw;
+  ep.lr = lr;
+  ep.transposed = 1;
+  ep.atomic = m->opt_update == HB_UPDATE_ATOMIC;
+  if (grads_only) ep.out0 = w->grads + Ly.w_off;
+  if (!grads_only && !m->peers.empty()) {  // f2: the update also goes to every peer replica
+    ep.npeer = (int)m->peers.size();
+    ep.pscale = m->peer_scale;
+    for (int p = 0; p < ep.npeer; ++p) {
+      ep.pm_off[p] = m->peers[p].first - m->master;
+      ep.ps_off[p] = m->peers[p].second - m->shadow;
+    }
+  }
+  ep.bias_upd = m->master + Ly.b_off;
+  ep.bias_grad = grads_only ? w->grads + Ly.b_off : nullptr;
+  const float* dwp = w->hws;
+  const float* dbp = w->hws + (size_t)hc.grid * C * n;
+  const int blocks = (int)(((int64_t)C * n + HU_X - 1) / HU_X);
+  ProfLayer pl(L - 1);
+  Prof pr(HB_PROF_WGRAD_GEMM, s);
+  if (grads_only)
+    head_update_kernel<EPI_WGRAD_STORE><<<blocks, dim3(HU_X, HU_Y), 0, s>>>(ep, dwp, dbp, hc.grid, C, n);
+  else
+    head_update_kernel<EPI_WGRAD_SGD><<<blocks, dim3(HU_X, HU_Y), 0, s>>>(ep, dwp, dbp, hc.grid, C, n);
+  HB_CUDA_TRY(cudaGetLastError());
+  pr.done(1, (double)hc.grid * C * n, (double)hc.grid * C * (n + 1) * 4.0 + (double)C * n * 10.0);
+  return HB_OK;
+}
+
 // Forward chain (Eq. (1)) of the bf16 tensor-core path.  X holds x_rows rows; the batch starts
 // at row *d_off (graph replay) or at row 0 (d_off == nullptr).  With want_grad the head writes
 // dZ_L and its bias partials; otherwise only the per-row losses (mlp_loss).
 static int forward_tc(hb_worker* w, const void* X, int64_t ldx, int64_t x_rows, const int32_t* y, const int* d_off,
-                      int b, bool want_grad, cudaStream_t s) {
+                      int b, bool want_grad, cudaStream_t s, const HeadCfg& hc) {
   hb_model* m = w->m;
   const int L = (int)m->layers.size();
   int rc;
@@ -904,7 +1077,10 @@ static int forward_tc(hb_worker* w, const void* X, int64_t ldx, int64_t x_rows, 
       continue;
     }
     // output layer + softmax cross-entropy: dZ_L = (softmax(z) - onehot(y)) / b, per-row loss
-    if (Ly.n_out <= 16) {
+    if (hc.ok) {  // small C: one CUDA-core pass, also the output layer's dX and dW partials (head.cuh)
+      rc = launch_head(w, hc, y, d_off, b, want_grad, s);
+      if (rc) return rc;
+    } else if (Ly.n_out <= 16) {
       ep.out0 = want_grad ? w->dZ[l] : nullptr;
       ep.ld0 = w->ld_dzL;
       ep.hilo = w->hilo ? 16 : 0;
@@ -1172,7 +1348,8 @@ static int step_gemms(hb_worker* w, const void* X, int64_t ldx, int64_t x_rows, 
                       int b, float lr, bool grads_only, cudaStream_t s, bool overlap) {
   hb_model* m = w->m;
   const int L = (int)m->layers.size();
-  int rc = forward_tc(w, X, ldx, x_rows, y, d_off, b, true, s);
+  const HeadCfg hc = head_cfg(w, b);
+  int rc = forward_tc(w, X, ldx, x_rows, y, d_off, b, true, s, hc);
   if (rc) return rc;
   // dW_l only has to follow dX_l (the last reader of W_l): it runs on the worker's second stream,
   // overlapping dX_{l-1} (HB_OPT_BWD_OVERLAP = 0 keeps everything on one stream)
@@ -1181,7 +1358,7 @@ static int step_gemms(hb_worker* w, const void* X, int64_t ldx, int64_t x_rows, 
     const Layer& Ly = m->layers[l];
     TcOp dZl{w->dZ[l], ld_dz(w, l), b, nullptr};
     TcOp Wl{m->shadow + Ly.w_off, Ly.ldw, 0, nullptr};
-    if (l > 0 && !(l == L - 1 && head_dx_fused(m))) {  // dZ_{l-1} = (dZ_l W_l) * sigma'(Z_{l-1}) + bias partials
+    if (l > 0 && !(l == L - 1 && (hc.ok || head_dx_fused(m)))) {  // dZ_{l-1} = (dZ_l W_l) * sigma'(Z_{l-1}) + bias partials
       const Layer& Lp = m->layers[l - 1];
       EpiArgs ep{};
     ep.no_pdl = !m->opt_pdl;
@@ -1202,7 +1379,11 @@ static int step_gemms(hb_worker* w, const void* X, int64_t ldx, int64_t x_rows, 
       HB_CUDA_TRY(cudaEventRecord(w->ev_bwd[l], s));
       HB_CUDA_TRY(cudaStreamWaitEvent(s2, w->ev_bwd[l], 0));
     }
-    rc = launch_wgrad(w, l, X, ldx, x_rows, d_off, b, lr, grads_only, s2, w->ws, (b + TC_BM - 1) / TC_BM);
+    if (l == L - 1 && hc.ok)  // the head kernel's dW_L / db_L partials, reduced and applied
+      rc = launch_head_update(w, hc, lr, grads_only, s2);
+    else  // the partials of dZ_l: per 128-row tile of its dX GEMM, or per CTA of the head kernel
+      rc = launch_wgrad(w, l, X, ldx, x_rows, d_off, b, lr, grads_only, s2, w->ws,
+                        l == L - 2 && hc.ok ? hc.grid : (b + TC_BM - 1) / TC_BM);
     if (rc) return rc;
   }
   if (s2 != s) {  // join: the step completes on the worker's stream
@@ -1550,6 +1731,7 @@ int clone_model(hb_model* m, hb_model** out) {
   r->opt_head_fuse = m->opt_head_fuse;
   r->opt_dw_pair = m->opt_dw_pair;
   r->opt_gemm_pair = m->opt_gemm_pair;
+  r->opt_head_kernel = m->opt_head_kernel;
   r->opt_pdl = m->opt_pdl;
   r->opt_graphs = m->opt_graphs;
   r->opt_inflight = m->opt_inflight;
@@ -1666,6 +1848,7 @@ int mlp_set_option(hb_model* m, int32_t key, int64_t v) {
     case HB_OPT_HEAD_FUSE: return flag(&m->opt_head_fuse);
     case HB_OPT_DW_PAIR: return flag(&m->opt_dw_pair);
     case HB_OPT_GEMM_PAIR: return flag(&m->opt_gemm_pair);
+    case HB_OPT_HEAD_KERNEL: return flag(&m->opt_head_kernel);
     case HB_OPT_PDL: return flag(&m->opt_pdl);
     case HB_OPT_GRAPHS: return flag(&m->opt_graphs);
     case HB_OPT_INFLIGHT:
@@ -1698,6 +1881,7 @@ int mlp_get_option(const hb_model* m, int32_t key, int64_t* v) {
     case HB_OPT_HEAD_FUSE: *v = m->opt_head_fuse; return HB_OK;
     case HB_OPT_DW_PAIR: *v = m->opt_dw_pair; return HB_OK;
     case HB_OPT_GEMM_PAIR: *v = m->opt_gemm_pair; return HB_OK;
+    case HB_OPT_HEAD_KERNEL: *v = m->opt_head_kernel; return HB_OK;
     case HB_OPT_PDL: *v = m->opt_pdl; return HB_OK;
     case HB_OPT_GRAPHS: *v = m->opt_graphs; return HB_OK;
     case HB_OPT_INFLIGHT: *v = m->opt_inflight; return HB_OK;
@@ -2120,7 +2304,7 @@ int mlp_loss(hb_model* m, const void* X, int64_t ldx, int32_t x_dtype, const int
     const int b = (int)std::min<int64_t>(chunk, n - r0);
     const void* Xc = static_cast<const char*>(X) + r0 * ldx * xes;
     if (bf) {
-      rc = forward_tc(w, Xc, ldx, b, y + r0, nullptr, b, false, s);
+      rc = forward_tc(w, Xc, ldx, b, y + r0, nullptr, b, false, s, head_cfg(w, b));
       if (rc) return rc;
     } else {
       const void* Ain = Xc;

@@ -61,6 +61,7 @@ struct hb_model {
   int opt_head_fuse = 0;            // HB_OPT_HEAD_FUSE: output layer's dX in the head epilogue
   int opt_dw_pair = 0;              // HB_OPT_DW_PAIR: split-K dW GEMMs on CTA pairs (cta_group::2)
   int opt_gemm_pair = 1;            // HB_OPT_GEMM_PAIR: forward / dX / unsplit dW GEMMs on persistent CTA pairs
+  int opt_head_kernel = 1;          // HB_OPT_HEAD_KERNEL: small-C output layer as one CUDA-core pass (head.cuh)
   int opt_pdl = 1;                  // HB_OPT_PDL: programmatic dependent launch
   int opt_graphs = 1;               // HB_OPT_GRAPHS: hogbatch_run replays one CUDA graph per (b, lr)
   int opt_inflight = 0;             // HB_OPT_INFLIGHT: steps a worker may enqueue ahead (0 = auto)
@@ -131,6 +132,7 @@ struct hb_worker {
   double* h_dsum = nullptr;     // pinned
   float* grads = nullptr;       // mlp_step_grads output (flat padded layout)
   float* ws = nullptr;          // split-K partial tiles of the dW GEMMs (148 x 128 x 256 fp32)
+  float* hws = nullptr;         // head kernel: per-CTA partial dW_L [grid x C x n] and db_L [grid x C]
   cudaStream_t s2 = nullptr;    // dW GEMMs overlap the next dX GEMM on this stream
   std::vector<cudaEvent_t> ev_bwd;  // per layer: "dX_l issued" (W_l no longer read)
   cudaEvent_t ev_join2 = nullptr;

@@ -51,6 +51,10 @@ def kernel_class(name):
         return EPI.get(args[3].strip(), "other") if len(args) >= 4 else "other"
     if "softmax_xent" in name:
         return "softmax_xent"
+    if "head_fused_kernel" in name:
+        return "head_kernel"
+    if "head_update_kernel" in name:
+        return "wgrad_sgd_gemm"
     return "other"
 
 
