@@ -246,7 +246,10 @@ def main():
         rows, b = (min(rows, 1024), min(b, 1024)) if dims[1] >= 4096 else (rows, b)
         v, cores, t = oracle_rate(cfg, rows, b, args.steps, args.warmup, eta0, args.b0)
         sample = f"fp64 NumPy oracle SGD steps (batch {b}) over the first {rows} rows of shard 0 of the same workload"
-        line = {"impl": "reference", "metric": METRIC, "value": v, "unit": "samples/s", "n_gpus": 0,
+        # n_gpus: the N this arm was launched for (the driver pairs the arms by N); the oracle itself
+        # runs on the host cores of rank 0 and uses no GPU
+        line = {"impl": "reference", "metric": METRIC, "value": v, "unit": "samples/s", "n_gpus": world,
+                "device": "host CPU (fp64 oracle, rank 0 only)",
                 "steps": args.steps, "warmup": args.warmup, "ms_per_step": t * 1e3, "higher_is_better": True,
                 "scaling": "weak", "vs_baseline": None, "dtype": "f64", "data": "synthetic",
                 "config": {"workload": cfg["workload"], "sample_rows_per_step": rows, "batch": b},
