@@ -241,7 +241,12 @@ static int choose_bn_wgrad(int M, int N, int K) {
   if (forced) return forced;
   if (K < 2048) return choose_bn(M, N, K);  // short K: no split-K, spread tiles over the SMs
   int bn = choose_bn_base(M, N);          // long K: split-K supplies the parallelism
-  while (bn > 64 && (long)((M + TC_BM - 1) / TC_BM) * ((N + bn - 1) / bn) * 4 < 148) bn /= 2;
+  const long mt = (M + TC_BM - 1) / TC_BM;
+  // 256-wide tiles x 4 splits filling >= 96 SMs beat narrower tiles on more SMs (operand bytes per
+  // MMA through shared memory; measured on B200, 1024 x 1024 x 8192 dW: BN 256 x 4 splits 21.6 us,
+  // BN 128 x 2 splits 26.5 us, BN 64 x 1 38.7 us — scripts/gpu_dw_sweep.sh)
+  if (N >= 256 && mt * ((N + 255) / 256) * 4 >= 96) return 256;
+  while (bn > 64 && mt * ((N + bn - 1) / bn) * 4 < 148) bn /= 2;
   return bn;
 }
 
