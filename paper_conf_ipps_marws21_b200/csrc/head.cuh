@@ -57,10 +57,10 @@ struct HeadArgs {
 
 // CMAX: classes rounded up (2, 4, 8); CW: columns per chunk (8 = 16-byte, 4 = 8-byte accesses);
 // CPT: chunks per thread (1, 2); RB rows per round, RB * CMAX <= 32 (one softmax lane per (row,
-// class) in warp 0).  Wide rows (n > 1024): CW = 8, RB = min(16 / CMAX, 4 / CPT), several CTAs'
-// rounds in flight per SM for n <= 4096 ... one 512-thread CTA for the widest; narrow rows
-// (n <= 1024): CW = 4 (twice the threads of 16-byte chunks), RB = 32 / CMAX, one CTA per SM, so
-// the per-round barriers and the softmax are paid per 32 / CMAX rows.
+// class) in warp 0).  Wide rows (n > 1024): CW = 8, RB = min(16 / CMAX, 4 / CPT), one CTA per SM
+// (up to 512 threads) with a ring of up to 4 stages; narrow rows (n <= 1024): CW = 4 (twice the
+// threads of 16-byte chunks), RB = 16 / CMAX (4 for CMAX = 8) and two CTAs per SM (100 KB rings), so one CTA's
+// barriers and softmax overlap the other's rounds.
 template <int CMAX, int CPT, int RB_, int CW_>
 struct HeadShape {
   static constexpr int RB = RB_, CW = CW_, Q = CW_ / 2;  // Q: packed bf16 pairs per chunk

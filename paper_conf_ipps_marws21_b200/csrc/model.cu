@@ -630,14 +630,14 @@ static HeadCfg head_shape(const hb_model* m, int b) {
   const int C = Ly.n_out, n = Ly.n_in;
   if (C > HEAD_MAX_C) return h;
   h.cmax = C <= 2 ? 2 : C <= 4 ? 4 : 8;
-  const bool narrow = n <= 1024;  // HeadShape: 8-byte chunks, 32 / CMAX rows per round, one CTA per SM
+  const bool narrow = n <= 1024;  // HeadShape: 8-byte chunks, 16 / CMAX rows per round, two CTAs per SM
   h.cw = narrow ? 4 : 8;
   const int maxt = narrow ? 256 : h.cmax <= 4 ? 512 : 256;  // HeadShape::MAXT
   const int nc = (n + h.cw - 1) / h.cw;
   h.T = std::min(maxt, (nc + 31) / 32 * 32);
   h.cpt = (nc + h.T - 1) / h.T;
   if (h.cmax * h.cpt > (h.cmax <= 4 ? 4 : 8)) return h;  // register budget (wider rows: tensor-core head)
-  h.rb = narrow ? 32 / h.cmax : std::max(1, std::min(16 / h.cmax, 4 / h.cpt));
+  h.rb = narrow ? (h.cmax == 8 ? 4 : 16 / h.cmax) : std::max(1, std::min(16 / h.cmax, 4 / h.cpt));
   static int nsm = 0;
   if (!nsm) {
     int dev = 0;
@@ -646,8 +646,12 @@ static HeadCfg head_shape(const hb_model* m, int b) {
     if (nsm <= 0) nsm = 148;
   }
   const int rounds = (b + h.rb - 1) / h.rb;
-  const int cap = narrow ? nsm : nsm * std::max(1, maxt / h.T);
-  const int g = std::min(rounds, cap);
+  const int cap = narrow ? 2 * nsm : nsm * std::max(1, maxt / h.T);
+  // every CTA's dW_L / bias partials (C x n floats) are re-read by the update kernel and its
+  // prologue (first bulk copies, W_L columns) is a fixed cost: at most ~2 MB of partials (but a CTA
+  // per SM), and at least 4 rounds per CTA once the batch exceeds one round per resident CTA
+  int g = std::min(rounds, std::min(cap, std::max(nsm, (int)((2 << 20) / (4L * C * n)))));
+  if (rounds > cap) g = std::max(1, std::min(g, rounds / 4));
   h.rows = (rounds + g - 1) / g * h.rb;
   h.grid = (b + h.rows - 1) / h.rows;
   h.ok = true;
@@ -937,7 +941,8 @@ static bool head_dx_fused(const hb_model* m) {
 template <int CMAX, int CPT, int RB, int CW>
 static int launch_head_t(const HeadCfg& hc, HeadArgs a, bool pdl, cudaStream_t s) {
   auto kern = head_fused_kernel<CMAX, CPT, RB, CW>;
-  constexpr int kMaxSmem = 200 * 1024;
+  // wide rows: one CTA per SM with the deepest ring that fits; narrow rows (CW = 4): two CTAs per SM
+  constexpr int kMaxSmem = CW == 4 ? 100 * 1024 : 200 * 1024;
   {
     int dev = 0;
     cudaGetDevice(&dev);
@@ -1001,8 +1006,8 @@ static int launch_head(hb_worker* w, const HeadCfg& hc, const int32_t* y, const 
     case 82202: rc = launch_head_t<2, 2, 2, 8>(hc, a, pdl, s); break;
     case 84104: rc = launch_head_t<4, 1, 4, 8>(hc, a, pdl, s); break;
     case 88102: rc = launch_head_t<8, 1, 2, 8>(hc, a, pdl, s); break;
-    case 42116: rc = launch_head_t<2, 1, 16, 4>(hc, a, pdl, s); break;
-    case 44108: rc = launch_head_t<4, 1, 8, 4>(hc, a, pdl, s); break;
+    case 42108: rc = launch_head_t<2, 1, 8, 4>(hc, a, pdl, s); break;
+    case 44104: rc = launch_head_t<4, 1, 4, 4>(hc, a, pdl, s); break;
     case 48104: rc = launch_head_t<8, 1, 4, 4>(hc, a, pdl, s); break;
     default: return fail(HB_EUNSUPPORTED, "head kernel shape");
   }

@@ -3,7 +3,7 @@ pass computing the logits, the softmax cross-entropy [PAPER.md L258], dZ_{L-1} (
 dW_L / db_L, then the in-place update of W_L, b_L (Eq. (3)) from the per-CTA partials.
 
 Against the fp64 oracle (normwise AND element-wise <= 1e-2, every row's loss, R13) for every template
-shape the launcher selects (classes rounded to 2 / 4 / 8; one or two eight-column chunks per thread),
+shape the launcher selects (classes rounded to 2 / 4 / 8; 16- or 8-byte column chunks, one or two per thread),
 ragged batches (rows not a multiple of the rows per round) and widths that are not a multiple of 8;
 and against the tensor-core head (option off) for the SGD update itself (Hogwild and atomic modes).
 """
@@ -19,17 +19,17 @@ from tests.helpers import dataset, grad_errors, init_params, params_to_flat, spl
 from tests.test_gpu_step import grads_case, make  # noqa: E402
 
 SHAPES = [
-    # dims, kind, b                         (CMAX, CPT)
-    ([54, 64, 64, 7], "covtype", 32),        # (8, 1), T = 32
+    # dims, kind, b                         template (CMAX, CPT, RB, CW), threads
+    ([54, 64, 64, 7], "covtype", 32),        # (8, 1, 4, 4), T = 32: narrow rows, 8-byte chunks
     ([54, 512, 512, 7], "covtype", 1),       # one row
-    ([54, 512, 512, 7], "covtype", 1000),    # (8, 1), T = 64
-    ([300, 1024, 1024, 2], "w8a", 777),      # (2, 1), T = 128
-    ([512, 4096, 2], "gauss", 600),          # (2, 2): the C4 head shape, T = 256
-    ([54, 2048, 4], "gauss", 301),           # (4, 1)
-    ([54, 3000, 3], "gauss", 99),            # (4, 1), T = 384: width not a multiple of 8 * T
-    ([54, 6000, 2], "gauss", 77),            # (2, 2), T = 512: two chunks per thread, the second partial
-    ([24, 60, 5], "gauss", 45),              # (8, 1), width 60: a partial 8-column chunk
-    ([24, 40, 6, 8], "gauss", 1),            # C = 8, hidden width 6 < 8
+    ([54, 512, 512, 7], "covtype", 1000),    # (8, 1, 4, 4), T = 128
+    ([300, 1024, 1024, 2], "w8a", 777),      # (2, 1, 8, 4), T = 256, two CTAs per SM
+    ([512, 4096, 2], "gauss", 600),          # (2, 1, 4, 8): the C4 head shape, T = 512
+    ([54, 2048, 4], "gauss", 301),           # (4, 1, 4, 8), T = 256
+    ([54, 3001, 3], "gauss", 99),            # (4, 1, 4, 8), T = 384: a partial 16-byte chunk (1 column)
+    ([54, 6000, 2], "gauss", 77),            # (2, 2, 2, 8), T = 512: two chunks per thread, the second partial
+    ([24, 62, 5], "gauss", 45),              # (8, 1, 4, 4): a partial 8-byte chunk (2 columns)
+    ([24, 40, 6, 8], "gauss", 1),            # C = 8, hidden width 6 < one chunk + a partial one
 ]
 
 
