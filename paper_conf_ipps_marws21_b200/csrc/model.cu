@@ -621,6 +621,7 @@ static int64_t ld_dz(const hb_worker* w, int l) {
 struct HeadCfg {
   bool ok = false;
   int cmax = 0, cw = 0, cpt = 0, T = 0, rb = 0, rows = 0, grid = 0;
+  int grid_max = 0;  // upper bound of grid over every batch size (sizes the worker's partial buffers)
 };
 static HeadCfg head_shape(const hb_model* m, int b) {
   HeadCfg h;
@@ -650,7 +651,8 @@ static HeadCfg head_shape(const hb_model* m, int b) {
   // every CTA's dW_L / bias partials (C x n floats) are re-read by the update kernel and its
   // prologue (first bulk copies, W_L columns) is a fixed cost: at most ~2 MB of partials (but a CTA
   // per SM), and at least 4 rounds per CTA once the batch exceeds one round per resident CTA
-  int g = std::min(rounds, std::min(cap, std::max(nsm, (int)((2 << 20) / (4L * C * n)))));
+  h.grid_max = std::min(cap, std::max(nsm, (int)((2 << 20) / (4L * C * n))));
+  int g = std::min(rounds, h.grid_max);
   if (rounds > cap) g = std::max(1, std::min(g, rounds / 4));
   h.rows = (rounds + g - 1) / g * h.rb;
   h.grid = (b + h.rows - 1) / h.rows;
@@ -764,15 +766,15 @@ static int alloc_worker(hb_model* m, int max_b, cudaStream_t stream, bool own, h
   const int C = m->layers.back().n_out;
   w->ldc = (int)round_up(C, 4);
   const int mt = (max_b + 127) / 128;
-  const HeadCfg hc = head_shape(m, max_b);  // the head kernel's grid grows with b: max_b bounds it
+  const HeadCfg hc = head_shape(m, max_b);  // hc.grid_max bounds the head kernel's grid at every b
   for (int l = 0; l < L; ++l) {
     float* p = nullptr;
-    const size_t rows = std::max<size_t>((size_t)4 * mt, hc.ok ? (size_t)hc.grid : 0);  // x4: per-quadrant (fused path)
+    const size_t rows = std::max<size_t>((size_t)4 * mt, hc.ok ? (size_t)hc.grid_max : 0);  // x4: per-quadrant (fused path)
     if (cudaMalloc(&p, rows * m->layers[l].n_out * 4) != cudaSuccess)
       return fail_free(fail(HB_ENOMEM, "bias partial alloc"));
     w->bpart.push_back(p);
   }
-  if (hc.ok && cudaMalloc(&w->hws, (size_t)hc.grid * C * (m->layers.back().n_in + 1) * 4) != cudaSuccess)
+  if (hc.ok && cudaMalloc(&w->hws, (size_t)hc.grid_max * C * (m->layers.back().n_in + 1) * 4) != cudaSuccess)
     return fail_free(fail(HB_ENOMEM, "head partial alloc"));
   if (m->prec == HB_PREC_BF16 && cudaMalloc(&w->ws, (size_t)148 * TC_BM * 256 * 4) != cudaSuccess)
     return fail_free(fail(HB_ENOMEM, "split-K workspace alloc"));

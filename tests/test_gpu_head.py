@@ -113,3 +113,19 @@ def test_head_kernel_is_the_default_and_reported_in_profiles():
     hb.prof_enable(False)
     assert prof["head_kernel"]["launches"] >= 1
     assert prof["head_gemm"]["launches"] == 0
+
+
+def test_head_kernel_grid_of_a_smaller_batch_fits_the_worker_buffers():
+    # the head kernel's grid is not monotone in b (at least 4 rounds per CTA only once b exceeds one
+    # round per resident CTA): a worker sized for 3200 rows stepping 2368 rows uses MORE CTAs (148)
+    # than at its max_b (100); its per-CTA partial buffers are sized for the bound over every b
+    dims = [300, 1024, 1024, 2]
+    X, y = dataset("w8a", 2368, seed=5)
+    params = init_params(dims, seed=2)
+    m, w, _ = make(dims, "bf16", 3200)
+    tX, ty = to_device(X, y, "bf16")
+    g, loss = w.step_grads(tX, ty, 2368)
+    dW, db, l_ref = mlp64.grads(params, X.astype(np.float64), y)
+    norm, elem = grad_errors(g, dims, dW, db)
+    assert max(norm) <= 1e-2 and max(elem) <= 1e-2, (norm, elem)
+    assert abs(loss - l_ref) / l_ref <= 1e-2
