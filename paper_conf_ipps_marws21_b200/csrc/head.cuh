@@ -17,14 +17,14 @@
 // dZ_L never leaves the chip, so dW_L is computed from fp32 dZ_L (no bf16 rounding of dZ_L,
 // which DESIGN.md R24 had to split into hi/lo planes for the tensor-core head).
 //
-// Layout: thread t of a T-thread CTA owns the 8-column chunks t, t + T, ... (CPT of them) of
-// every row; rows arrive in shared memory by bulk copies (a ring of stages, see below) and dZ_{L-1}
-// rows leave as coalesced 16-byte-per-lane stores.  A CTA
-// walks a contiguous row range RB rows at a time: partial dot products for RB rows x C classes
-// are reduced across the CTA (warp shuffles, then one shared-memory pass in fixed warp order),
-// RB threads finish the softmax of one row each, and every thread then applies dZ_L of those
-// rows to its columns (dX, dW_L and bias partials).  Deterministic: every reduction has a fixed
-// order independent of timing.
+// Layout: thread t of a T-thread CTA owns the column chunks t, t + T, ... (CPT of them, CW = 8 or 4
+// columns each) of every row; rows arrive in shared memory by bulk copies (a ring of stages, see
+// below) and dZ_{L-1} rows leave as coalesced 16- / 8-byte-per-lane stores.  A CTA walks a
+// contiguous row range RB rows at a time: partial dot products for RB rows x C classes are reduced
+// across the CTA (a transposed warp reduction, then one shared-memory pass in fixed warp order),
+// warp 0 finishes the softmax with one lane per (row, class), and every thread then applies dZ_L
+// of those rows to its columns (dX, dW_L and bias partials).  Deterministic: every reduction has a
+// fixed order independent of timing.  DESIGN.md §5.3.
 #pragma once
 
 #include "common.cuh"
@@ -33,7 +33,6 @@
 namespace hb {
 
 constexpr int HEAD_MAX_C = 8;
-constexpr int HEAD_MAX_T = 512;
 
 struct HeadArgs {
   const __nv_bfloat16* H;  // H_{L-1} [b x ld] bf16 (row 0 = the batch's first row)
