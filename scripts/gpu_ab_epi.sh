@@ -2,8 +2,8 @@
 # A/B: 8 vs 16 epilogue warps in the tcgen05 GEMM (variant library via HB_LIB): GPU tests on the
 # variant, then bench lines of both builds
 mkdir -p gpurun_out/ab; O=gpurun_out/ab
-V=paper_conf_ipps_marws21_b200/variants/libhogbatch_epi16.so
-HB_LIB=$V timeout -s KILL 1200 python -m pytest tests -m gpu -q -x --timeout 600 > $O/tests_epi16.log 2>&1; tail -2 $O/tests_epi16.log
+V=${VARIANT:-paper_conf_ipps_marws21_b200/variants/libhogbatch_epi16.so}
+[ -z "$NO_TESTS" ] && HB_LIB=$V timeout -s KILL 1200 python -m pytest tests -m gpu -q -x --timeout 600 > $O/tests_epi16.log 2>&1; tail -2 $O/tests_epi16.log
 line() { python - "$1" <<'PY'
 import json, sys
 d = json.loads(open("gpurun_out/ab/b.json").read().strip().splitlines()[-1])
