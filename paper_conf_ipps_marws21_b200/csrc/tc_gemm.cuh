@@ -173,15 +173,23 @@ __device__ __forceinline__ void bias_reduce_update(const EpiArgs& ep, int lo, in
 // and 32 x 82 tiles) the traffic minimum is near m = 17.  GROUP_M = 16 measured 1.60 GB of DRAM
 // traffic per layer-1 wgrad+SGD launch against 2.08 GB at 8, and +1.1 % C4 samples/s
 // (profiles/r02_group_m.txt).
+// CTA pairs have ~74 pair tiles in flight, so the same model gives A re-reads tiles_n*m/74 and B
+// re-reads tiles_mp/m per group of m PAIR rows: the minimum for both C4 layer-1 GEMMs (32 x 16 and
+// 16 x 82 pair tiles) is near m = 8.6, i.e. 8 pair rows (16 row tiles, as before the pairs).
 #ifndef HB_GROUP_M
 #define HB_GROUP_M 16
 #endif
+#ifndef HB_GROUP_M_PAIR
+#define HB_GROUP_M_PAIR 8
+#endif
 constexpr int TC_GROUP_M = HB_GROUP_M;
+constexpr int TC_GROUP_M_PAIR = HB_GROUP_M_PAIR;
+template <int GROUP>
 __device__ __forceinline__ void tile_coords(int t, int tiles_m, int tiles_n, int& m_tile, int& n_tile) {
-  const int per_group = TC_GROUP_M * tiles_n;
+  const int per_group = GROUP * tiles_n;
   const int g = t / per_group;
-  const int first_m = g * TC_GROUP_M;
-  const int gm = min(tiles_m - first_m, TC_GROUP_M);
+  const int first_m = g * GROUP;
+  const int gm = min(tiles_m - first_m, GROUP);
   const int r = t - g * per_group;
   m_tile = first_m + r % gm;
   n_tile = r / gm;
@@ -709,10 +717,10 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
       n_tile = blockIdx.y;
     } else if (PAIR) {
       int mp;
-      tile_coords(t, tiles_mp, tiles_n, mp, n_tile);
+      tile_coords<TC_GROUP_M_PAIR>(t, tiles_mp, tiles_n, mp, n_tile);
       m_tile = 2 * mp + (int)half;
     } else {
-      tile_coords(t, tiles_m, tiles_n, m_tile, n_tile);
+      tile_coords<TC_GROUP_M>(t, tiles_m, tiles_n, m_tile, n_tile);
     }
   };
 
