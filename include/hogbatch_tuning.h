@@ -19,6 +19,10 @@ extern "C" {
 /* tuning only: mean device microseconds of one tensor-core GEMM launch of the given kind
  * (0 forward+sigmoid, 1 dgrad+sigma', 2 wgrad+SGD) and shape on zero-filled scratch buffers */
 int hb_bench_gemm(int32_t kind, int32_t M, int32_t N, int32_t K, int32_t iters, float* us_out);
+/* kind: 0 forward, 1 dX, 2 dW + fused SGD, 3 dW storing the fp32 gradient (unfused baseline).
+ * hb_bench_sgd_apply: the unfused SGD update alone (W -= lr G, shadow rewritten) over n fp32
+ * weights (n % 4 == 0), mean device microseconds per launch. */
+int hb_bench_sgd_apply(int64_t n, int32_t iters, float* us_out);
 /* tuning only: per-CTA phase timestamps (8 globaltimer ns values per CTA, cap entries) of one launch */
 /* tuning only: hb_rc_trace(NULL, cap) arms per-step globaltimer stamps (10 per CTA per step, 24 steps
  * per CTA) in later fused row-block launches; hb_rc_trace(host, cap) reads the last launch's */

@@ -35,7 +35,7 @@ EXPORTS = ("hb_last_error", "hb_abi_version", "hb_device_ok", "mlp_create", "mlp
            "mlp_worker_create_nested", "hb_coord_create", "hb_coord_destroy", "hb_coord_reset",
            "hb_coord_schedule", "hb_coord_idle", "mlp_attach_peers", "mlp_ipc_handle", "mlp_attach_ipc_peers")
 # tuning build only (include/hogbatch_tuning.h): not exported by the product library
-TUNING_EXPORTS = ("hb_bench_gemm", "hb_bench_gemm_phases", "hb_rc_trace", "hb_bench_step")
+TUNING_EXPORTS = ("hb_bench_gemm", "hb_bench_gemm_phases", "hb_rc_trace", "hb_bench_step", "hb_bench_sgd_apply")
 PROF_LAYERS = 16
 PROF_CLASSES = ("fwd_gemm", "head_gemm", "softmax_xent", "dgrad_gemm", "wgrad_sgd_gemm", "bias_sgd", "other",
                 "rowchain", "step_kernel", "head_kernel")
@@ -134,6 +134,7 @@ def load():
         "hb_prof_enable": ([I32], C.c_int),
         "hb_rc_trace": ([VP, I64], C.c_int),
         "hb_bench_step": ([VP, VP, I64, VP, I32, I32, I32, P(F)], C.c_int),
+        "hb_bench_sgd_apply": ([I64, I32, P(F)], C.c_int),
         "hb_prof_read": ([P(ProfEntry), I32, I32], C.c_int),
         "hb_bench_gemm": ([I32, I32, I32, I32, I32, P(F)], C.c_int),
         "hb_bench_gemm_phases": ([I32, I32, I32, I32, P(C.c_uint64), I64], C.c_int),

@@ -2175,6 +2175,64 @@ static int bench_gemm_impl(int32_t kind, int32_t M, int32_t N, int32_t K, int32_
 int hb_bench_gemm(int32_t kind, int32_t M, int32_t N, int32_t K, int32_t iters, float* us_out) {
   return bench_gemm_impl(kind, M, N, K, iters, us_out, nullptr, 0);
 }
+
+// Unfused SGD baseline: W -= lr * G over n fp32 weights with the bf16 shadow rewritten,
+// G read from HBM — 14 bytes per weight (W and G read, W and shadow written)
+static __global__ void sgd_apply_kernel(float* __restrict__ W, const float* __restrict__ G, __nv_bfloat16* __restrict__ Sh,
+                                        int64_t n4, float lr) {
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n4; i += (int64_t)gridDim.x * blockDim.x) {
+    float4 w = reinterpret_cast<float4*>(W)[i];
+    const float4 g = __ldcs(reinterpret_cast<const float4*>(G) + i);
+    w.x += __fmul_rn(-lr, g.x);
+    w.y += __fmul_rn(-lr, g.y);
+    w.z += __fmul_rn(-lr, g.z);
+    w.w += __fmul_rn(-lr, g.w);
+    reinterpret_cast<float4*>(W)[i] = w;
+    reinterpret_cast<uint2*>(Sh)[i] = make_uint2(pack_bf16x2(w.x, w.y), pack_bf16x2(w.z, w.w));
+  }
+}
+// tuning only: mean device microseconds of sgd_apply_kernel over n weights (graph of iters launches)
+int hb_bench_sgd_apply(int64_t n, int32_t iters, float* us_out) {
+  HB_CHECK_ARG(us_out && n > 0 && n % 4 == 0 && iters > 0, "bad args");
+  float *W = nullptr, *G = nullptr;
+  __nv_bfloat16* Sh = nullptr;
+  if (cudaMalloc(&W, n * 4) || cudaMalloc(&G, n * 4) || cudaMalloc(&Sh, n * 2)) return fail(HB_ENOMEM, "bench alloc");
+  cudaMemset(W, 0, n * 4);
+  cudaMemset(G, 0, n * 4);
+  cudaStream_t s;
+  cudaStreamCreate(&s);
+  int nsm = 148;
+  cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, 0);
+  const int grid = nsm * 8;
+  sgd_apply_kernel<<<grid, 256, 0, s>>>(W, G, Sh, n / 4, 0.f);
+  cudaGraph_t g = nullptr;
+  cudaGraphExec_t ge = nullptr;
+  cudaStreamBeginCapture(s, cudaStreamCaptureModeThreadLocal);
+  for (int i = 0; i < iters; ++i) sgd_apply_kernel<<<grid, 256, 0, s>>>(W, G, Sh, n / 4, 0.f);
+  cudaStreamEndCapture(s, &g);
+  cudaGraphInstantiate(&ge, g, 0);
+  cudaGraphLaunch(ge, s);
+  cudaEvent_t e0, e1;
+  cudaEventCreate(&e0);
+  cudaEventCreate(&e1);
+  cudaEventRecord(e0, s);
+  cudaGraphLaunch(ge, s);
+  cudaEventRecord(e1, s);
+  cudaError_t ce = cudaStreamSynchronize(s);
+  float ms = 0.f;
+  cudaEventElapsedTime(&ms, e0, e1);
+  *us_out = ms * 1000.f / iters;
+  cudaEventDestroy(e0);
+  cudaEventDestroy(e1);
+  cudaGraphExecDestroy(ge);
+  cudaGraphDestroy(g);
+  cudaStreamDestroy(s);
+  cudaFree(W);
+  cudaFree(G);
+  cudaFree(Sh);
+  if (ce != cudaSuccess) return fail(HB_ECUDA, std::string("bench sgd apply: ") + cudaGetErrorString(ce));
+  return HB_OK;
+}
 // tuning only: per-CTA phase timestamps of one launch (8 globaltimer values per CTA)
 int hb_bench_gemm_phases(int32_t kind, int32_t M, int32_t N, int32_t K, unsigned long long* host_ts, int64_t cap) {
   float us = 0.f;
@@ -2183,9 +2241,11 @@ int hb_bench_gemm_phases(int32_t kind, int32_t M, int32_t N, int32_t K, unsigned
 static int bench_gemm_impl(int32_t kind, int32_t M, int32_t N, int32_t K, int32_t iters, float* us_out,
                            unsigned long long* host_ts, int64_t cap) {
   HB_CHECK_ARG(us_out && M > 0 && N > 0 && K > 0 && iters > 0 && kind >= 0 && kind <= 3, "bad args");
-  const int64_t lda = round_up(kind == 2 ? M : K, 8), ldb = round_up(kind == 0 ? K : N, 8);
+  // kind 0 forward, 1 dX, 2 dW + fused SGD, 3 dW storing the fp32 gradient (the unfused baseline)
+  const bool dw = kind >= 2;
+  const int64_t lda = round_up(dw ? M : K, 8), ldb = round_up(kind == 0 ? K : N, 8);
   const int64_t ldo = round_up(N, 8);
-  const int64_t arows = kind == 2 ? K : M, brows = kind == 0 ? N : K;
+  const int64_t arows = dw ? K : M, brows = kind == 0 ? N : K;
   void *A = nullptr, *B = nullptr, *O = nullptr, *S = nullptr;
   float *W = nullptr, *bias = nullptr, *ws = nullptr, *bp = nullptr;
   __nv_bfloat16* Wsh = nullptr;
@@ -2225,10 +2285,14 @@ static int bench_gemm_impl(int32_t kind, int32_t M, int32_t N, int32_t K, int32_
     ep.bpart_out = bp;
     ep.ldp = N;
   } else {
-    epi = EPI_WGRAD_SGD;
+    epi = kind == 3 ? EPI_WGRAD_STORE : EPI_WGRAD_SGD;
     a_mn = b_mn = true;
     ep.master = W;
     ep.shadow = Wsh;
+    if (kind == 3) {
+      ep.out0 = W;  // dW [M x ldo] fp32
+      ep.bias_grad = bias;
+    }
     ep.ldw = ldo;
     ep.lr = 0.f;
     ep.ws = ws;
