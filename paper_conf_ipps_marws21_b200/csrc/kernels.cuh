@@ -268,6 +268,21 @@ static __global__ void densify_csr_kernel(const int64_t* __restrict__ indptr, co
   }
 }
 
+// the inverse scatter: zeros at the nonzero positions of rows [r0, r1) of a CSR structure (the
+// previous dataset staged into X), so re-densifying a same-shape dataset needs no full memset
+template <typename T>
+static __global__ void zero_csr_kernel(const int64_t* __restrict__ indptr, const int32_t* __restrict__ indices,
+                                       int64_t r0, int64_t r1, int64_t n_cols, T* X, int64_t ldx) {
+  const int64_t r = r0 + ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) / 32;
+  const int lane = threadIdx.x & 31;
+  if (r >= r1) return;
+  T* row = X + r * ldx;
+  for (int64_t k = indptr[r] + lane; k < indptr[r + 1]; k += 32) {
+    const int32_t c = indices[k];
+    if (c >= 0 && c < n_cols) row[c] = T(0.f);
+  }
+}
+
 // HB_CHECK=labels (hb_policy.check_labels): flag any label outside [0, C)
 static __global__ void check_labels_kernel(const int32_t* __restrict__ y, int64_t n, int C, int* bad) {
   int any = 0;

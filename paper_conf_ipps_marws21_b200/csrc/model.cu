@@ -1700,9 +1700,20 @@ int mlp_destroy(hb_model* m) {
 
 namespace hb {
 int densify_csr_rows(const int64_t* indptr, const int32_t* indices, const void* vals, int xdt, int64_t r0, int64_t r1,
-                     int64_t n_cols, void* X, int64_t ldx, cudaStream_t s, int* bad) {
+                     int64_t n_cols, void* X, int64_t ldx, cudaStream_t s, int* bad, bool zero_first) {
   const size_t es = xdt == HB_BF16 ? 2 : 4;
-  HB_CUDA_TRY(cudaMemsetAsync(static_cast<char*>(X) + (size_t)r0 * ldx * es, 0, (size_t)(r1 - r0) * ldx * es, s));
+  if (zero_first)
+    HB_CUDA_TRY(cudaMemsetAsync(static_cast<char*>(X) + (size_t)r0 * ldx * es, 0, (size_t)(r1 - r0) * ldx * es, s));
+  if (!vals) {  // zero the nonzeros of rows [r0, r1) only (the rest of the rows is already zero)
+    const unsigned blocks0 = (unsigned)(((r1 - r0) * 32 + 255) / 256);
+    if (xdt == HB_BF16)
+      zero_csr_kernel<__nv_bfloat16><<<blocks0, 256, 0, s>>>(indptr, indices, r0, r1, n_cols, static_cast<__nv_bfloat16*>(X), ldx);
+    else
+      zero_csr_kernel<float><<<blocks0, 256, 0, s>>>(indptr, indices, r0, r1, n_cols, static_cast<float*>(X), ldx);
+    HB_CUDA_TRY(cudaGetLastError());
+    g_launches.fetch_add(1, std::memory_order_relaxed);
+    return HB_OK;
+  }
   const int64_t warps = r1 - r0;
   const unsigned blocks = (unsigned)((warps * 32 + 255) / 256);
   if (xdt == HB_BF16)

@@ -84,6 +84,14 @@ struct hb_model {
   // stream and one event per staged chunk of rows
   void* stage_x = nullptr;
   size_t stage_x_cap = 0;
+  // stage_x holds exactly the densification (zeros elsewhere) of the host CSR dataset whose
+  // structure is still in csr_ptr / csr_idx: the next CSR staging of the same shape zeroes only
+  // those nonzeros instead of the whole dense buffer
+  struct {
+    bool valid = false;
+    int64_t n = 0, ldx = 0, n_cols = 0;
+    int xdt = 0;
+  } csr_dense;
   int32_t* stage_y = nullptr;
   size_t stage_y_cap = 0;
   cudaStream_t copy_stream = nullptr;
@@ -154,7 +162,7 @@ int clone_model(hb_model* m, hb_model** out);
 // zero rows [r0, r1) of the dense X [.. x ldx] (dtype xdt) and scatter the CSR rows into them on s;
 // *bad (device int) is set if a column index is outside [0, n_cols)
 int densify_csr_rows(const int64_t* indptr, const int32_t* indices, const void* vals, int xdt, int64_t r0, int64_t r1,
-                     int64_t n_cols, void* X, int64_t ldx, cudaStream_t s, int* bad);
+                     int64_t n_cols, void* X, int64_t ldx, cudaStream_t s, int* bad, bool zero_first = true);
 // One SGD step.  X / y: the batch's first row, or (d_off != nullptr, tensor-core path) the
 // dataset base with the batch's first row read from *d_off on the device.  x_rows = rows of X.
 int run_step(hb_worker* w, const void* X, int64_t ldx, int32_t xdt, int64_t x_rows, const int32_t* y,

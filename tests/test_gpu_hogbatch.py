@@ -220,6 +220,41 @@ def test_csr_dataset_is_densified_and_bitwise_equal_to_dense(where):
         hb.hogbatch_run([w], pol, csr, torch.from_numpy(y.astype(np.int32)), epochs=1)
 
 
+def test_csr_restaging_zeroes_only_the_previous_nonzeros():
+    # a second host CSR dataset of the same shape re-uses the dense staging buffer: only the first
+    # dataset's nonzeros are zeroed (through its structure, still on the device), no full memset;
+    # the run on dataset B after dataset A equals, bit for bit, a run on B's dense device copy
+    from synth import sparse_like
+    _gpu()
+    dims, N = [2000, 256, 2], 3000
+    t = lambda a, dt: torch.from_numpy(np.ascontiguousarray(a)).to(dt)
+    data = []
+    for seed in (3, 4):
+        (indptr, indices, vals), y = sparse_like(N, 2000, 51.5, 0.31, False, seed=seed)
+        X = np.zeros((N, 2000), np.float32)
+        X[np.repeat(np.arange(N), np.diff(indptr)), indices] = vals
+        csr = hb.CSR(t(indptr.astype(np.int64), torch.int64).pin_memory(), t(indices, torch.int32).pin_memory(),
+                     t(vals, torch.bfloat16).pin_memory(), 2000)
+        data.append((X, y, csr, t(y.astype(np.int32), torch.int32).pin_memory()))
+    pol = hb.Policy(kind=hb.HB_MINIBATCH, workers=[hb.WorkerSpec(256, 256, 256)], eta0=0.1, b0=32, eval_loss=True)
+    out = []
+    for fmt in ("dense", "csr"):
+        m = hb.MLP(dims)
+        m.set_option("stage_rows", 700)
+        w = hb.Worker(m, 256)
+        if fmt == "csr":  # stage dataset A first (its nonzeros stay in the dense buffer)
+            hb.hogbatch_run([w], pol, data[0][2], data[0][3], epochs=1)
+        m.set_params(params_to_flat(init_params(dims)))
+        if fmt == "dense":
+            tX, ty = to_device(data[1][0], data[1][1])
+            st = hb.hogbatch_run([w], pol, tX, ty, epochs=2)
+        else:
+            st = hb.hogbatch_run([w], pol, data[1][2], data[1][3], epochs=2)
+        out.append((m.get_params(), st["epoch_loss"]))
+    assert np.array_equal(out[0][0], out[1][0])
+    assert out[0][1] == out[1][1]
+
+
 def test_host_dataset_mixed_pointers_rejected():
     X, y, m, params, tX, ty = setup([54, 64, 7], "bf16", 256, 1024)
     w = hb.Worker(m, 256)
