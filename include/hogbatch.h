@@ -203,8 +203,8 @@ int mlp_fused_path(const hb_model* m, int32_t batch, int32_t* cluster_size);
  *   HB_OPT_GRAPHS           1 = hogbatch_run replays one CUDA graph per (batch size, lr) (default)
  *   HB_OPT_INFLIGHT         steps a worker may have enqueued before the oldest completes in
  *                           hogbatch_run (1..4; 0 = auto: 2 for a single worker, else 1, R23)
- *   HB_OPT_STAGE_ROWS       rows per H2D staging chunk of a host dataset (0 = auto: <= 32768 rows
- *                           and <= 32 MB)
+ *   HB_OPT_STAGE_ROWS       rows per H2D staging chunk of a host dataset (0 = auto: chunks growing
+ *                           from 4096 rows by doubling, each <= 32768 rows and <= 32 MB)
  *   HB_OPT_UPDATE           HB_UPDATE_HOGWILD (plain read-modify-write of the shared model, Hogwild
  *                           [L128, L170]; default) or HB_UPDATE_ATOMIC (the dW epilogue adds -lr*dW
  *                           with atomic adds: no concurrent update is lost)
