@@ -21,7 +21,7 @@ timeout -s KILL 900 ncu --set full --clock-control none --import-source on -k re
   python scripts/c4_step.py 1 > $O/ncu_c4.log 2>&1; echo "ncu full rc=$?"
 # summarise on the box (gpurun copies back <= 64 MiB): per-launch summary, raw metrics, details page of
 # the longest launch; the .ncu-rep itself stays behind
-python scripts/ncu_traffic.py $O/c4_step.ncu-rep c4 > $O/ncu_c4_summary.txt 2>&1; cp profiles/ncu_traffic.json $O/ 2>/dev/null
+python scripts/ncu_traffic.py $O/c4_step.ncu-rep realsim > $O/ncu_c4_summary.txt 2>&1; cp profiles/ncu_traffic.json $O/ 2>/dev/null
 ncu -i $O/c4_step.ncu-rep --page raw --csv > $O/ncu_c4_raw.csv 2>/dev/null
 ncu -i $O/c4_step.ncu-rep --page details --print-details all -k regex:tc_gemm_kernel --launch-skip 0 --launch-count 1 > $O/ncu_c4_l1fwd_details.txt 2>/dev/null
 ncu -i $O/c4_step.ncu-rep --page details > $O/ncu_c4_details.txt 2>/dev/null
