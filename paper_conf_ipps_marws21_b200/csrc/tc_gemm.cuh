@@ -44,8 +44,12 @@ constexpr int TC_THREADS = 128 + TC_EPI_THREADS;   // 4 control warps + the epil
 // The tile is written in 64-column chunks through TWO staging buffers: chunk j is staged while the
 // bulk stores of chunk j-1 drain, so the staging costs 2 x NOUT x 16 KB whatever BN (B200, C3
 // 8192x1024x1024: 256-wide tiles with a whole-tile staged epilogue were epilogue-bound).
+// CTA pairs load half of B per stage, so their ring keeps 5 stages next to two H staging buffers:
+// measured on B200 (scripts/gpu_ab_nbuf.sh, C4, alternating reps) 2.123 / 2.128 M samples/s against
+// 2.093 / 2.106 M with one buffer and 6 stages; staging sigma' as well (HB_PAIR_NOUT = 2, 4 stages)
+// measured slower (2.077 / 2.066 M)
 #ifndef HB_PAIR_NBUF
-#define HB_PAIR_NBUF 1
+#define HB_PAIR_NBUF 2
 #endif
 #ifndef HB_PAIR_NOUT
 #define HB_PAIR_NOUT 1
