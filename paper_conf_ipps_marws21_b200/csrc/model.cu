@@ -410,6 +410,9 @@ struct SkPlanEntry {
   int layer;
 };
 static thread_local std::vector<SkPlanEntry>* g_plan = nullptr;
+// Set while a step graph is captured with a training-loss accumulator: the step adds the sum of its
+// row losses into *g_loss_acc on a side stream (off the step's critical path, before its join)
+static thread_local double* g_loss_acc = nullptr;
 
 static int gemm_tc_p(int epi, bool a_mn, bool b_mn, int M, int N, int K, TcOp A, TcOp B, const EpiArgs& ep,
                      cudaStream_t s) {
@@ -1218,6 +1221,7 @@ static int run_step_rowchain(hb_worker* w, const RcCfg& c, const void* X, int64_
       int rc = launch_wgrad(w, l, X, ldx, x_rows, d_off, b, lr, grads_only, s, w->ws_l[l], 4 * ((b + 127) / 128));
       if (rc) return rc;
     }
+    if (g_loss_acc) sum_rows_into(w, b, g_loss_acc, s, true);
     return HB_OK;
   }
   HB_CUDA_TRY(cudaEventRecord(w->ev_chain, s));
@@ -1237,6 +1241,7 @@ static int run_step_rowchain(hb_worker* w, const RcCfg& c, const void* X, int64_
                           4 * ((b + 127) / 128),  // per-quadrant bias partials of the chain
                           wide ? bn : 0, sp);  // the small head keeps its BN 16 tiles, 4 splits
     if (rc) return rc;
+    if (l == L - 1 && g_loss_acc) sum_rows_into(w, b, g_loss_acc, w->sdw[l], true);  // row losses of the chain
     HB_CUDA_TRY(cudaEventRecord(w->ev_dw[l], w->sdw[l]));
   }
   for (int l = L - 1; l >= 0; --l) HB_CUDA_TRY(cudaStreamWaitEvent(s, w->ev_dw[l], 0));
@@ -1350,7 +1355,11 @@ static int run_step_tc(hb_worker* w, const void* X, int64_t ldx, int64_t x_rows,
     const RcCfg c = rowchain_cfg(m, b);
     if (c.ok && !w->sdw.empty()) return run_step_rowchain(w, c, X, ldx, x_rows, y, d_off, b, lr, grads_only, s);
   }
-  if (step_kernel_ok(w, b)) return run_step_persistent(w, X, ldx, x_rows, y, d_off, b, lr, grads_only, s);
+  if (step_kernel_ok(w, b)) {
+    int rc = run_step_persistent(w, X, ldx, x_rows, y, d_off, b, lr, grads_only, s);
+    if (!rc && g_loss_acc) sum_rows_into(w, b, g_loss_acc, s, true);
+    return rc;
+  }
   return step_gemms(w, X, ldx, x_rows, y, d_off, b, lr, grads_only, s, m->opt_bwd_overlap && w->s2);
 }
 
@@ -1366,6 +1375,13 @@ static int step_gemms(hb_worker* w, const void* X, int64_t ldx, int64_t x_rows, 
   // dW_l only has to follow dX_l (the last reader of W_l): it runs on the worker's second stream,
   // overlapping dX_{l-1} (HB_OPT_BWD_OVERLAP = 0 keeps everything on one stream)
   cudaStream_t s2 = overlap ? w->s2 : s;
+  if (g_loss_acc && !g_plan) {  // the step's row losses into the training-loss accumulator, on s2
+    if (s2 != s) {
+      HB_CUDA_TRY(cudaEventRecord(w->ev_join2, s));
+      HB_CUDA_TRY(cudaStreamWaitEvent(s2, w->ev_join2, 0));
+    }
+    sum_rows_into(w, b, g_loss_acc, s2, true);
+  }
   for (int l = L - 1; l >= 0; --l) {
     const Layer& Ly = m->layers[l];
     TcOp dZl{w->dZ[l], ld_dz(w, l), b, nullptr};
@@ -1419,7 +1435,7 @@ void clear_graphs(hb_worker* w) {
 }
 
 int step_graph(hb_worker* w, const void* X, int64_t ldx, int64_t x_rows, const int32_t* y, int64_t off, int b,
-               float lr) {
+               float lr, double* loss_acc) {
   if (w->g_X != X || w->g_y != y || w->g_ldx != ldx || w->g_rows != x_rows) {
     clear_graphs(w);
     w->g_X = X;
@@ -1433,14 +1449,16 @@ int step_graph(hb_worker* w, const void* X, int64_t ldx, int64_t x_rows, const i
   // word when it starts, so up to HB_MAX_INFLIGHT replays of this worker may be enqueued
   const int slot = w->slot;
   w->slot = (w->slot + 1) % HB_MAX_INFLIGHT;
-  auto key = std::make_tuple(b, lrbits, slot);
+  auto key = std::make_tuple(b, lrbits, slot, (const double*)loss_acc);
   auto it = w->graphs.find(key);
   if (it == w->graphs.end()) {
     cudaStream_t s = w->stream;
     const int64_t l0 = g_launches.load();
     HB_CUDA_TRY(cudaStreamBeginCapture(s, cudaStreamCaptureModeThreadLocal));
     cudaMemcpyAsync(w->d_off, w->h_off + slot, sizeof(int), cudaMemcpyHostToDevice, s);
+    g_loss_acc = loss_acc;
     int rc = run_step(w, X, ldx, HB_BF16, x_rows, y, w->d_off, b, lr, false, s);
+    g_loss_acc = nullptr;
     cudaGraph_t graph = nullptr;
     cudaError_t ce = cudaStreamEndCapture(s, &graph);
     cudaStreamCaptureStatus cs = cudaStreamCaptureStatusNone;
@@ -1474,6 +1492,8 @@ int worker_execute(hb_worker* w, const void* X, int64_t ldx, int32_t xdt, int64_
   const size_t xes = xdt == HB_BF16 ? 2 : 4;
   auto xrow = [&](int64_t o) { return static_cast<const char*>(X) + o * ldx * xes; };
   if (w->subs.empty()) {
+    if (graphs && loss_dst && accumulate)  // the step graph accumulates its own row losses (side stream)
+      return step_graph(w, X, ldx, x_rows, y, off, b, lr, loss_dst);
     int rc = graphs ? step_graph(w, X, ldx, x_rows, y, off, b, lr)
                     : run_step(w, xrow(off), ldx, xdt, b, y + off, nullptr, b, lr, false, w->stream);
     if (!rc && loss_dst) sum_rows_into(w, b, loss_dst, w->stream, accumulate);

@@ -132,7 +132,7 @@ struct hb_worker {
     cudaGraphExec_t exec = nullptr;
     int launches = 0;
   };
-  std::map<std::tuple<int, uint32_t, int>, Graph> graphs;  // (b, lr bits, slot)
+  std::map<std::tuple<int, uint32_t, int, const double*>, Graph> graphs;  // (b, lr bits, slot, loss accumulator)
   const void* g_X = nullptr;
   const void* g_y = nullptr;
   int64_t g_ldx = 0, g_rows = 0;
@@ -170,7 +170,7 @@ int run_step(hb_worker* w, const void* X, int64_t ldx, int32_t xdt, int64_t x_ro
 // One SGD step replayed from a CUDA graph captured for (b, lr) on the dataset (X, y): the
 // batch's row offset is copied from pinned host memory by the graph's first node.
 int step_graph(hb_worker* w, const void* X, int64_t ldx, int64_t x_rows, const int32_t* y, int64_t off, int b,
-               float lr);
+               float lr, double* loss_acc = nullptr);
 void clear_graphs(hb_worker* w);
 // One ExecuteWork(B) of a worker on rows [off, off + b) of the dataset (X, y with x_rows rows):
 // a plain worker runs one SGD step; a nested worker splits B into its t sub-batches (the first
